@@ -1,0 +1,299 @@
+#!/usr/bin/env python
+"""Benchmark of the hot path: pack + unpack of the paper's lower-triangular
+matrix (BASELINE.json configs[1]: 4096x4096 f64 lower triangle via
+MPI_Type_indexed, PAPER.md [L22:c2839 §5.1]) on B200, one rank per GPU.
+
+One step = dt_pack of the whole triangle from the column-major matrix into a
+contiguous buffer + dt_unpack of it into a second matrix (all §8(a) rows that
+run on one GPU: S3 position resolve, S4 work split, S5 pack, S6 unpack; S1/S2
+construct + commit happen once, before timing, as the paper's cached DEVs
+[L24:c2714]).  Metric (BASELINE.json): pack/unpack GB/s counting payload bytes
+read + written, i.e. 2*payload per kernel, reported against the measured HBM
+copy peak.  At N>1 every rank runs the same step on its own matrices (weak
+scaling, no data-path collective; the transfer path is `--workload c3`).
+
+L2 hygiene: a 2xL2 scratch buffer is rewritten before every timed kernel, and
+only the pack/unpack kernels themselves are inside the CUDA-event intervals.
+
+`--impl reference` times the CPU oracle (oracle/) on the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "pack/unpack GB/s vs HBM peak; GPU↔GPU non-contig transfer GB/s vs NVLink"
+UNIT = "GB/s"
+WORKLOAD = "C2: lower triangle of 4096x4096 f64 (MPI_Type_indexed, 4096 blocks of 8..32768 B), pack+unpack"
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """Samples SM clock and clock-event reasons with NVML during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, index):
+        self.samples, self.reasons, self.max_mhz = [], 0, None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:  # noqa: BLE001
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            self.sample()
+            time.sleep(0.01)
+
+    def sample(self):
+        if self.nv is None:
+            return
+        try:
+            self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+            self.reasons |= self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        except Exception:  # noqa: BLE001
+            pass
+
+    def __enter__(self):
+        self.t = threading.Thread(target=self._run, daemon=True)
+        self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self.t.join()
+        self.sample()
+
+    def summary(self):
+        rs = [n for b, n in self.REASONS.items() if self.reasons & b and n != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": rs, "samples": len(self.samples)}
+
+
+def dist_init():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as tdist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        import torch
+        torch.cuda.set_device(local)
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    return ws, rank, local
+
+
+def c2_buffers(torch, n=4096):
+    from workloads import c2_lower_triangle, fill_bytes, seed_for
+    rec, org, parent = c2_lower_triangle(n)
+    src_h = fill_bytes(parent, seed_for(2))
+    return rec, org, parent, src_h
+
+
+def time_oracle_c2(seconds=10.0, threads=1):
+    """CPU oracle (as it stands) on the C2 workload: pack + unpack per rep."""
+    import numpy as np
+
+    import oracle
+    from workloads import c2_lower_triangle, fill_bytes, seed_for
+    rec, org, parent = c2_lower_triangle(4096)
+    ot = oracle.from_recipe(rec)
+    src = fill_bytes(parent, seed_for(2))
+    dst = np.full(parent, 0xA5, dtype=np.uint8)
+    payload = ot.size
+    reps, t0 = 0, time.perf_counter()
+    tp = tu = 0.0
+    while True:
+        a = time.perf_counter()
+        packed = oracle.pack(ot, 1, src, org, threads=threads)
+        b = time.perf_counter()
+        oracle.unpack(ot, 1, packed, dst, org, threads=threads)
+        c = time.perf_counter()
+        tp += b - a
+        tu += c - b
+        reps += 1
+        if c - t0 >= seconds:
+            break
+    value = 4.0 * payload * reps / (tp + tu) / 1e9
+    return {"value": round(value, 4), "unit": UNIT, "cores": threads, "kind": "oracle",
+            "sample": f"{reps} x (pack+unpack of the full C2 triangle, {payload} B payload), "
+                      f"{tp + tu:.1f} s wall, single process"}, reps, tp + tu
+
+
+def run_reference(args):
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if ws > 1 and rank != 0:
+        return
+    secs = max(3.0, min(60.0, 0.5 * (args.steps + args.warmup)))
+    cb, reps, wall = time_oracle_c2(seconds=secs)
+    line = {"impl": "reference", "metric": METRIC, "value": cb["value"], "unit": UNIT, "n_gpus": args.gpus,
+            "steps": reps, "warmup": 0, "ms_per_step": round(1e3 * wall / reps, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
+            "config": {"workload": WORKLOAD, "impl": "CPU oracle (oracle/oracle.c typemap walk), 1 thread"},
+            "cpu_baseline": cb,
+            "e2e": {"value": cb["value"], "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    ws, rank, local = dist_init()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    rec, org, parent, src_h = c2_buffers(torch)
+    t = dt.from_recipe(rec).commit()
+    payload = t.size
+    src = torch.from_numpy(src_h).to(dev)
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8, device=dev)
+    packed = torch.empty(payload, dtype=torch.uint8, device=dev)
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    flush = torch.empty(2 * l2, dtype=torch.uint8, device=dev)
+    s = torch.cuda.current_stream()
+
+    def step(evs=None):
+        flush.fill_(1)
+        if evs: evs[0].record(s)
+        dt.pack(t, 1, src, packed, origin_offset=org, stream=s)
+        if evs: evs[1].record(s)
+        flush.fill_(2)
+        if evs: evs[2].record(s)
+        dt.unpack(t, 1, packed, dst, origin_offset=org, stream=s)
+        if evs: evs[3].record(s)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    # correctness spot check of this exact launch configuration against the oracle-free closed form
+    M = src_h.view(np.float64).reshape(4096, 4096)
+    exp_head = M[np.triu_indices(4096)][:4096].view(np.uint8)
+    assert np.array_equal(packed[: exp_head.size].cpu().numpy(), exp_head), "packed stream mismatch"
+
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(args.steps)]
+    w0, w1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if ws > 1:
+        import torch.distributed as tdist
+        tdist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        w0.record(s)
+        for i in range(args.steps):
+            step(evs[i])
+        w1.record(s)
+        torch.cuda.synchronize()
+    tpk = [e[0].elapsed_time(e[1]) for e in evs]
+    tup = [e[2].elapsed_time(e[3]) for e in evs]
+    kern_ms = sum(tpk) + sum(tup)
+    wall_ms = w0.elapsed_time(w1)
+    if ws > 1:
+        import torch.distributed as tdist
+        x = torch.tensor([kern_ms, wall_ms], dtype=torch.float64, device=dev)
+        tdist.all_reduce(x, op=tdist.ReduceOp.MAX)
+        kern_ms, wall_ms = float(x[0]), float(x[1])
+    bytes_per_step = 4 * payload  # pack R+W + unpack R+W
+    value = ws * bytes_per_step * args.steps / (kern_ms * 1e-3) / 1e9
+    peak, peak_src = load_peaks()
+    avg_pack = statistics.mean(tpk)
+    avg_unpack = statistics.mean(tup)
+    dom_ms, dom = (avg_pack, "pack") if avg_pack >= avg_unpack else (avg_unpack, "unpack")
+    achieved = 2 * payload / (dom_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(f"c2_{dom}")
+    e2e = run_e2e(args, t, src_h, org, parent, payload, dev) if rank == 0 else None
+    line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(kern_ms / args.steps, 5), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
+            "config": {"workload": WORKLOAD, "payload_bytes": payload, "bytes_per_step": bytes_per_step,
+                       "l2": "flushed: 2xL2 scratch write before every timed kernel (outside the event intervals)",
+                       "ms_per_step_wall_incl_flush": round(wall_ms / args.steps, 4),
+                       "pack_ms": round(avg_pack, 5), "unpack_ms": round(avg_unpack, 5),
+                       "pack_gbs": round(2 * payload / (avg_pack * 1e-3) / 1e9, 1),
+                       "unpack_gbs": round(2 * payload / (avg_unpack * 1e-3) / 1e9, 1),
+                       "parallelism": f"replicas x{ws}" if ws > 1 else "1 GPU"},
+            "roofline": {"bound": "hbm", "kernel": f"k_seg<{dom}> (dt_{dom})", "achieved": round(achieved, 1),
+                         "peak": peak, "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4),
+                         "traffic": traffic,
+                         "algorithmic_bytes_per_launch": 2 * payload},
+            "gpu_launches": 2 * args.steps, "clocks": clk.summary(), "e2e": e2e}
+    if rank == 0 and ws == 1 and not args.no_cpu:
+        line["cpu_baseline"] = time_oracle_c2(seconds=args.cpu_seconds)[0]
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        import torch.distributed as tdist
+        tdist.destroy_process_group()
+
+
+def run_e2e(args, t, src_h, org, parent, payload, dev):
+    """Same metric through the public host-buffer C-ABI (dt_pack_host/dt_unpack_host):
+    H2D of the layout span + pack + D2H of the packed stream, then H2D of the packed
+    stream and the destination span + unpack + D2H of the span."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    src = torch.from_numpy(src_h).pin_memory()
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8).pin_memory()
+    pk = torch.empty(payload, dtype=torch.uint8).pin_memory()
+    s = torch.cuda.current_stream()
+    for _ in range(2):
+        dt.pack_host(t, 1, src.data_ptr() + org, pk.data_ptr(), stream=s)
+        dt.unpack_host(t, 1, pk.data_ptr(), dst.data_ptr() + org, stream=s)
+    steps = max(3, min(args.steps, 20))
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        dt.pack_host(t, 1, src.data_ptr() + org, pk.data_ptr(), stream=s)
+        dt.unpack_host(t, 1, pk.data_ptr(), dst.data_ptr() + org, stream=s)
+    torch.cuda.synchronize()
+    el = time.perf_counter() - t0
+    span = t.true_extent[1]
+    return {"value": round(4 * payload * steps / el / 1e9, 3), "unit": UNIT,
+            "h2d_bytes_per_step": 2 * span + payload, "d2h_bytes_per_step": payload + span,
+            "steps": steps, "note": "host pinned buffers; wall clock incl. all copies and syncs"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

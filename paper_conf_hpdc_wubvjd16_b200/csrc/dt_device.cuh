@@ -1,0 +1,233 @@
+// dt_device.cuh — device-side building blocks of the pack/unpack engine, shared
+// by the standalone kernels (dt_kernels.cu) and the pipelined transfer kernel
+// (dt_xfer.cu).  Everything here moves bytes with integer vector types.
+//
+//   position resolve: stream byte p -> element e = p / tsize
+//     (fast division), block b = upper_bound(boff, p mod tsize) (32-ary warp
+//     search) and the element displacement by mixed radix over the levels;
+//   seg_range  (S5/S6 long runs): a warp walks block segments of its slice and
+//     copies each with coalesced vectors and head/tail peeling;
+//   word_range (S5/S6 short blocks): each thread assembles one 16-byte vector of
+//     the packed stream from G-byte words located through a shared-memory word
+//     table of the template.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "dt_internal.h"
+
+namespace dt {
+
+// q = floor(n/d) via a 64x64 high multiply by m = floor((2^64-1)/d) and one
+// correction step (the estimate is q or q-1 for every 64-bit n).
+struct FastDiv {
+  uint64_t d, m;
+};
+static inline FastDiv make_fd(uint64_t d) { return FastDiv{d, d ? ~0ull / d : 0ull}; }
+__device__ __forceinline__ uint64_t fdiv(uint64_t n, const FastDiv& f) {
+  uint64_t q = __umul64hi(n, f.m);
+  if (n - q * f.d >= f.d) q++;
+  return q;
+}
+
+// Parameters of one pack or unpack over a committed descriptor.
+struct KP {
+  const uint8_t* nc;  // non-contiguous origin (pack: source, unpack: destination)
+  uint8_t* c;         // packed stream buffer; c[0] <-> stream byte pos
+  int64_t pos, len;
+  int64_t tsize, nblocks;
+  const int64_t* bd;
+  const int64_t* bl;
+  const int64_t* boff;
+  int64_t bd0, bl0;  // single-block template
+  int32_t nlev;
+  int32_t nwords;    // word-table entries (short kernel)
+  int64_t cnt[kMaxLevels];
+  int64_t stride[kMaxLevels];
+  const int64_t* table[kMaxLevels];
+  FastDiv fcnt[kMaxLevels];
+  FastDiv ftsize;
+  int64_t per_warp;
+  const int32_t* wtab;
+};
+
+// byte displacement of element e: mixed radix over the levels, last fastest
+__device__ __forceinline__ int64_t elem_disp(const KP& P, uint64_t e) {
+  int64_t disp = 0;
+#pragma unroll
+  for (int l = kMaxLevels - 1; l >= 0; --l) {
+    if (l < P.nlev) {
+      uint64_t i;
+      if (l == 0) {
+        i = e;
+      } else {
+        uint64_t q = fdiv(e, P.fcnt[l]);
+        i = e - q * (uint64_t)P.cnt[l];
+        e = q;
+      }
+      disp += P.table[l] ? __ldg(P.table[l] + i) : (int64_t)i * P.stride[l];
+    }
+  }
+  return disp;
+}
+
+// ---------------------------------------------------------------- loads/stores
+// Load policy: LD_CS streams (evict-first); LD_CG bypasses L1 (for ring slots a
+// peer rewrites while this kernel runs).
+enum { LD_CS = 0, LD_CG = 1 };
+template <int POL, typename V>
+__device__ __forceinline__ V ldv(const V* p) {
+  if (POL == LD_CG) return __ldcg(p);
+  return __ldcs(p);
+}
+template <typename V>
+__device__ __forceinline__ void stv(V* p, const V& v) {
+  __stcs(p, v);
+}
+
+// Copy n bytes with the whole warp, vector width V chosen from the relative
+// alignment of src and dst; head bytes peel dst to V alignment, tail bytes
+// follow (the paper's prologue/middle/epilogue, [L16:c3618 §3.1]).
+template <int POL, typename V, int U>
+__device__ __forceinline__ void warp_copy_v(uint8_t* __restrict__ dst, const uint8_t* __restrict__ src, int64_t n,
+                                            int lane) {
+  constexpr int W = sizeof(V);
+  int64_t head = (int64_t)((0 - (uintptr_t)dst) & (W - 1));
+  if (head > n) head = n;
+  if (lane < head) dst[lane] = src[lane];
+  dst += head;
+  src += head;
+  n -= head;
+  const int64_t nv = n / W;
+  V* d = reinterpret_cast<V*>(dst);
+  const V* s = reinterpret_cast<const V*>(src);
+  int64_t i = lane;
+  for (; i + 32 * (U - 1) < nv; i += 32 * U) {
+    V v[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) v[u] = ldv<POL>(s + i + 32 * u);
+#pragma unroll
+    for (int u = 0; u < U; u++) stv(d + i + 32 * u, v[u]);
+  }
+  for (; i < nv; i += 32) stv(d + i, ldv<POL>(s + i));
+  const int64_t tail = n - nv * W;
+  if (lane < tail) dst[nv * W + lane] = src[nv * W + lane];
+}
+
+template <int POL>
+__device__ __forceinline__ void warp_copy(uint8_t* dst, const uint8_t* src, int64_t n, int lane) {
+  if (n <= 0) return;
+  const unsigned rel = (unsigned)(((uintptr_t)src - (uintptr_t)dst) & 15);
+  if (rel == 0) warp_copy_v<POL, uint4, 4>(dst, src, n, lane);
+  else if ((rel & 7) == 0) warp_copy_v<POL, uint2, 8>(dst, src, n, lane);
+  else if ((rel & 3) == 0) warp_copy_v<POL, unsigned int, 8>(dst, src, n, lane);
+  else if ((rel & 1) == 0) warp_copy_v<POL, unsigned short, 8>(dst, src, n, lane);
+  else warp_copy_v<POL, unsigned char, 8>(dst, src, n, lane);
+}
+
+// largest b with boff[b] <= q (boff strictly increasing, boff[0] == 0): 32-ary
+// warp search, log32(nblocks) rounds of one coalesced probe each.
+__device__ __forceinline__ int64_t warp_find_block(const int64_t* __restrict__ boff, int64_t nb, int64_t q,
+                                                   int lane) {
+  int64_t lo = 0, hi = nb;
+  while (hi - lo > 1) {
+    int64_t step = (hi - lo + 31) / 32;
+    int64_t idx = lo + (int64_t)lane * step;
+    bool ok = idx < hi && __ldg(boff + idx) <= q;
+    unsigned m = __ballot_sync(0xffffffffu, ok);
+    int k = 31 - __clz(m);  // lane 0 always true
+    lo = lo + (int64_t)k * step;
+    hi = min(hi, lo + step);
+  }
+  return lo;
+}
+
+// One warp copies stream bytes [p, p1) (P.pos <= p < p1 <= P.pos + P.len).
+// POL applies to the loads (pack reads the layout, unpack reads the packed side).
+template <bool UNPACK, bool SINGLE, int POL>
+__device__ __forceinline__ void seg_range(const KP& P, int64_t p, const int64_t p1, const int lane) {
+  if (p >= p1) return;
+  uint64_t e = fdiv((uint64_t)p, P.ftsize);
+  int64_t r = p - (int64_t)e * P.tsize;
+  int64_t b = 0;
+  if (!SINGLE) {
+    b = warp_find_block(P.boff, P.nblocks, r, lane);
+    r -= __ldg(P.boff + b);
+  }
+  int64_t ed = elem_disp(P, e);
+  while (true) {
+    const int64_t blen = SINGLE ? P.bl0 : __ldg(P.bl + b);
+    const int64_t bdsp = SINGLE ? P.bd0 : __ldg(P.bd + b);
+    const int64_t seg = min(blen - r, p1 - p);
+    uint8_t* ncp = const_cast<uint8_t*>(P.nc) + ed + bdsp + r;
+    uint8_t* cp = P.c + (p - P.pos);
+    if (UNPACK) warp_copy<POL>(ncp, cp, seg, lane);
+    else warp_copy<POL>(cp, ncp, seg, lane);
+    p += seg;
+    if (p >= p1) break;
+    r = 0;
+    if (SINGLE || ++b == P.nblocks) {
+      b = 0;
+      ++e;
+      ed = elem_disp(P, e);
+    }
+  }
+}
+
+template <int G>
+struct WordT;
+template <> struct WordT<1> { typedef unsigned char T; };
+template <> struct WordT<2> { typedef unsigned short T; };
+template <> struct WordT<4> { typedef unsigned int T; };
+template <> struct WordT<8> { typedef unsigned long long T; };
+template <> struct WordT<16> { typedef uint4 T; };
+
+// Threads tid, tid+nthr, ... each handle one VW-byte vector of the packed
+// stream [P.pos, P.pos+P.len) (which must be G-aligned and G-granular); wt is
+// the template's word table in shared memory.
+template <bool UNPACK, int G, int VW, int POL>
+__device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64_t tid, int64_t nthr) {
+  typedef typename WordT<G>::T W;
+  typedef typename WordT<VW>::T VT;
+  constexpr int NW = VW / G;
+  const int64_t nvec = (P.len + VW - 1) / VW;
+  const int64_t end = P.pos + P.len;
+  for (int64_t v = tid; v < nvec; v += nthr) {
+    const int64_t s0 = P.pos + v * VW;
+    uint64_t e = fdiv((uint64_t)s0, P.ftsize);
+    int w = (int)((s0 - (int64_t)e * P.tsize) / G);
+    int64_t ed = elem_disp(P, e);
+    const int64_t rem = (end - s0) / G;
+    const int nvalid = rem < NW ? (int)rem : NW;
+    union {
+      VT vec;
+      W word[NW];
+    } u;
+    if (UNPACK) {
+      if (nvalid == NW) u.vec = ldv<POL>(reinterpret_cast<const VT*>(P.c + v * VW));
+      else
+        for (int k = 0; k < nvalid; k++) u.word[k] = reinterpret_cast<const W*>(P.c + v * VW)[k];
+    }
+#pragma unroll
+    for (int k = 0; k < NW; k++) {
+      if (k < nvalid) {
+        W* a = reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed + wt[w]);
+        if (UNPACK) *a = u.word[k];
+        else u.word[k] = ldv<POL>(a);
+        if (++w == P.nwords && k + 1 < nvalid) {
+          w = 0;
+          ++e;
+          ed = elem_disp(P, e);
+        }
+      }
+    }
+    if (!UNPACK) {
+      if (nvalid == NW) stv(reinterpret_cast<VT*>(P.c + v * VW), u.vec);
+      else
+        for (int k = 0; k < nvalid; k++) reinterpret_cast<W*>(P.c + v * VW)[k] = u.word[k];
+    }
+  }
+}
+
+}  // namespace dt

@@ -1,0 +1,108 @@
+// dt_internal.h — private structures of libdt (host type system, GPU descriptor,
+// kernel parameters).  Not part of the C-ABI (include/dt.h is).
+#pragma once
+#include <cstdint>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/dt.h"
+
+namespace dt {
+
+constexpr int kMaxLevels = 8;          // levels a kernel walks (incl. the instance level)
+constexpr int64_t kMaxFlatBlocks = int64_t(1) << 28;  // cap on an expanded block list
+constexpr int64_t kMaxWordTable = 12288;              // word-table kernel: entries in smem
+
+void set_error(const char* fmt, ...);
+
+// One level of the element iteration space above the block template.
+// Element index decomposes mixed-radix over the levels, the LAST level fastest
+// (typemap order: outer constructor loops are slow).  A regular level
+// contributes idx*stride bytes, a list level contributes table[idx] bytes.
+struct Level {
+  int64_t cnt = 1;
+  int64_t stride = 0;
+  std::shared_ptr<std::vector<int64_t>> table;  // non-null => list level
+  bool is_list() const { return table != nullptr; }
+  int64_t contrib(int64_t i) const { return table ? (*table)[i] : i * stride; }
+};
+
+// Flattened form of one type instance: for each element e (in typemap order)
+// the template blocks (bd[i] + disp(e), bl[i]) in order.  This is the B200
+// re-encoding of the paper's DEV list ([L16:c5201 §3.2]): regular nests stay
+// implicit (the paper's vector kernel, [L16:c2243 §3.1]) and only irregular
+// parts are listed.
+struct Form {
+  std::vector<Level> lv;           // outermost first
+  std::vector<int64_t> bd, bl;     // template blocks (bytes), typemap order
+  int64_t tsize() const { int64_t s = 0; for (auto x : bl) s += x; return s; }
+  int64_t nelem() const { int64_t n = 1; for (auto& l : lv) n *= l.cnt; return n; }
+  bool empty() const { return bl.empty(); }
+};
+
+void normalize(Form& f);
+// Expand into merged blocks (typemap order).  Returns false if > cap.
+bool expand(const Form& f, std::vector<int64_t>& d, std::vector<int64_t>& l, int64_t cap);
+int64_t form_granularity(const Form& f);
+
+// Per-device copy of the descriptor.
+struct DeviceDesc {
+  int device = -1;
+  int64_t* bd = nullptr;    // template disps
+  int64_t* bl = nullptr;    // template lens
+  int64_t* boff = nullptr;  // exclusive prefix of bl (device scan)
+  std::vector<int64_t*> tables;  // per level (nullptr for regular levels)
+  // word tables for the short kernel, keyed by granularity (1,2,4,8,16)
+  int32_t* wtab[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+};
+
+enum Kind { K_BASIC, K_CONTIG, K_HVECTOR, K_HINDEXED, K_STRUCT, K_SUBARRAY, K_RESIZED };
+
+}  // namespace dt
+
+struct dt_type_s {
+  int refcnt = 1;
+  bool predefined = false;
+  dt::Kind kind = dt::K_BASIC;
+  int basic = 0;
+  int64_t count = 0, blocklen = 0, stride = 0;           // stride in bytes
+  std::vector<int64_t> bls, dps;                          // bytes
+  std::vector<dt_type_s*> types;                          // struct components
+  int ndims = 0, order = 0;
+  std::vector<int64_t> sizes, subsizes, starts;
+  dt_type_s* old = nullptr;
+  // bounds
+  int64_t size = 0, lb = 0, ub = 0, true_lb = 0, true_ub = 0, align = 1;
+  bool has_lb = false, has_ub = false;
+  // commit state
+  std::mutex mu;
+  bool committed = false;
+  std::unique_ptr<dt::Form> form;        // host form (built lazily)
+  std::vector<dt::DeviceDesc> devs;      // per device uploads
+  // overlap cache (unpack legality) for the last count checked
+  int64_t ovl_count = -1;
+  int ovl_result = 0;
+  int64_t extent() const { return ub - lb; }
+};
+
+namespace dt {
+// kernels.cu
+struct KLevels {
+  int n = 0;
+  int64_t cnt[kMaxLevels];
+  int64_t stride[kMaxLevels];
+  const int64_t* table[kMaxLevels];
+};
+dt_status upload_desc(dt_type_s* t, const Form& f, DeviceDesc& dd);
+void free_desc(DeviceDesc& dd);
+dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDesc& dd, int64_t count,
+                             const void* nc, void* c, int64_t pos, int64_t len, void* stream);
+int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
+                int64_t* gran);
+void build_levels(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count, KLevels& L);
+dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out);
+const Form& get_form(dt_type_s* t);
+dt_status ensure_wtab_pub(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out);
+}  // namespace dt

@@ -1,0 +1,664 @@
+// dt_kernels.cu — sm_100a kernels of libdt and the pack/unpack entry points.
+//
+//   k_scan_*   device exclusive prefix of the template block lengths with warp
+//              shuffles (the paper computes DEV packed displacements on the CPU,
+//              [L16:c5996 §3.2]; here the scan runs on the GPU at commit).
+//   k_seg      "warp-per-block" pack/unpack for long runs: every warp owns an
+//              equal slice of the packed stream (the paper's equal-size CUDA DEVs
+//              per warp, S = 1/2/4 KB, [L16:c5678]-[L18:c753 §3.2], so skewed block
+//              lengths — the triangle — no longer cost occupancy, [L24:c282 §5.1]),
+//              resolves its start position once (mixed-radix element index +
+//              32-ary warp search over the block prefix) and walks block segments,
+//              copying each with coalesced 16-byte vectors and head/tail peeling
+//              ([L16:c2741]-[L16:c3777 §3.1]; the paper used 8 B/thread on Kepler).
+//   k_word     "thread-per-element" pack/unpack for short blocks (4-64 B): a word
+//              table of the template (granularity G) lives in shared memory, each
+//              thread assembles one 16-byte vector of the packed stream, so the
+//              contiguous side is written/read with full coalesced 16 B accesses.
+//
+// Everything is byte movement on integer vector types: no floating point.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+
+#include "dt_device.cuh"
+#include "dt_internal.h"
+
+namespace dt {
+
+// --------------------------------------------------------------- scan (K6)
+// Block-wide exclusive scan of one int64 per thread using warp shuffles.
+template <int NT>
+__device__ __forceinline__ int64_t block_exclusive_scan(int64_t v, int64_t* total) {
+  __shared__ int64_t wsum[NT / 32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int64_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int64_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) wsum[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    int64_t s = lane < NT / 32 ? wsum[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int64_t y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < NT / 32) wsum[lane] = s;  // inclusive warp prefix
+  }
+  __syncthreads();
+  int64_t before = w ? wsum[w - 1] : 0;
+  *total = wsum[NT / 32 - 1];
+  __syncthreads();
+  return before + x - v;
+}
+
+constexpr int kScanNT = 256, kScanItems = 4, kScanTile = kScanNT * kScanItems;
+
+__global__ void __launch_bounds__(kScanNT) k_scan_local(const int64_t* __restrict__ in, int64_t* __restrict__ out,
+                                                        int64_t* __restrict__ sums, int64_t n) {
+  int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanItems;
+  int64_t v[kScanItems], s = 0;
+#pragma unroll
+  for (int k = 0; k < kScanItems; k++) {
+    v[k] = base + k < n ? in[base + k] : 0;
+    s += v[k];
+  }
+  int64_t tot;
+  int64_t ex = block_exclusive_scan<kScanNT>(s, &tot);
+#pragma unroll
+  for (int k = 0; k < kScanItems; k++) {
+    if (base + k < n) out[base + k] = ex;
+    ex += v[k];
+  }
+  if (threadIdx.x == 0) sums[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kScanNT) k_scan_sums(int64_t* sums, int64_t nb) {
+  int64_t carry = 0;
+  for (int64_t b0 = 0; b0 < nb; b0 += kScanNT) {
+    int64_t i = b0 + threadIdx.x;
+    int64_t v = i < nb ? sums[i] : 0, tot;
+    int64_t ex = block_exclusive_scan<kScanNT>(v, &tot);
+    if (i < nb) sums[i] = carry + ex;
+    carry += tot;
+  }
+}
+
+__global__ void __launch_bounds__(kScanNT) k_scan_add(int64_t* out, const int64_t* sums, int64_t n) {
+  int64_t base = (int64_t)blockIdx.x * kScanTile;
+  int64_t add = sums[blockIdx.x];
+  for (int k = threadIdx.x; k < kScanTile; k += kScanNT)
+    if (base + k < n) out[base + k] += add;
+}
+
+// --------------------------------------------------------------- standalone kernels
+template <bool UNPACK, bool SINGLE>
+__global__ void __launch_bounds__(256) k_seg(const KP P) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t p = P.pos + gw * P.per_warp;
+  const int64_t p1 = min(p + P.per_warp, P.pos + P.len);
+  seg_range<UNPACK, SINGLE, LD_CS>(P, p, p1, lane);
+}
+
+template <bool UNPACK, int G, int VW>
+__global__ void __launch_bounds__(256) k_word(const KP P) {
+  extern __shared__ int32_t wt[];
+  for (int i = threadIdx.x; i < P.nwords; i += blockDim.x) wt[i] = P.wtab[i];
+  __syncthreads();
+  word_range<UNPACK, G, VW, LD_CS>(P, wt, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                                   (int64_t)gridDim.x * blockDim.x);
+}
+// --------------------------------------------------------------- host side
+static int g_num_sms = 0;
+static int num_sms() {
+  if (!g_num_sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (g_num_sms <= 0) g_num_sms = 148;
+  }
+  return g_num_sms;
+}
+
+static dt_status cuda_fail(cudaError_t e, const char* what) {
+  set_error("%s: %s", what, cudaGetErrorString(e));
+  return DT_ERR_CUDA;
+}
+#define CU(call)                                        \
+  do {                                                  \
+    cudaError_t _e = (call);                            \
+    if (_e != cudaSuccess) return cuda_fail(_e, #call); \
+  } while (0)
+
+void free_desc(DeviceDesc& dd) {
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (dd.device >= 0 && dd.device != cur) cudaSetDevice(dd.device);
+  cudaFree(dd.bd);
+  cudaFree(dd.bl);
+  cudaFree(dd.boff);
+  for (auto* p : dd.tables) cudaFree(p);
+  for (auto*& w : dd.wtab) { cudaFree(w); w = nullptr; }
+  dd.bd = dd.bl = dd.boff = nullptr;
+  dd.tables.clear();
+  if (cur >= 0 && dd.device >= 0 && dd.device != cur) cudaSetDevice(cur);
+}
+
+static int log2_small(int64_t g) { return g == 1 ? 0 : g == 2 ? 1 : g == 4 ? 2 : g == 8 ? 3 : 4; }
+
+dt_status upload_desc(dt_type_s* t, const Form& f, DeviceDesc& dd) {
+  (void)t;
+  cudaStream_t s;
+  CU(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  const int64_t nb = (int64_t)f.bl.size();
+  const size_t bytes = sizeof(int64_t) * (size_t)std::max<int64_t>(nb, 1);
+  CU(cudaMalloc(&dd.bd, bytes));
+  CU(cudaMalloc(&dd.bl, bytes));
+  CU(cudaMalloc(&dd.boff, bytes));
+  if (nb > 0) {
+    CU(cudaMemcpyAsync(dd.bd, f.bd.data(), sizeof(int64_t) * nb, cudaMemcpyHostToDevice, s));
+    CU(cudaMemcpyAsync(dd.bl, f.bl.data(), sizeof(int64_t) * nb, cudaMemcpyHostToDevice, s));
+    const int64_t ntile = (nb + kScanTile - 1) / kScanTile;
+    int64_t* sums = nullptr;
+    CU(cudaMallocAsync(&sums, sizeof(int64_t) * ntile, s));
+    k_scan_local<<<(unsigned)ntile, kScanNT, 0, s>>>(dd.bl, dd.boff, sums, nb);
+    k_scan_sums<<<1, kScanNT, 0, s>>>(sums, ntile);
+    k_scan_add<<<(unsigned)ntile, kScanNT, 0, s>>>(dd.boff, sums, nb);
+    CU(cudaGetLastError());
+    CU(cudaFreeAsync(sums, s));
+  }
+  dd.tables.assign(f.lv.size(), nullptr);
+  for (size_t i = 0; i < f.lv.size(); i++) {
+    if (!f.lv[i].is_list()) continue;
+    const auto& tab = *f.lv[i].table;
+    CU(cudaMalloc(&dd.tables[i], sizeof(int64_t) * tab.size()));
+    CU(cudaMemcpyAsync(dd.tables[i], tab.data(), sizeof(int64_t) * tab.size(), cudaMemcpyHostToDevice, s));
+  }
+  CU(cudaStreamSynchronize(s));
+  // sanity: the device prefix must end at tsize - last len
+  if (nb > 0) {
+    int64_t last = 0;
+    CU(cudaMemcpy(&last, dd.boff + nb - 1, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    if (last != f.tsize() - f.bl.back()) {
+      set_error("device scan mismatch (%lld vs %lld)", (long long)last, (long long)(f.tsize() - f.bl.back()));
+      cudaStreamDestroy(s);
+      return DT_ERR_CUDA;
+    }
+  }
+  CU(cudaStreamDestroy(s));
+  return DT_OK;
+}
+
+// word table of the template at granularity g: word k -> byte offset of its
+// source inside the element (int32).  Built lazily per granularity.
+static dt_status ensure_wtab(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out) {
+  int li = log2_small(g);
+  if (!dd.wtab[li]) {
+    const int64_t nw = f.tsize() / g;
+    std::vector<int32_t> h((size_t)nw);
+    int64_t k = 0;
+    for (size_t b = 0; b < f.bl.size(); b++)
+      for (int64_t o = 0; o < f.bl[b]; o += g) h[(size_t)k++] = (int32_t)(f.bd[b] + o);
+    CU(cudaMalloc(&dd.wtab[li], sizeof(int32_t) * std::max<int64_t>(nw, 1)));
+    CU(cudaMemcpy(dd.wtab[li], h.data(), sizeof(int32_t) * nw, cudaMemcpyHostToDevice));
+  }
+  *out = dd.wtab[li];
+  return DT_OK;
+}
+
+dt_status ensure_wtab_pub(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out) {
+  return ensure_wtab(f, dd, g, out);
+}
+
+static int64_t lowp2(uint64_t x) {
+  if (x == 0) return 16;
+  int64_t g = (int64_t)(x & (~x + 1));
+  return g > 16 ? 16 : g;
+}
+
+// Levels for one launch: the committed form's levels with the instance level
+// (count, extent) prepended as the outermost level, merged when regular.
+void build_levels(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count, KLevels& L) {
+  L.n = 0;
+  int off = 0;
+  if (count > 1) {
+    L.cnt[0] = count;
+    L.stride[0] = t->extent();
+    L.table[0] = nullptr;
+    L.n = 1;
+    off = 1;
+  }
+  for (size_t i = 0; i < f.lv.size(); i++) {
+    L.cnt[off + i] = f.lv[i].cnt;
+    L.stride[off + i] = f.lv[i].stride;
+    L.table[off + i] = f.lv[i].is_list() ? (dd ? dd->tables[i] : reinterpret_cast<const int64_t*>(1)) : nullptr;
+    L.n++;
+  }
+  // merge the instance level into the next regular level when contiguous in index space
+  if (count > 1 && L.n >= 2 && !L.table[1] && L.stride[0] == L.cnt[1] * L.stride[1]) {
+    L.cnt[1] *= L.cnt[0];
+    for (int i = 0; i + 1 < L.n; i++) {
+      L.cnt[i] = L.cnt[i + 1];
+      L.stride[i] = L.stride[i + 1];
+      L.table[i] = L.table[i + 1];
+    }
+    L.n--;
+  }
+}
+
+static bool template_fits_int32(const Form& f) {
+  for (size_t b = 0; b < f.bd.size(); b++)
+    if (f.bd[b] < INT32_MIN || f.bd[b] + f.bl[b] > INT32_MAX) return false;
+  return true;
+}
+
+// Effective template of one launch: a single-block template whose innermost
+// regular level continues the run (e.g. count instances of a contiguous type)
+// becomes one longer run, when that makes it a long-run copy.
+struct Eff {
+  KLevels L;
+  int64_t tsize, nblocks, bd0, bl0;
+  bool merged;
+};
+static Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count) {
+  Eff E;
+  build_levels(f, dd, t, count, E.L);
+  E.tsize = f.tsize();
+  E.nblocks = (int64_t)f.bl.size();
+  E.bd0 = f.bd.empty() ? 0 : f.bd[0];
+  E.bl0 = f.bl.empty() ? 0 : f.bl[0];
+  E.merged = false;
+  KLevels& L = E.L;
+  while (E.nblocks == 1 && L.n >= 1 && !L.table[L.n - 1] && L.stride[L.n - 1] == E.bl0 &&
+         E.bl0 * L.cnt[L.n - 1] >= 256) {
+    E.bl0 *= L.cnt[L.n - 1];
+    E.tsize = E.bl0;
+    L.n--;
+    E.merged = true;
+  }
+  return E;
+}
+
+int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
+                int64_t* gran) {
+  if (len <= 0 || f.bl.empty()) return 0;
+  const int64_t nb = (int64_t)f.bl.size();
+  const int64_t ts = f.tsize();
+  int64_t g = form_granularity(f);
+  for (int i = 0; i < L.n; i++)
+    if (!L.table[i]) g = std::min(g, lowp2((uint64_t)L.stride[i]));  // list tables counted in form
+  g = std::min(g, lowp2(nc_addr));
+  g = std::min(g, lowp2(c_addr));
+  g = std::min(g, lowp2((uint64_t)pos));
+  g = std::min(g, lowp2((uint64_t)len));
+  *gran = g;
+  const double mean = (double)ts / (double)nb;
+  if (mean < 256.0 && ts / g <= kMaxWordTable && ts % g == 0 && template_fits_int32(f)) return 2;
+  return 1;
+}
+
+template <bool UNPACK>
+static void launch_word(const KP& P, int64_t g, bool vec16, unsigned grid, size_t smem, cudaStream_t s) {
+#define LW(G, VW) k_word<UNPACK, G, VW><<<grid, 256, smem, s>>>(P)
+  if (vec16) {
+    switch (g) {
+      case 1: LW(1, 16); break;
+      case 2: LW(2, 16); break;
+      case 4: LW(4, 16); break;
+      case 8: LW(8, 16); break;
+      default: LW(16, 16); break;
+    }
+  } else {
+    switch (g) {
+      case 1: LW(1, 1); break;
+      case 2: LW(2, 2); break;
+      case 4: LW(4, 4); break;
+      case 8: LW(8, 8); break;
+      default: LW(16, 16); break;
+    }
+  }
+#undef LW
+}
+
+dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDesc& dd, int64_t count, const void* nc,
+                             void* c, int64_t pos, int64_t len, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  Eff E = effective(f, &dd, t, count);
+  const KLevels& L = E.L;
+  KP P;
+  std::memset(&P, 0, sizeof(P));
+  P.nc = (const uint8_t*)nc;
+  P.c = (uint8_t*)c;
+  P.pos = pos;
+  P.len = len;
+  P.tsize = E.tsize;
+  P.nblocks = E.nblocks;
+  P.bd = dd.bd;
+  P.bl = dd.bl;
+  P.boff = dd.boff;
+  P.bd0 = E.bd0;
+  P.bl0 = E.bl0;
+  P.nlev = L.n;
+  for (int i = 0; i < L.n; i++) {
+    P.cnt[i] = L.cnt[i];
+    P.stride[i] = L.stride[i];
+    P.table[i] = L.table[i];
+    P.fcnt[i] = make_fd((uint64_t)L.cnt[i]);
+  }
+  P.ftsize = make_fd((uint64_t)P.tsize);
+  int64_t g = 1;
+  int kind = E.merged ? 1 : plan_kernel(f, L, (uint64_t)(uintptr_t)nc, (uint64_t)(uintptr_t)c, pos, len, &g);
+  if (kind == 0) return DT_OK;
+  const int sms = num_sms();
+  if (kind == 1) {
+    const int64_t max_warps = (int64_t)sms * 8 * 8;  // 8 CTAs x 8 warps per SM
+    int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
+    int64_t per = (len + nw - 1) / nw;
+    per = (per + 511) & ~int64_t(511);
+    nw = (len + per - 1) / per;
+    P.per_warp = per;
+    unsigned grid = (unsigned)((nw + 7) / 8);
+    const bool single = P.nblocks == 1;
+    if (unpack) {
+      if (single) k_seg<true, true><<<grid, 256, 0, s>>>(P);
+      else k_seg<true, false><<<grid, 256, 0, s>>>(P);
+    } else {
+      if (single) k_seg<false, true><<<grid, 256, 0, s>>>(P);
+      else k_seg<false, false><<<grid, 256, 0, s>>>(P);
+    }
+  } else {
+    const int32_t* wt = nullptr;
+    dt_status st = ensure_wtab(f, dd, g, &wt);
+    if (st != DT_OK) return st;
+    P.wtab = wt;
+    P.nwords = (int32_t)(f.tsize() / g);
+    const bool vec16 = (((uintptr_t)c) & 15) == 0;
+    const int64_t vw = vec16 ? 16 : g;
+    const int64_t nvec = (len + vw - 1) / vw;
+    const int64_t maxg = (int64_t)sms * 8;
+    unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(maxg, (nvec + 255) / 256));
+    size_t smem = sizeof(int32_t) * (size_t)P.nwords;
+    if (unpack) launch_word<true>(P, g, vec16, grid, smem, s);
+    else launch_word<false>(P, g, vec16, grid, smem, s);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+  return DT_OK;
+}
+
+dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out) {
+  int dev = 0;
+  CU(cudaGetDevice(&dev));
+  const Form& f = get_form(t);
+  std::lock_guard<std::mutex> g(t->mu);
+  for (auto& dd : t->devs)
+    if (dd.device == dev) { *out = &dd; return DT_OK; }
+  t->devs.emplace_back();
+  DeviceDesc& dd = t->devs.back();
+  dd.device = dev;
+  dt_status st = upload_desc(t, f, dd);
+  if (st != DT_OK) {
+    free_desc(dd);
+    t->devs.pop_back();
+    return st;
+  }
+  *out = &dd;
+  return DT_OK;
+}
+
+// Unpack legality (reading A9): the typemap of `count` instances must not
+// overlap.  Cheap structural proof first, exact sorted-interval check if needed.
+static int check_nonoverlap(dt_type_s* t, const Form& f, int64_t count) {
+  if (f.bl.empty() || count == 0) return 1;
+  // template: sorted intervals
+  std::vector<std::pair<int64_t, int64_t>> iv;
+  iv.reserve(f.bl.size());
+  for (size_t i = 0; i < f.bl.size(); i++) iv.push_back({f.bd[i], f.bd[i] + f.bl[i]});
+  std::sort(iv.begin(), iv.end());
+  for (size_t i = 1; i < iv.size(); i++)
+    if (iv[i].first < iv[i - 1].second) return 0;
+  int64_t lo = iv.front().first, hi = 0;
+  for (auto& x : iv) hi = std::max(hi, x.second);
+  bool proven = true;
+  auto level = [&](int64_t cnt, int64_t stride, const std::vector<int64_t>* tab) {
+    if (!proven || cnt <= 1) return;
+    const int64_t span = hi - lo;
+    if (tab) {
+      std::vector<int64_t> s(*tab);
+      std::sort(s.begin(), s.end());
+      for (size_t i = 1; i < s.size(); i++)
+        if (s[i] - s[i - 1] < span) { proven = false; return; }
+      lo += s.front();
+      hi += s.back();
+    } else {
+      if ((stride < 0 ? -stride : stride) < span) { proven = false; return; }
+      int64_t last = (cnt - 1) * stride;
+      lo += std::min<int64_t>(0, last);
+      hi += std::max<int64_t>(0, last);
+    }
+  };
+  for (int i = (int)f.lv.size() - 1; i >= 0; i--) level(f.lv[i].cnt, f.lv[i].stride, f.lv[i].table.get());
+  level(count, t->extent(), nullptr);
+  if (proven) return 1;
+  // exact check on the expanded list
+  Form g = f;
+  if (count > 1) {
+    Level l;
+    l.cnt = count;
+    l.stride = t->extent();
+    g.lv.insert(g.lv.begin(), l);
+  }
+  std::vector<int64_t> d, len;
+  if (!expand(g, d, len, int64_t(1) << 26)) return -1;
+  iv.clear();
+  for (size_t i = 0; i < d.size(); i++) iv.push_back({d[i], d[i] + len[i]});
+  std::sort(iv.begin(), iv.end());
+  for (size_t i = 1; i < iv.size(); i++)
+    if (iv[i].first < iv[i - 1].second) return 0;
+  return 1;
+}
+
+static dt_status check_dev_ptr(const void* p, const char* what) {
+  cudaPointerAttributes a;
+  cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    set_error("%s: not a device pointer (%s)", what, cudaGetErrorString(e));
+    return DT_ERR_ARG;
+  }
+  if (a.type != cudaMemoryTypeDevice && a.type != cudaMemoryTypeManaged) {
+    set_error("%s: host pointer passed to a device entry point (no CPU fallback)", what);
+    return DT_ERR_ARG;
+  }
+  return DT_OK;
+}
+
+static bool g_check_ptrs = true;
+
+static dt_status pack_common(bool unpack, dt_t t, int64_t count, const void* nc, void* c, int64_t pos, int64_t* len,
+                             void* stream) {
+  if (!t || !len || count < 0 || pos < 0 || *len < 0) {
+    set_error("dt_%s: bad argument", unpack ? "unpack" : "pack");
+    return DT_ERR_ARG;
+  }
+  if (!t->committed) {
+    set_error("dt_%s: type not committed", unpack ? "unpack" : "pack");
+    return DT_ERR_NOT_COMMITTED;
+  }
+  const int64_t total = count * t->size;
+  int64_t n = pos >= total ? 0 : std::min<int64_t>(*len, total - pos);
+  *len = n;
+  if (n == 0) return DT_OK;
+  if (!nc || !c) {
+    set_error("dt_%s: NULL buffer", unpack ? "unpack" : "pack");
+    return DT_ERR_ARG;
+  }
+  if (g_check_ptrs) {
+    dt_status st = check_dev_ptr((const uint8_t*)nc + t->true_lb, "origin");
+    if (st != DT_OK) return st;
+    st = check_dev_ptr(c, "packed");
+    if (st != DT_OK) return st;
+  }
+  DeviceDesc* dd = nullptr;
+  dt_status st = ensure_committed_on_device(t, &dd);
+  if (st != DT_OK) return st;
+  const Form& f = get_form(t);
+  if (unpack) {
+    std::lock_guard<std::mutex> g(t->mu);
+    if (t->ovl_count != count) {
+      t->ovl_result = check_nonoverlap(t, f, count);
+      t->ovl_count = count;
+    }
+    if (t->ovl_result != 1) {
+      set_error("dt_unpack: typemap entries overlap%s", t->ovl_result < 0 ? " (could not be proven disjoint)" : "");
+      return DT_ERR_OVERLAP;
+    }
+  }
+  return launch_pack_unpack(unpack, t, f, *dd, count, nc, c, pos, n, stream);
+}
+
+}  // namespace dt
+
+using namespace dt;
+
+extern "C" {
+
+dt_status dt_commit(dt_t t) {
+  if (!t) {
+    set_error("dt_commit: NULL type");
+    return DT_ERR_ARG;
+  }
+  try {
+    get_form(t);
+  } catch (...) {
+    set_error("dt_commit: flattening failed (too many blocks or out of memory)");
+    return DT_ERR_NOMEM;
+  }
+  DeviceDesc* dd = nullptr;
+  dt_status st = ensure_committed_on_device(t, &dd);
+  if (st != DT_OK) return st;
+  t->committed = true;
+  if (const char* e = getenv("DT_NOCHECK")) g_check_ptrs = (e[0] == '0');
+  return DT_OK;
+}
+
+dt_status dt_pack(dt_t t, int64_t count, const void* origin, void* packed, int64_t pos, int64_t* len, void* stream) {
+  return pack_common(false, t, count, origin, packed, pos, len, stream);
+}
+
+dt_status dt_unpack(dt_t t, int64_t count, const void* packed, void* origin, int64_t pos, int64_t* len,
+                    void* stream) {
+  return pack_common(true, t, count, origin, const_cast<void*>(packed), pos, len, stream);
+}
+
+dt_status dt_plan(dt_t t, int64_t count, uint64_t origin_addr, uint64_t packed_addr, int64_t pos, int64_t len,
+                  int* kernel, int64_t* granularity) {
+  if (!t || !kernel || !granularity || count < 0 || pos < 0 || len < 0) {
+    set_error("dt_plan: bad argument");
+    return DT_ERR_ARG;
+  }
+  const Form* f;
+  try {
+    f = &get_form(t);
+  } catch (...) {
+    set_error("dt_plan: flattening failed");
+    return DT_ERR_NOMEM;
+  }
+  const int64_t total = count * t->size;
+  const int64_t n = pos >= total ? 0 : std::min<int64_t>(len, total - pos);
+  Eff E = effective(*f, nullptr, t, count);
+  *granularity = 1;
+  *kernel = n <= 0 ? 0 : E.merged ? 1 : plan_kernel(*f, E.L, origin_addr, packed_addr, pos, n, granularity);
+  return DT_OK;
+}
+
+// Host-buffer entry points: stage the span the layout touches through device
+// scratch memory (H2D), run the GPU kernel, copy the result back (D2H).
+static void* g_scratch[2] = {nullptr, nullptr};
+static size_t g_scratch_sz[2] = {0, 0};
+static int g_scratch_dev = -1;
+static std::mutex g_scratch_mu;
+
+static dt_status scratch(int i, size_t n, void** out) {
+  int dev = 0;
+  CU(cudaGetDevice(&dev));
+  if (g_scratch_dev != dev) {
+    for (int k = 0; k < 2; k++) { g_scratch[k] = nullptr; g_scratch_sz[k] = 0; }
+    g_scratch_dev = dev;
+  }
+  if (g_scratch_sz[i] < n) {
+    if (g_scratch[i]) cudaFree(g_scratch[i]);
+    g_scratch[i] = nullptr;
+    g_scratch_sz[i] = 0;
+    CU(cudaMalloc(&g_scratch[i], n));
+    g_scratch_sz[i] = n;
+  }
+  *out = g_scratch[i];
+  return DT_OK;
+}
+
+static dt_status host_common(bool unpack, dt_t t, int64_t count, const void* a, void* b, int64_t pos, int64_t* len,
+                             void* stream) {
+  if (!t || !len || count < 0 || pos < 0 || *len < 0 || !a || !b) {
+    set_error("dt_%s_host: bad argument", unpack ? "unpack" : "pack");
+    return DT_ERR_ARG;
+  }
+  if (!t->committed) {
+    set_error("dt_%s_host: type not committed", unpack ? "unpack" : "pack");
+    return DT_ERR_NOT_COMMITTED;
+  }
+  const int64_t total = count * t->size;
+  const int64_t n = pos >= total ? 0 : std::min<int64_t>(*len, total - pos);
+  *len = n;
+  if (n == 0) return DT_OK;
+  // span of count instances: [true_lb + min(0,(count-1)ext), true_ub + max(0,(count-1)ext))
+  const int64_t last = (count - 1) * t->extent();
+  const int64_t lo = t->true_lb + std::min<int64_t>(0, last);
+  const int64_t hi = t->true_ub + std::max<int64_t>(0, last);
+  std::lock_guard<std::mutex> g(g_scratch_mu);
+  void *dspan, *dpack;
+  dt_status st = scratch(0, (size_t)(hi - lo), &dspan);
+  if (st != DT_OK) return st;
+  st = scratch(1, (size_t)n, &dpack);
+  if (st != DT_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  uint8_t* dorigin = (uint8_t*)dspan - lo;
+  bool saved = g_check_ptrs;
+  g_check_ptrs = false;
+  int64_t m = n;
+  if (!unpack) {
+    const uint8_t* horigin = (const uint8_t*)a;
+    CU(cudaMemcpyAsync(dspan, horigin + lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, s));
+    st = pack_common(false, t, count, dorigin, dpack, pos, &m, stream);
+    if (st == DT_OK) CU(cudaMemcpyAsync(b, dpack, (size_t)n, cudaMemcpyDeviceToHost, s));
+  } else {
+    uint8_t* horigin = (uint8_t*)b;
+    // gaps must stay untouched: bring the destination span in, scatter, send it back
+    CU(cudaMemcpyAsync(dspan, horigin + lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, s));
+    CU(cudaMemcpyAsync(dpack, a, (size_t)n, cudaMemcpyHostToDevice, s));
+    st = pack_common(true, t, count, dpack, dorigin, pos, &m, stream);
+    if (st == DT_OK) CU(cudaMemcpyAsync(horigin + lo, dspan, (size_t)(hi - lo), cudaMemcpyDeviceToHost, s));
+  }
+  g_check_ptrs = saved;
+  if (st != DT_OK) return st;
+  CU(cudaStreamSynchronize(s));
+  return DT_OK;
+}
+
+dt_status dt_pack_host(dt_t t, int64_t count, const void* origin, void* packed, int64_t pos, int64_t* len,
+                       void* stream) {
+  return host_common(false, t, count, origin, packed, pos, len, stream);
+}
+dt_status dt_unpack_host(dt_t t, int64_t count, const void* packed, void* origin, int64_t pos, int64_t* len,
+                         void* stream) {
+  return host_common(true, t, count, packed, origin, pos, len, stream);
+}
+
+}  // extern "C"

@@ -1,0 +1,906 @@
+// dt_xfer.cu — GPU<->GPU pipelined transfer of non-contiguous data (S7).
+//
+// Paper ([L18:c4394]-[L20:c4670 §4.1], Fig. 4): the sender packs fragments into a
+// GPU staging buffer exposed to the receiver over CUDA IPC; the receiver unpacks
+// each fragment as soon as the sender signals it and acknowledges it so the
+// fragment can be reused; with a pipeline the cost falls to "the cost of the
+// data transfer plus the cost of the most expensive operation (pack or unpack)
+// on a single fragment" ([L18:c4932]).  Connection setup exchanges the IPC
+// handle once ([L20:c3123], [L20:c3807]); the receiver sends "start packing"
+// ([L20:c3973]); the sender signals "unpack fragment i" ([L20:c3380]) and the
+// receiver acks ([L20:c4133]).
+//
+// B200 design:
+//  * P2P mode: ONE persistent kernel per call (or per group of calls) whose
+//    send-role CTAs pack fragment k straight into the receiver's ring slot k%D in
+//    peer HBM over NVLink (remote 16-byte stores), then publish it with a
+//    release.sys add of the bytes written to the receiver's ready[slot]; the
+//    receive-role CTAs spin (ld.acquire.sys) on their local ready[slot], unpack
+//    the slot into the user's layout and add the bytes consumed to the sender's
+//    ack[slot].  Chunk != launch: the chunk size only sets flow-control
+//    granularity.  Counters are cumulative bytes per slot; each side keeps its
+//    base per (peer, channel) in device memory, double-buffered by message parity.
+//    Header {seq, nbytes} + "go" word implement the handshake and truncation check.
+//  * NCCL mode: double-buffered chunks: pack(k) -> ncclSend/ncclRecv -> unpack(k)
+//    on three internal streams with per-slot events.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <vector>
+
+#include "dt_device.cuh"
+#include "dt_internal.h"
+
+namespace dt {
+
+constexpr int kMaxOps = 16;
+constexpr int kMaxCh = 6;  // concurrent messages per (pair, direction) inside one group
+constexpr uint64_t kAbort = 1ull << 63;
+
+struct XOp {
+  KP P;            // pack (send role) or unpack (recv role) over the user's layout
+  int32_t role;    // 0 send, 1 recv
+  int32_t kind;    // 1 segment walk, 2 word table
+  int32_t single;  // segment walk over a single-block template
+  int32_t g;       // word granularity
+  int64_t n;       // send: bytes; recv: capacity in bytes
+  int64_t chunk;
+  int32_t depth, cta0, ncta, pad;
+  uint8_t* ring;   // slot 0 of the (pair, channel) ring (send: peer memory; recv: local)
+  uint64_t* ready; // [depth]  send: peer; recv: local
+  uint64_t* ack;   // [depth]  send: local; recv: peer
+  uint64_t* hdr;   // [2] {seq, nbytes}  send: peer; recv: local
+  uint64_t* go;    // [1]     send: local; recv: peer
+  const uint64_t* base_in;  // [depth] cumulative bytes per slot before this message
+  uint64_t* base_out;       // [depth] after it
+  uint64_t seq;
+  int32_t* err;
+};
+
+struct XArgs {
+  int32_t nops;
+  int32_t pad;
+  int64_t timeout_ns;
+  XOp ops[kMaxOps];
+};
+
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_sys_add(uint64_t* p, uint64_t v) {
+  asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+enum { XERR_TIMEOUT = 1, XERR_TRUNCATE = 2 };
+
+// spin until pred(*p) holds; false on timeout (sets *err)
+template <typename Pred>
+__device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeout_ns, int32_t* err, uint64_t* out) {
+  uint64_t v = ld_acquire_sys(p);
+  if (pred(v)) { *out = v; return true; }
+  const uint64_t t0 = gtimer();
+  int ns = 32;
+  while (true) {
+    __nanosleep(ns);
+    if (ns < 1024) ns <<= 1;
+    v = ld_acquire_sys(p);
+    if (pred(v)) { *out = v; return true; }
+    if ((int64_t)(gtimer() - t0) > timeout_ns) {
+      atomicCAS(err, 0, XERR_TIMEOUT);
+      return false;
+    }
+  }
+}
+
+// pack or unpack stream bytes [lo, lo+len) of the current chunk with this CTA.
+template <bool UNPACK>
+__device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int64_t lo, int64_t len,
+                                          const int32_t* wt) {
+  P.c = slot + lo;  // slot maps stream byte 0 of the message (see caller)
+  P.pos = lo;
+  P.len = len;
+  constexpr int POL = UNPACK ? LD_CG : LD_CS;  // ring slots are rewritten by the peer: bypass L1
+  if (X.kind == 2) {
+    const int64_t body = len - len % X.g;
+    KP Q = P;
+    Q.len = body;
+    switch (X.g) {
+      case 1: word_range<UNPACK, 1, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 2: word_range<UNPACK, 2, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 4: word_range<UNPACK, 4, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 8: word_range<UNPACK, 8, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
+      default: word_range<UNPACK, 16, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
+    }
+    if (body < len && threadIdx.x < 32)  // ragged tail (< G bytes): one warp walks it
+      seg_range<UNPACK, false, POL>(P, lo + body, lo + len, threadIdx.x & 31);
+    return;
+  }
+  const int nw = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  int64_t per = (len + nw - 1) / nw;
+  per = (per + 127) & ~int64_t(127);
+  const int64_t a = lo + (int64_t)w * per, b = min(a + per, lo + len);
+  if (X.single) seg_range<UNPACK, true, POL>(P, a, b, lane);
+  else seg_range<UNPACK, false, POL>(P, a, b, lane);
+}
+
+__global__ void __launch_bounds__(256) k_xfer(const __grid_constant__ XArgs A) {
+  extern __shared__ int32_t wt[];
+  __shared__ uint64_t s_val;
+  __shared__ int s_stop;
+  int op = 0;
+  for (int i = 0; i < A.nops; i++)
+    if ((int)blockIdx.x >= A.ops[i].cta0 && (int)blockIdx.x < A.ops[i].cta0 + A.ops[i].ncta) op = i;
+  const XOp& X = A.ops[op];
+  const int j = (int)blockIdx.x - X.cta0;
+  if (X.kind == 2)
+    for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
+  const int64_t C = X.chunk;
+  const int D = X.depth;
+  if (threadIdx.x == 0) s_stop = 0;
+  __syncthreads();
+
+  int64_t n = X.n;
+  if (X.role == 0) {
+    // ---- send role: header, wait for "go" (receiver-driven, [L20:c3973])
+    if (j == 0 && threadIdx.x == 0) {
+      st_release_sys(X.hdr + 1, (uint64_t)n);
+      st_release_sys(X.hdr, X.seq);
+    }
+    if (threadIdx.x == 0) {
+      uint64_t v = 0;
+      const uint64_t seq = X.seq;
+      bool ok = spin(X.go, [seq](uint64_t x) { return (x & ~kAbort) >= seq; }, A.timeout_ns, X.err, &v);
+      s_stop = !ok ? 2 : (v & kAbort) ? 1 : 0;
+      if (s_stop == 1 && j == 0) atomicCAS(X.err, 0, XERR_TRUNCATE);
+    }
+    __syncthreads();
+    if (s_stop) {
+      if (s_stop == 1 && j == 0 && (int)threadIdx.x < D) X.base_out[threadIdx.x] = X.base_in[threadIdx.x];
+      return;
+    }
+  } else {
+    // ---- recv role: read the header, check capacity, send "go"
+    if (threadIdx.x == 0) {
+      uint64_t v = 0;
+      const uint64_t seq = X.seq;
+      bool ok = spin(X.hdr, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v);
+      s_val = ok ? ld_acquire_sys(X.hdr + 1) : 0;
+      s_stop = ok ? 0 : 1;
+    }
+    __syncthreads();
+    if (s_stop) return;
+    n = (int64_t)s_val;
+    if (n > X.n) {
+      if (j == 0 && threadIdx.x == 0) {
+        atomicCAS(X.err, 0, XERR_TRUNCATE);
+        st_release_sys(X.go, X.seq | kAbort);
+      }
+      if (j == 0 && (int)threadIdx.x < D) X.base_out[threadIdx.x] = X.base_in[threadIdx.x];
+      return;
+    }
+    if (j == 0 && threadIdx.x == 0) st_release_sys(X.go, X.seq);
+  }
+
+  const int64_t K = (n + C - 1) / C;
+  for (int64_t k = 0; k < K; k++) {
+    const int slot = (int)(k % D);
+    const int64_t round = k / D;
+    const int64_t clen = min(C, n - k * C);
+    int64_t sub = (clen + X.ncta - 1) / X.ncta;
+    sub = (sub + 511) & ~int64_t(511);
+    const int64_t lo = (int64_t)j * sub;
+    if (lo >= clen) continue;
+    const int64_t len = min(sub, clen - lo);
+    uint8_t* sl = X.ring + (int64_t)slot * C - k * C;  // so that stream byte k*C lands at slot start
+    const uint64_t base = X.base_in[slot] + (uint64_t)round * (uint64_t)C;
+    if (threadIdx.x == 0) {
+      uint64_t v;
+      bool ok;
+      if (X.role == 0) ok = spin(X.ack + slot, [base](uint64_t x) { return x >= base; }, A.timeout_ns, X.err, &v);
+      else {
+        const uint64_t need = base + (uint64_t)clen;
+        ok = spin(X.ready + slot, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v);
+      }
+      s_stop = ok ? 0 : 1;
+    }
+    __syncthreads();
+    if (s_stop) return;
+    if (X.role == 0) cta_chunk<false>(X, X.P, sl, k * C + lo, len, wt);
+    else cta_chunk<true>(X, X.P, sl, k * C + lo, len, wt);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence_system();
+      red_release_sys_add(X.role == 0 ? X.ready + slot : X.ack + slot, (uint64_t)len);
+    }
+  }
+  // cumulative per-slot bytes after this message (read by the next message's kernel)
+  if (j == 0 && (int)threadIdx.x < D) {
+    const int s = threadIdx.x;
+    uint64_t add = 0;
+    for (int64_t k = s; k < K; k += D) add += (uint64_t)min(C, n - k * C);
+    X.base_out[s] = X.base_in[s] + add;
+  }
+}
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+typedef struct { char internal[128]; } ncclUniqueId_t;
+typedef void* ncclComm_t;
+struct Nccl {
+  void* h = nullptr;
+  int (*GetUniqueId)(ncclUniqueId_t*) = nullptr;
+  int (*CommInitRank)(ncclComm_t*, int, ncclUniqueId_t, int) = nullptr;
+  int (*Send)(const void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+  int (*Recv)(void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+  int (*GroupStart)() = nullptr;
+  int (*GroupEnd)() = nullptr;
+  int (*CommDestroy)(ncclComm_t) = nullptr;
+  const char* (*GetErrorString)(int) = nullptr;
+};
+static Nccl g_nccl;
+static std::mutex g_nccl_mu;
+
+static bool load_nccl() {
+  std::lock_guard<std::mutex> g(g_nccl_mu);
+  if (g_nccl.h) return true;
+  const char* names[] = {"libnccl.so.2", "libnccl.so", nullptr};
+  void* h = nullptr;
+  // prefer the copy torch already loaded (same SONAME), else the pip wheel's, else the system one
+  for (int i = 0; names[i] && !h; i++) h = dlopen(names[i], RTLD_NOW | RTLD_NOLOAD);
+  if (!h && getenv("DT_NCCL_LIB")) h = dlopen(getenv("DT_NCCL_LIB"), RTLD_NOW);
+  for (int i = 0; names[i] && !h; i++) h = dlopen(names[i], RTLD_NOW);
+  if (!h) return false;
+#define SYM(f, n) g_nccl.f = (decltype(g_nccl.f))dlsym(h, n)
+  SYM(GetUniqueId, "ncclGetUniqueId");
+  SYM(CommInitRank, "ncclCommInitRank");
+  SYM(Send, "ncclSend");
+  SYM(Recv, "ncclRecv");
+  SYM(GroupStart, "ncclGroupStart");
+  SYM(GroupEnd, "ncclGroupEnd");
+  SYM(CommDestroy, "ncclCommDestroy");
+  SYM(GetErrorString, "ncclGetErrorString");
+#undef SYM
+  if (!g_nccl.GetUniqueId || !g_nccl.CommInitRank || !g_nccl.Send || !g_nccl.Recv || !g_nccl.GroupStart ||
+      !g_nccl.GroupEnd || !g_nccl.CommDestroy)
+    return false;
+  g_nccl.h = h;
+  return true;
+}
+
+}  // namespace dt
+
+using namespace dt;
+
+// ------------------------------------------------------------------ comm object
+struct HandleBlob {
+  uint32_t magic;
+  int32_t rank;
+  int64_t pid;
+  int32_t device;
+  int32_t pad;
+  uint64_t ring_ptr, flags_ptr;
+  cudaIpcMemHandle_t ring_h, flags_h;
+};
+static const uint32_t kMagic = 0xD7A7C0DEu;
+
+struct PendingOp {
+  const void* sbuf;
+  int64_t scount;
+  dt_t stype;
+  int dest;
+  void* rbuf;
+  int64_t rcount;
+  dt_t rtype;
+  int source;
+};
+
+struct dt_comm_s {
+  int rank = 0, nranks = 1, device = 0;
+  dt_xfer_opts o{};
+  int nch = kMaxCh;
+  uint8_t* ring = nullptr;
+  uint64_t* flags = nullptr;
+  uint64_t* bases = nullptr;  // [2 parities][2 dirs][nranks][nch][depth]
+  size_t ring_bytes = 0, flag_words = 0;
+  std::vector<uint8_t*> peer_ring;
+  std::vector<uint64_t*> peer_flags;
+  std::vector<bool> opened;
+  bool connected = false;
+  std::vector<uint64_t> send_seq, recv_seq;  // [nranks*nch]
+  // group
+  bool in_group = false;
+  std::vector<PendingOp> pending;
+  // NCCL mode
+  ncclComm_t nccl = nullptr;
+  cudaStream_t s_pack = nullptr, s_net = nullptr, s_unpack = nullptr;
+  std::vector<cudaEvent_t> ev;
+  uint8_t* stage = nullptr;  // send staging [kMaxOps][depth][chunk]
+  uint8_t* rstage = nullptr; // recv staging
+  int64_t* szbuf = nullptr;  // device size handshake buffers [2][kMaxOps]
+  int64_t* szhost = nullptr; // pinned
+  // layout helpers
+  size_t ready_idx(int src, int ch, int slot) const { return ((size_t)src * nch + ch) * o.depth + slot; }
+  size_t hdr_idx(int src, int ch) const { return (size_t)nranks * nch * o.depth + ((size_t)src * nch + ch) * 2; }
+  size_t ack_idx(int dst, int ch, int slot) const {
+    return (size_t)nranks * nch * (o.depth + 2) + ((size_t)dst * nch + ch) * o.depth + slot;
+  }
+  size_t go_idx(int dst, int ch) const { return (size_t)nranks * nch * (2 * o.depth + 2) + (size_t)dst * nch + ch; }
+  size_t err_idx() const { return (size_t)nranks * nch * (2 * o.depth + 3); }
+  size_t ring_off(int src, int ch) const { return (((size_t)src * nch + ch) * o.depth) * (size_t)o.chunk_bytes; }
+  uint64_t* base(int parity, int dir, int peer, int ch) const {
+    return bases + ((((size_t)parity * 2 + dir) * nranks + peer) * nch + ch) * o.depth;
+  }
+};
+
+static dt_status cufail(cudaError_t e, const char* what) {
+  set_error("%s: %s", what, cudaGetErrorString(e));
+  return DT_ERR_CUDA;
+}
+#define CU(call)                                      \
+  do {                                                \
+    cudaError_t _e = (call);                          \
+    if (_e != cudaSuccess) return cufail(_e, #call);  \
+  } while (0)
+#define NC(call)                                                                         \
+  do {                                                                                   \
+    int _r = (call);                                                                     \
+    if (_r != 0) {                                                                       \
+      set_error("%s: nccl error %d (%s)", #call, _r,                                     \
+                g_nccl.GetErrorString ? g_nccl.GetErrorString(_r) : "?");                \
+      return DT_ERR_NCCL;                                                                \
+    }                                                                                    \
+  } while (0)
+
+static void fill_opts(dt_xfer_opts& o, const dt_xfer_opts* in) {
+  o.chunk_bytes = 1 << 20;
+  o.depth = 4;
+  o.mode = DT_XFER_P2P;
+  o.ctas = 0;
+  o.reserved = 0;
+  if (in) {
+    if (in->chunk_bytes > 0) o.chunk_bytes = in->chunk_bytes;
+    if (in->depth > 0) o.depth = in->depth;
+    o.mode = in->mode;
+    o.ctas = in->ctas;
+  }
+  o.chunk_bytes = (o.chunk_bytes + 511) & ~int64_t(511);
+}
+
+extern "C" {
+
+dt_status dt_nccl_unique_id(void* out128) {
+  if (!out128) {
+    set_error("dt_nccl_unique_id: NULL");
+    return DT_ERR_ARG;
+  }
+  if (!load_nccl()) {
+    set_error("NCCL library not found");
+    return DT_ERR_NCCL;
+  }
+  ncclUniqueId_t id;
+  NC(g_nccl.GetUniqueId(&id));
+  std::memcpy(out128, &id, 128);
+  return DT_OK;
+}
+
+dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int device, const dt_xfer_opts* o,
+                       dt_comm_t* out) {
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks || device < 0) {
+    set_error("dt_comm_init: bad argument");
+    return DT_ERR_ARG;
+  }
+  auto* c = new dt_comm_s;
+  c->rank = rank;
+  c->nranks = nranks;
+  c->device = device;
+  fill_opts(c->o, o);
+  if (c->o.mode != DT_XFER_P2P && c->o.mode != DT_XFER_NCCL) {
+    delete c;
+    set_error("dt_comm_init: unknown mode");
+    return DT_ERR_ARG;
+  }
+  cudaError_t e = cudaSetDevice(device);
+  if (e != cudaSuccess) {
+    delete c;
+    return cufail(e, "cudaSetDevice");
+  }
+  c->ring_bytes = (size_t)nranks * c->nch * c->o.depth * (size_t)c->o.chunk_bytes;
+  c->flag_words = c->err_idx() + 1;
+  if (c->o.mode == DT_XFER_P2P) {
+    e = cudaMalloc(&c->ring, c->ring_bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&c->flags, c->flag_words * 8);
+    if (e == cudaSuccess) e = cudaMemset(c->flags, 0, c->flag_words * 8);
+    const size_t nb = (size_t)2 * 2 * nranks * c->nch * c->o.depth;
+    if (e == cudaSuccess) e = cudaMalloc(&c->bases, nb * 8);
+    if (e == cudaSuccess) e = cudaMemset(c->bases, 0, nb * 8);
+    if (e != cudaSuccess) {
+      cudaFree(c->ring);
+      cudaFree(c->flags);
+      cudaFree(c->bases);
+      delete c;
+      return cufail(e, "dt_comm_init alloc");
+    }
+  } else {
+    if (!load_nccl()) {
+      delete c;
+      set_error("dt_comm_init: NCCL library not found");
+      return DT_ERR_NCCL;
+    }
+    if (!nccl_unique_id) {
+      delete c;
+      set_error("dt_comm_init: NCCL mode needs a unique id");
+      return DT_ERR_ARG;
+    }
+    ncclUniqueId_t id;
+    std::memcpy(&id, nccl_unique_id, 128);
+    int r = g_nccl.CommInitRank(&c->nccl, nranks, id, rank);
+    if (r != 0) {
+      delete c;
+      set_error("ncclCommInitRank failed: %d", r);
+      return DT_ERR_NCCL;
+    }
+    const size_t st = (size_t)kMaxOps * c->o.depth * (size_t)c->o.chunk_bytes;
+    e = cudaMalloc(&c->stage, st);
+    if (e == cudaSuccess) e = cudaMalloc(&c->rstage, st);
+    if (e == cudaSuccess) e = cudaMalloc(&c->szbuf, sizeof(int64_t) * 2 * kMaxOps);
+    if (e == cudaSuccess) e = cudaMallocHost(&c->szhost, sizeof(int64_t) * 2 * kMaxOps);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s_pack, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s_net, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s_unpack, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+      delete c;
+      return cufail(e, "dt_comm_init nccl alloc");
+    }
+    c->ev.resize((size_t)kMaxOps * c->o.depth * 3 + 2);
+    for (auto& x : c->ev) cudaEventCreateWithFlags(&x, cudaEventDisableTiming);
+  }
+  c->peer_ring.assign(nranks, nullptr);
+  c->peer_flags.assign(nranks, nullptr);
+  c->opened.assign(nranks, false);
+  c->send_seq.assign((size_t)nranks * c->nch, 0);
+  c->recv_seq.assign((size_t)nranks * c->nch, 0);
+  c->peer_ring[rank] = c->ring;
+  c->peer_flags[rank] = c->flags;
+  if (nranks == 1 || c->o.mode == DT_XFER_NCCL) c->connected = true;
+  *out = c;
+  return DT_OK;
+}
+
+dt_status dt_comm_local_handle(dt_comm_t c, void* out, size_t* nbytes) {
+  if (!c || !nbytes) {
+    set_error("dt_comm_local_handle: NULL");
+    return DT_ERR_ARG;
+  }
+  if (!out || *nbytes < sizeof(HandleBlob)) {
+    *nbytes = sizeof(HandleBlob);
+    if (!out) return DT_OK;
+    set_error("dt_comm_local_handle: buffer too small");
+    return DT_ERR_ARG;
+  }
+  HandleBlob b;
+  std::memset(&b, 0, sizeof(b));
+  b.magic = kMagic;
+  b.rank = c->rank;
+  b.pid = (int64_t)getpid();
+  b.device = c->device;
+  b.ring_ptr = (uint64_t)(uintptr_t)c->ring;
+  b.flags_ptr = (uint64_t)(uintptr_t)c->flags;
+  if (c->o.mode == DT_XFER_P2P) {
+    CU(cudaIpcGetMemHandle(&b.ring_h, c->ring));
+    CU(cudaIpcGetMemHandle(&b.flags_h, c->flags));
+  }
+  std::memcpy(out, &b, sizeof(b));
+  *nbytes = sizeof(b);
+  return DT_OK;
+}
+
+dt_status dt_comm_connect(dt_comm_t c, const void* all, size_t per) {
+  if (!c || !all || per < sizeof(HandleBlob)) {
+    set_error("dt_comm_connect: bad argument");
+    return DT_ERR_ARG;
+  }
+  if (c->o.mode != DT_XFER_P2P) {
+    c->connected = true;
+    return DT_OK;
+  }
+  CU(cudaSetDevice(c->device));
+  const int64_t mypid = (int64_t)getpid();
+  for (int r = 0; r < c->nranks; r++) {
+    HandleBlob b;
+    std::memcpy(&b, (const uint8_t*)all + (size_t)r * per, sizeof(b));
+    if (b.magic != kMagic || b.rank != r) {
+      set_error("dt_comm_connect: malformed handle of rank %d", r);
+      return DT_ERR_ARG;
+    }
+    if (r == c->rank) continue;
+    if (b.pid == mypid) {  // same process (e.g. several devices driven by one process)
+      c->peer_ring[r] = (uint8_t*)(uintptr_t)b.ring_ptr;
+      c->peer_flags[r] = (uint64_t*)(uintptr_t)b.flags_ptr;
+      if (b.device != c->device) {
+        cudaError_t e = cudaDeviceEnablePeerAccess(b.device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cufail(e, "cudaDeviceEnablePeerAccess");
+        cudaGetLastError();
+      }
+      continue;
+    }
+    void *pr = nullptr, *pf = nullptr;
+    CU(cudaIpcOpenMemHandle(&pr, b.ring_h, cudaIpcMemLazyEnablePeerAccess));
+    CU(cudaIpcOpenMemHandle(&pf, b.flags_h, cudaIpcMemLazyEnablePeerAccess));
+    c->peer_ring[r] = (uint8_t*)pr;
+    c->peer_flags[r] = (uint64_t*)pf;
+    c->opened[r] = true;
+  }
+  c->connected = true;
+  return DT_OK;
+}
+
+dt_status dt_group_start(dt_comm_t c) {
+  if (!c) {
+    set_error("dt_group_start: NULL");
+    return DT_ERR_ARG;
+  }
+  c->in_group = true;
+  c->pending.clear();
+  return DT_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------ issue
+static int64_t lowp2u(uint64_t x) {
+  if (x == 0) return 16;
+  int64_t g = (int64_t)(x & (~x + 1));
+  return g > 16 ? 16 : g;
+}
+
+// Fill the pack/unpack params of one side of an op (no chunk-specific fields).
+static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbytes, int64_t chunk, XOp& X) {
+  DeviceDesc* dd = nullptr;
+  dt_status st = ensure_committed_on_device(t, &dd);
+  if (st != DT_OK) return st;
+  const Form& f = get_form(t);
+  KLevels L;
+  build_levels(f, dd, t, count, L);
+  KP& P = X.P;
+  std::memset(&P, 0, sizeof(P));
+  P.nc = (const uint8_t*)nc;
+  P.tsize = f.tsize();
+  P.nblocks = (int64_t)f.bl.size();
+  P.bd = dd->bd;
+  P.bl = dd->bl;
+  P.boff = dd->boff;
+  P.bd0 = f.bd.empty() ? 0 : f.bd[0];
+  P.bl0 = f.bl.empty() ? 0 : f.bl[0];
+  P.nlev = L.n;
+  for (int i = 0; i < L.n; i++) {
+    P.cnt[i] = L.cnt[i];
+    P.stride[i] = L.stride[i];
+    P.table[i] = L.table[i];
+    P.fcnt[i] = make_fd((uint64_t)L.cnt[i]);
+  }
+  P.ftsize = make_fd((uint64_t)P.tsize);
+  int64_t g = 1;
+  // chunk starts are multiples of `chunk` (a multiple of 512) and ring slots are aligned
+  int kind = plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
+  if (kind == 2 && lowp2u((uint64_t)chunk) < g) kind = 1;
+  X.kind = kind == 2 ? 2 : 1;
+  X.single = P.nblocks == 1;
+  X.g = (int32_t)g;
+  if (X.kind == 2) {
+    const int32_t* wt = nullptr;
+    st = ensure_wtab_pub(f, *dd, g, &wt);
+    if (st != DT_OK) return st;
+    P.wtab = wt;
+    P.nwords = (int32_t)(f.tsize() / g);
+  }
+  return DT_OK;
+}
+
+static int default_ctas(const dt_comm_s* c) { return c->o.ctas > 0 ? c->o.ctas : 16; }
+
+static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cudaStream_t s) {
+  XArgs A;
+  std::memset(&A, 0, sizeof(A));
+  const char* to = getenv("DT_TIMEOUT_MS");
+  A.timeout_ns = (int64_t)(to ? atoll(to) : 30000) * 1000000ll;
+  int nops = 0, cta = 0;
+  size_t smem = 0;
+  std::vector<int> sch(c->nranks, 0), rch(c->nranks, 0);
+  const int G = default_ctas(c);
+  for (const auto& p : ops) {
+    if (p.dest >= 0) {
+      if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
+      const int ch = sch[p.dest]++;
+      if (ch >= c->nch) { set_error("dt_sendrecv: more than %d messages to one peer in a group", c->nch); return DT_ERR_UNSUPPORTED; }
+      XOp& X = A.ops[nops++];
+      const int64_t n = p.scount * p.stype->size;
+      dt_status st = side_params(p.stype, p.scount, p.sbuf, n, c->o.chunk_bytes, X);
+      if (st != DT_OK) return st;
+      X.role = 0;
+      X.n = n;
+      X.chunk = c->o.chunk_bytes;
+      X.depth = c->o.depth;
+      X.cta0 = cta;
+      X.ncta = G;
+      cta += G;
+      uint64_t* pf = c->peer_flags[p.dest];
+      X.ring = c->peer_ring[p.dest] + c->ring_off(c->rank, ch);
+      X.ready = pf + c->ready_idx(c->rank, ch, 0);
+      X.hdr = pf + c->hdr_idx(c->rank, ch);
+      X.ack = c->flags + c->ack_idx(p.dest, ch, 0);
+      X.go = c->flags + c->go_idx(p.dest, ch);
+      uint64_t& sq = c->send_seq[(size_t)p.dest * c->nch + ch];
+      const int par = (int)(sq & 1);
+      X.base_in = c->base(par, 0, p.dest, ch);
+      X.base_out = c->base(par ^ 1, 0, p.dest, ch);
+      X.seq = ++sq;
+      X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
+      if (X.kind == 2) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+    }
+    if (p.source >= 0) {
+      if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
+      const int ch = rch[p.source]++;
+      if (ch >= c->nch) { set_error("dt_sendrecv: more than %d messages from one peer in a group", c->nch); return DT_ERR_UNSUPPORTED; }
+      XOp& X = A.ops[nops++];
+      const int64_t cap = p.rcount * p.rtype->size;
+      dt_status st = side_params(p.rtype, p.rcount, p.rbuf, cap, c->o.chunk_bytes, X);
+      if (st != DT_OK) return st;
+      X.role = 1;
+      X.n = cap;
+      X.chunk = c->o.chunk_bytes;
+      X.depth = c->o.depth;
+      X.cta0 = cta;
+      X.ncta = G;
+      cta += G;
+      uint64_t* pf = c->peer_flags[p.source];
+      X.ring = c->ring + c->ring_off(p.source, ch);
+      X.ready = c->flags + c->ready_idx(p.source, ch, 0);
+      X.hdr = c->flags + c->hdr_idx(p.source, ch);
+      X.ack = pf + c->ack_idx(c->rank, ch, 0);
+      X.go = pf + c->go_idx(c->rank, ch);
+      uint64_t& sq = c->recv_seq[(size_t)p.source * c->nch + ch];
+      const int par = (int)(sq & 1);
+      X.base_in = c->base(par, 1, p.source, ch);
+      X.base_out = c->base(par ^ 1, 1, p.source, ch);
+      X.seq = ++sq;
+      X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
+      if (X.kind == 2) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+    }
+  }
+  if (nops == 0) return DT_OK;
+  A.nops = nops;
+  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
+  void* args[] = {&A};
+  CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(256), args, smem, s));
+  return DT_OK;
+}
+
+// NCCL mode: size handshake, then per chunk round: pack -> send/recv -> unpack,
+// double-buffered over `depth` staging slots on three internal streams.
+static dt_status issue_nccl(dt_comm_s* c, const std::vector<PendingOp>& ops, cudaStream_t s) {
+  const int64_t C = c->o.chunk_bytes;
+  const int D = c->o.depth;
+  std::vector<const PendingOp*> sends, recvs;
+  for (const auto& p : ops) {
+    if (p.dest >= 0) sends.push_back(&p);
+    if (p.source >= 0) recvs.push_back(&p);
+  }
+  if ((int)sends.size() > kMaxOps || (int)recvs.size() > kMaxOps) {
+    set_error("dt_sendrecv: too many ops in one group");
+    return DT_ERR_UNSUPPORTED;
+  }
+  // handshake: exchange byte counts (the receiver learns n, checks capacity)
+  for (size_t i = 0; i < sends.size(); i++) c->szhost[i] = sends[i]->scount * sends[i]->stype->size;
+  CU(cudaMemcpyAsync(c->szbuf, c->szhost, sizeof(int64_t) * sends.size(), cudaMemcpyHostToDevice, s));
+  NC(g_nccl.GroupStart());
+  for (size_t i = 0; i < sends.size(); i++) NC(g_nccl.Send(c->szbuf + i, 8, 1 /*uint8*/, sends[i]->dest, c->nccl, s));
+  for (size_t i = 0; i < recvs.size(); i++)
+    NC(g_nccl.Recv(c->szbuf + kMaxOps + i, 8, 1, recvs[i]->source, c->nccl, s));
+  NC(g_nccl.GroupEnd());
+  CU(cudaMemcpyAsync(c->szhost + kMaxOps, c->szbuf + kMaxOps, sizeof(int64_t) * recvs.size(),
+                     cudaMemcpyDeviceToHost, s));
+  CU(cudaStreamSynchronize(s));
+  std::vector<int64_t> sn(sends.size()), rn(recvs.size());
+  for (size_t i = 0; i < sends.size(); i++) sn[i] = c->szhost[i];
+  for (size_t i = 0; i < recvs.size(); i++) {
+    rn[i] = c->szhost[kMaxOps + i];
+    if (rn[i] > recvs[i]->rcount * recvs[i]->rtype->size) {
+      set_error("dt_sendrecv: message of %lld bytes truncated by a %lld-byte receive", (long long)rn[i],
+                (long long)(recvs[i]->rcount * recvs[i]->rtype->size));
+      return DT_ERR_TRUNCATE;
+    }
+  }
+  int64_t K = 0;
+  for (auto x : sn) K = std::max(K, (x + C - 1) / C);
+  for (auto x : rn) K = std::max(K, (x + C - 1) / C);
+  cudaEvent_t* ev = c->ev.data();
+  auto ev_packed = [&](int slot) { return ev[slot]; };
+  auto ev_net = [&](int slot) { return ev[D + slot]; };
+  auto ev_unpacked = [&](int slot) { return ev[2 * D + slot]; };
+  cudaEvent_t ev_start = ev[3 * D], ev_end = ev[3 * D + 1];
+  CU(cudaEventRecord(ev_start, s));
+  CU(cudaStreamWaitEvent(c->s_pack, ev_start, 0));
+  CU(cudaStreamWaitEvent(c->s_net, ev_start, 0));
+  CU(cudaStreamWaitEvent(c->s_unpack, ev_start, 0));
+  const size_t slot_span = (size_t)kMaxOps * C;
+  for (int64_t k = 0; k < K; k++) {
+    const int slot = (int)(k % D);
+    if (k >= D) CU(cudaStreamWaitEvent(c->s_pack, ev_net(slot), 0));  // staging slot sent
+    for (size_t i = 0; i < sends.size(); i++) {
+      int64_t pos = k * C, len = std::min<int64_t>(C, sn[i] - pos);
+      if (len <= 0) continue;
+      dt_status st = dt_pack(sends[i]->stype, sends[i]->scount, sends[i]->sbuf, c->stage + slot * slot_span + i * C,
+                             pos, &len, c->s_pack);
+      if (st != DT_OK) return st;
+    }
+    CU(cudaEventRecord(ev_packed(slot), c->s_pack));
+    CU(cudaStreamWaitEvent(c->s_net, ev_packed(slot), 0));
+    if (k >= D) CU(cudaStreamWaitEvent(c->s_net, ev_unpacked(slot), 0));  // receive slot free
+    NC(g_nccl.GroupStart());
+    for (size_t i = 0; i < sends.size(); i++) {
+      int64_t len = std::min<int64_t>(C, sn[i] - k * C);
+      if (len > 0) NC(g_nccl.Send(c->stage + slot * slot_span + i * C, (size_t)len, 1, sends[i]->dest, c->nccl, c->s_net));
+    }
+    for (size_t i = 0; i < recvs.size(); i++) {
+      int64_t len = std::min<int64_t>(C, rn[i] - k * C);
+      if (len > 0)
+        NC(g_nccl.Recv(c->rstage + slot * slot_span + i * C, (size_t)len, 1, recvs[i]->source, c->nccl, c->s_net));
+    }
+    NC(g_nccl.GroupEnd());
+    CU(cudaEventRecord(ev_net(slot), c->s_net));
+    CU(cudaStreamWaitEvent(c->s_unpack, ev_net(slot), 0));
+    for (size_t i = 0; i < recvs.size(); i++) {
+      int64_t pos = k * C, len = std::min<int64_t>(C, rn[i] - pos);
+      if (len <= 0) continue;
+      dt_status st = dt_unpack(recvs[i]->rtype, recvs[i]->rcount, c->rstage + slot * slot_span + i * C,
+                               recvs[i]->rbuf, pos, &len, c->s_unpack);
+      if (st != DT_OK) return st;
+    }
+    CU(cudaEventRecord(ev_unpacked(slot), c->s_unpack));
+  }
+  // join: the caller's stream waits for all three internal streams
+  CU(cudaEventRecord(ev_end, c->s_pack));
+  CU(cudaStreamWaitEvent(s, ev_end, 0));
+  CU(cudaEventRecord(ev_end, c->s_net));
+  CU(cudaStreamWaitEvent(s, ev_end, 0));
+  CU(cudaEventRecord(ev_end, c->s_unpack));
+  CU(cudaStreamWaitEvent(s, ev_end, 0));
+  return DT_OK;
+}
+
+static dt_status validate(dt_comm_s* c, const PendingOp& p) {
+  if (p.dest >= c->nranks || p.source >= c->nranks || p.dest < -1 || p.source < -1) {
+    set_error("dt_sendrecv: rank out of range");
+    return DT_ERR_ARG;
+  }
+  if (p.dest >= 0) {
+    if (!p.stype || p.scount < 0 || (!p.sbuf && p.scount * p.stype->size > 0)) {
+      set_error("dt_sendrecv: bad send arguments");
+      return DT_ERR_ARG;
+    }
+    if (!p.stype->committed) {
+      set_error("dt_sendrecv: send type not committed");
+      return DT_ERR_NOT_COMMITTED;
+    }
+  }
+  if (p.source >= 0) {
+    if (!p.rtype || p.rcount < 0 || (!p.rbuf && p.rcount * p.rtype->size > 0)) {
+      set_error("dt_sendrecv: bad receive arguments");
+      return DT_ERR_ARG;
+    }
+    if (!p.rtype->committed) {
+      set_error("dt_sendrecv: receive type not committed");
+      return DT_ERR_NOT_COMMITTED;
+    }
+  }
+  if (!c->connected) {
+    set_error("dt_sendrecv: dt_comm_connect() not called");
+    return DT_ERR_ARG;
+  }
+  return DT_OK;
+}
+
+static dt_status issue(dt_comm_s* c, const std::vector<PendingOp>& ops, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  if (c->o.mode == DT_XFER_NCCL) return issue_nccl(c, ops, s);
+  return issue_p2p(c, ops, s);
+}
+
+extern "C" {
+
+dt_status dt_sendrecv(const void* sbuf, int64_t scount, dt_t stype, int dest, void* rbuf, int64_t rcount, dt_t rtype,
+                      int source, dt_comm_t c, const dt_xfer_opts* o, void* stream) {
+  if (!c) {
+    set_error("dt_sendrecv: NULL comm");
+    return DT_ERR_ARG;
+  }
+  if (o && ((o->chunk_bytes > 0 && ((o->chunk_bytes + 511) & ~int64_t(511)) != c->o.chunk_bytes) ||
+            (o->depth > 0 && o->depth != c->o.depth) || o->mode != c->o.mode)) {
+    set_error("dt_sendrecv: opts differ from the comm's (chunk/depth/mode are fixed at dt_comm_init)");
+    return DT_ERR_UNSUPPORTED;
+  }
+  PendingOp p{sbuf, scount, stype, dest, rbuf, rcount, rtype, source};
+  dt_status st = validate(c, p);
+  if (st != DT_OK) return st;
+  if (c->in_group) {
+    c->pending.push_back(p);
+    return DT_OK;
+  }
+  std::vector<PendingOp> one{p};
+  return issue(c, one, stream);
+}
+
+dt_status dt_group_end(dt_comm_t c, void* stream) {
+  if (!c || !c->in_group) {
+    set_error("dt_group_end: no open group");
+    return DT_ERR_ARG;
+  }
+  c->in_group = false;
+  std::vector<PendingOp> ops;
+  ops.swap(c->pending);
+  return issue(c, ops, stream);
+}
+
+dt_status dt_comm_check(dt_comm_t c) {
+  if (!c) {
+    set_error("dt_comm_check: NULL");
+    return DT_ERR_ARG;
+  }
+  if (!c->flags) return DT_OK;
+  int32_t e = 0;
+  CU(cudaMemcpy(&e, c->flags + c->err_idx(), sizeof(e), cudaMemcpyDeviceToHost));
+  if (e == 0) return DT_OK;
+  int32_t z = 0;
+  CU(cudaMemcpy(c->flags + c->err_idx(), &z, sizeof(z), cudaMemcpyHostToDevice));
+  if (e == XERR_TRUNCATE) {
+    set_error("dt_sendrecv: receive capacity smaller than the message (truncation)");
+    return DT_ERR_TRUNCATE;
+  }
+  set_error("dt_sendrecv: device-side wait for a peer flag timed out");
+  return DT_ERR_TIMEOUT;
+}
+
+dt_status dt_comm_free(dt_comm_t* pc) {
+  if (!pc || !*pc) {
+    set_error("dt_comm_free: NULL");
+    return DT_ERR_ARG;
+  }
+  dt_comm_s* c = *pc;
+  cudaSetDevice(c->device);
+  for (int r = 0; r < c->nranks; r++) {
+    if (!c->opened[r]) continue;
+    cudaIpcCloseMemHandle(c->peer_ring[r]);
+    cudaIpcCloseMemHandle(c->peer_flags[r]);
+  }
+  cudaFree(c->ring);
+  cudaFree(c->flags);
+  cudaFree(c->bases);
+  cudaFree(c->stage);
+  cudaFree(c->rstage);
+  cudaFree(c->szbuf);
+  if (c->szhost) cudaFreeHost(c->szhost);
+  for (auto e : c->ev) cudaEventDestroy(e);
+  if (c->s_pack) cudaStreamDestroy(c->s_pack);
+  if (c->s_net) cudaStreamDestroy(c->s_net);
+  if (c->s_unpack) cudaStreamDestroy(c->s_unpack);
+  if (c->nccl && g_nccl.CommDestroy) g_nccl.CommDestroy(c->nccl);
+  delete c;
+  *pc = nullptr;
+  return DT_OK;
+}
+
+}  // extern "C"

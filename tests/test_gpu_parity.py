@@ -1,0 +1,244 @@
+"""GPU parity (T2): libdt's CUDA pack/unpack vs the CPU oracle, byte for byte.
+
+Bit-exact is the bar (pure byte movement; sources are splitmix64 words, so NaN
+payloads and signed zeros must survive).  Destinations are poisoned 0xA5 with
+4 KiB guard zones on both sides; unpack must leave every byte outside the
+typemap untouched.  Workloads: SURVEY §8(d) configs C1-C5 (paper: V [L22:c1966],
+T [L22:c2839], SHOC-style faces [L14:c1929], LAMMPS-style index lists
+[L14:c2154]) at full size, plus random tiny types with ragged pos/len splits
+and misaligned origins (prologue/epilogue [L16:c3618 §3.1]).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from workloads import (c1_submatrix, c2_lower_triangle, c3_block_cyclic, c4_face, c5_particles, c5b_irregular,
+                       fill_bytes, stair_triangle, upper_triangle)
+
+pytestmark = pytest.mark.gpu
+
+GUARD = 4096
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    torch.cuda.init()
+    return torch
+
+
+def _dev(torch, host: np.ndarray):
+    return torch.from_numpy(np.ascontiguousarray(host)).cuda()
+
+
+def _poisoned(torch, n):
+    return torch.full((n + 2 * GUARD,), 0xA5, dtype=torch.uint8, device="cuda")
+
+
+def check_pack_unpack(torch, recipe, origin, parent, count=1, pos=0, nbytes=None, seed=1, origin_pad=0):
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    ot = oracle.from_recipe(recipe)
+    t = dt.from_recipe(recipe).commit()
+    ext = ot.extent
+    span = parent + max(0, (count - 1) * ext)
+    org = origin + origin_pad
+    src_h = fill_bytes(span + origin_pad + 64, seed)
+    total = count * ot.size
+    n = max(0, min(total - pos, total if nbytes is None else nbytes))
+    exp = oracle.pack(ot, count, src_h, org, pos, n)
+    src_d = _dev(torch, src_h)
+    out = _poisoned(torch, n)
+    got_n = dt.pack(t, count, src_d, out.data_ptr() + GUARD, pos, n, origin_offset=org)
+    torch.cuda.synchronize()
+    assert got_n == n
+    o = out.cpu().numpy()
+    assert np.all(o[:GUARD] == 0xA5) and np.all(o[GUARD + n:] == 0xA5), "pack wrote outside its output"
+    assert np.array_equal(o[GUARD:GUARD + n], exp), "pack mismatch"
+    # unpack the oracle's bytes into a poisoned layout
+    dst_h = np.full(span + origin_pad + 64, 0xA5, dtype=np.uint8)
+    oracle.unpack(ot, count, exp, dst_h, org, pos)
+    dst_d = _poisoned(torch, len(dst_h))
+    pk = _dev(torch, exp) if n else torch.zeros(1, dtype=torch.uint8, device="cuda")
+    got_n = dt.unpack(t, count, pk, dst_d.data_ptr() + GUARD, pos, n, origin_offset=org)
+    torch.cuda.synchronize()
+    assert got_n == n
+    d = dst_d.cpu().numpy()
+    assert np.all(d[:GUARD] == 0xA5) and np.all(d[GUARD + len(dst_h):] == 0xA5), "unpack wrote outside the span"
+    assert np.array_equal(d[GUARD:GUARD + len(dst_h)], dst_h), "unpack mismatch"
+
+
+# ------------------------------------------------------------------ the paper's workloads at full size
+@pytest.mark.parametrize("r0c0", [(0, 0), (1, 1), (3, 7)])
+def test_c1_submatrix(torch_cuda, r0c0):
+    rec, org, parent = c1_submatrix(256, 1024, *r0c0)
+    check_pack_unpack(torch_cuda, rec, org, parent)
+
+
+def test_c2_lower_triangle_full(torch_cuda):
+    rec, org, parent = c2_lower_triangle(4096)
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=0x5EED0002)
+
+
+@pytest.mark.parametrize("n", [1, 2, 33, 1000])
+def test_triangles_small(torch_cuda, n):
+    for mk in (c2_lower_triangle, upper_triangle):
+        rec, org, parent = mk(n)
+        check_pack_unpack(torch_cuda, rec, org, parent)
+    rec, org, parent = stair_triangle(max(n, 64), 32)
+    check_pack_unpack(torch_cuda, rec, org, parent)
+
+
+def test_c3_block_cyclic_full(torch_cuda):
+    rec, org, parent = c3_block_cyclic(8192, 64)
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=0x5EED0003)
+
+
+@pytest.mark.parametrize("face", ["x-", "x+", "y-", "y+", "z-", "z+"])
+@pytest.mark.parametrize("ghost", [False, True])
+def test_c4_halo_faces_full(torch_cuda, face, ghost):
+    rec, org, parent = c4_face(face, 512, 1, ghost)
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=0x5EED0004)
+
+
+@pytest.mark.parametrize("m", [1 << 10, 1 << 16, 1 << 22, 1 << 26])
+def test_c5_particles(torch_cuda, m):
+    rec, org, parent = c5_particles(m)
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=0x5EED0005)
+
+
+@pytest.mark.parametrize("m", [1 << 10, 1 << 20])
+def test_c5b_irregular(torch_cuda, m):
+    rec, org, parent = c5b_irregular(m)
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=0x5EED0006)
+
+
+# ------------------------------------------------------------------ resume from a byte position
+@pytest.mark.parametrize("name", ["C1", "C2", "C4x", "C5"])
+def test_pos_len_fragments(torch_cuda, name):
+    mk = {"C1": lambda: c1_submatrix(64, 200, 1, 2), "C2": lambda: c2_lower_triangle(300),
+          "C4x": lambda: c4_face("x+", 40), "C5": lambda: c5_particles(56 * 500)}[name]
+    rec, org, parent = mk()
+    rng = np.random.default_rng(7)
+    size = oracle.from_recipe(rec).size
+    for count in (1, 2):
+        total = size * count
+        for _ in range(4):
+            a, b = sorted(rng.integers(0, total + 1, size=2))
+            check_pack_unpack(torch_cuda, rec, org, parent, count=count, pos=int(a), nbytes=int(b - a))
+
+
+def test_concatenated_fragments_equal_whole(torch_cuda):
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c2_lower_triangle(512)
+    t = dt.from_recipe(rec).commit()
+    src = _dev(torch, fill_bytes(parent, 3))
+    n = t.size
+    whole = torch.empty(n, dtype=torch.uint8, device="cuda")
+    dt.pack(t, 1, src, whole)
+    cuts = [0, 1, 7, 4096, 4097, 100000, n - 3, n]
+    parts = torch.empty(n, dtype=torch.uint8, device="cuda")
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        dt.pack(t, 1, src, parts.data_ptr() + a, a, b - a)
+    torch.cuda.synchronize()
+    assert torch.equal(whole, parts)
+
+
+# ------------------------------------------------------------------ random tiny types, misaligned origins
+def test_random_tiny_types(torch_cuda):
+    from tests.test_oracle_pins import _tiny_types
+    rng = np.random.default_rng(11)
+    tys = _tiny_types()
+    for i, r in enumerate(tys[::3]):
+        ot = oracle.from_recipe(r)
+        info = ot.info()
+        if info["size"] == 0:
+            continue
+        lo = min(0, info["true_lb"], info["true_lb"] + 2 * info["extent"])
+        hi = max(info["true_ub"], info["true_ub"] + 2 * info["extent"], 1)
+        count = int(rng.integers(1, 4))
+        total = count * info["size"]
+        a, b = sorted(rng.integers(0, total + 1, size=2))
+        # overlapping typemaps are only packed (unpack is rejected, reading A9)
+        try:
+            check_pack_unpack(torch_cuda, r, -lo + 16, hi - lo + 32, count=count, pos=int(a), nbytes=int(b - a),
+                              seed=i, origin_pad=int(rng.integers(0, 16)))
+        except Exception as e:  # noqa: BLE001
+            if "DT_ERR_OVERLAP" not in str(e):
+                raise
+
+
+def test_unpack_rejects_overlap(torch_cuda):
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    t = dt.Type.basic("INT32").vector(4, 3, 2).commit()    # stride < blocklen: overlapping
+    buf = torch.zeros(1024, dtype=torch.uint8, device="cuda")
+    pk = torch.zeros(t.size, dtype=torch.uint8, device="cuda")
+    dt.pack(t, 1, buf, pk)                                   # pack of an overlapping map is legal
+    with pytest.raises(dt.DTError) as e:
+        dt.unpack(t, 1, pk, buf)
+    assert e.value.name == "DT_ERR_OVERLAP"
+
+
+def test_host_pointer_rejected(torch_cuda):
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    t = dt.Type.basic("DOUBLE").vector(4, 1, 2).commit()
+    h = np.zeros(256, dtype=np.uint8)
+    import torch
+    d = torch.zeros(256, dtype=torch.uint8, device="cuda")
+    with pytest.raises(dt.DTError) as e:
+        dt.pack(t, 1, h.ctypes.data, d)
+    assert e.value.name == "DT_ERR_ARG"
+
+
+def test_host_entry_points(torch_cuda):
+    """dt_pack_host / dt_unpack_host (the e2e path): host buffers in and out."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c2_lower_triangle(700)
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    src = fill_bytes(parent, 5)
+    out = np.zeros(t.size, dtype=np.uint8)
+    dt.pack_host(t, 1, src.ctypes.data + org, out.ctypes.data, stream=0)
+    assert np.array_equal(out, oracle.pack(ot, 1, src, org))
+    dst = np.full(parent, 0xA5, dtype=np.uint8)
+    dt.unpack_host(t, 1, out.ctypes.data, dst.ctypes.data + org, stream=0)
+    exp = np.full(parent, 0xA5, dtype=np.uint8)
+    oracle.unpack(ot, 1, out, exp, org)
+    assert np.array_equal(dst, exp)
+
+
+def test_full_size_sampled_c5_large(torch_cuda):
+    """BASELINE sizes where the oracle cannot produce the whole stream quickly:
+    compare sampled stream bytes against the oracle's per-position addresses."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c5_particles(1 << 30)
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    src_h = fill_bytes(parent, 0x5EED0005)
+    src = _dev(torch, src_h)
+    n = t.size
+    out = torch.empty(n, dtype=torch.uint8, device="cuda")
+    dt.pack(t, 1, src, out)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(5)
+    ps = np.unique(np.concatenate([rng.integers(0, n, size=200000), [0, n - 1]]))
+    addr = oracle.addr_of(ot, 1, ps)
+    got = out[torch.from_numpy(ps).cuda()].cpu().numpy()
+    assert np.array_equal(got, src_h[org + addr])
+    # unpack then re-pack equals the packed stream (untouched-gap check on a sample)
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8, device="cuda")
+    dt.unpack(t, 1, out, dst)
+    back = torch.empty_like(out)
+    dt.pack(t, 1, dst, back)
+    torch.cuda.synchronize()
+    assert torch.equal(back, out)
+    covered = np.zeros(parent, dtype=bool)
+    covered[org + addr] = True
+    gaps = np.flatnonzero(~covered)[:: 97]
+    idx = rec[2][:2000] + 4  # bytes 4..7 of a selected particle are padding: never written
+    assert np.all(dst[torch.from_numpy(idx).cuda()].cpu().numpy() == 0xA5)
+    del gaps
