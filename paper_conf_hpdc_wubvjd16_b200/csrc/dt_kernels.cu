@@ -643,7 +643,7 @@ static dt_status host_common(bool unpack, dt_t t, int64_t count, const void* a, 
     // gaps must stay untouched: bring the destination span in, scatter, send it back
     CU(cudaMemcpyAsync(dspan, horigin + lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, s));
     CU(cudaMemcpyAsync(dpack, a, (size_t)n, cudaMemcpyHostToDevice, s));
-    st = pack_common(true, t, count, dpack, dorigin, pos, &m, stream);
+    st = pack_common(true, t, count, dorigin, dpack, pos, &m, stream);
     if (st == DT_OK) CU(cudaMemcpyAsync(horigin + lo, dspan, (size_t)(hi - lo), cudaMemcpyDeviceToHost, s));
   }
   g_check_ptrs = saved;

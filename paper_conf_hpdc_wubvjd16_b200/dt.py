@@ -310,3 +310,97 @@ def unpack_host(t: Type, count: int, packed_addr: int, origin_addr: int, pos: in
     n = I64((count * t.size - pos) if nbytes is None else nbytes)
     _check(lib().dt_unpack_host(t.h, count, packed_addr, origin_addr, pos, C.byref(n), _stream(stream)))
     return n.value
+
+
+# ------------------------------------------------------------------ GPU <-> GPU transfer
+def exchange_blobs(blob: bytes, group=None) -> bytes:
+    """All-gather one equal-size byte blob per rank (rank-major concatenation)
+    through torch.distributed — plumbing for dt_comm_connect's IPC handles."""
+    import torch.distributed as tdist
+    ws = tdist.get_world_size(group)
+    out = [None] * ws
+    tdist.all_gather_object(out, blob, group=group)
+    assert all(len(b) == len(blob) for b in out), "handle blobs differ in size"
+    return b"".join(out)
+
+
+def broadcast_id(idbytes, group=None) -> bytes:
+    """Broadcast rank 0's 128-byte NCCL unique id."""
+    import torch.distributed as tdist
+    obj = [idbytes]
+    tdist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+class Comm:
+    """dt_comm_t: this rank's endpoint (receive rings + flags, or a NCCL communicator)."""
+
+    def __init__(self, rank: int, nranks: int, device: int, chunk_bytes: int = 1 << 20, depth: int = 4,
+                 mode: int = XFER_P2P, ctas: int = 0, nccl_id: bytes | None = None):
+        self.opts = XferOpts(chunk_bytes, depth, mode, ctas, 0)
+        self.h = P()
+        self.rank, self.nranks = rank, nranks
+        idbuf = C.create_string_buffer(nccl_id, 128) if nccl_id else None
+        _check(lib().dt_comm_init(rank, nranks, idbuf, device, C.byref(self.opts), C.byref(self.h)))
+
+    @staticmethod
+    def nccl_unique_id() -> bytes:
+        buf = C.create_string_buffer(128)
+        _check(lib().dt_nccl_unique_id(buf))
+        return buf.raw
+
+    @classmethod
+    def from_process_group(cls, group=None, device: int | None = None, **opts):
+        """Create the endpoint on every rank of `group` and connect the ring mappings
+        (IPC handles all-gathered once, [L20:c3123], [L20:c3807])."""
+        import torch
+        import torch.distributed as tdist
+        rank, ws = tdist.get_rank(group), tdist.get_world_size(group)
+        if device is None:
+            device = torch.cuda.current_device()
+        nid = None
+        if opts.get("mode", XFER_P2P) == XFER_NCCL:
+            nid = broadcast_id(cls.nccl_unique_id() if rank == 0 else None, group)
+        c = cls(rank, ws, device, nccl_id=nid, **opts)
+        c.connect(exchange_blobs(c.local_handle(), group))
+        return c
+
+    def local_handle(self) -> bytes:
+        n = C.c_size_t(0)
+        _check(lib().dt_comm_local_handle(self.h, None, C.byref(n)))
+        buf = C.create_string_buffer(n.value)
+        _check(lib().dt_comm_local_handle(self.h, buf, C.byref(n)))
+        return buf.raw[: n.value]
+
+    def connect(self, all_handles: bytes):
+        per = len(all_handles) // self.nranks
+        buf = C.create_string_buffer(all_handles, len(all_handles))
+        _check(lib().dt_comm_connect(self.h, buf, per))
+
+    def sendrecv(self, sbuf, scount, stype, dest, rbuf, rcount, rtype, source, stream=None, sbuf_offset=0,
+                 rbuf_offset=0):
+        sp = (_ptr(sbuf) + sbuf_offset) if sbuf is not None else None
+        rp = (_ptr(rbuf) + rbuf_offset) if rbuf is not None else None
+        _check(lib().dt_sendrecv(sp, scount, stype.h if stype else None, dest, rp, rcount,
+                                 rtype.h if rtype else None, source, self.h, None, _stream(stream)))
+
+    def group_start(self):
+        _check(lib().dt_group_start(self.h))
+
+    def group_end(self, stream=None):
+        _check(lib().dt_group_end(self.h, _stream(stream)))
+
+    def check(self):
+        _check(lib().dt_comm_check(self.h))
+
+    def free(self):
+        if self.h:
+            _check(lib().dt_comm_free(C.byref(self.h)))
+            self.h = P()
+
+    def __del__(self):
+        try:
+            if self.h and _lib is not None:
+                _lib.dt_comm_free(C.byref(self.h))
+        except Exception:
+            pass

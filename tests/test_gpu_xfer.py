@@ -1,0 +1,202 @@
+"""GPU transfer parity (T3/T4): dt_sendrecv must deliver exactly
+oracle_unpack(rtype, oracle_pack(stype, sbuf)) into the receive layout and leave
+every other byte untouched.  On one B200 the sender and
+receiver are the same GPU: loopback inside one process (the paper's "1GPU"
+case, [L26:c1686 §5.2.1]) and two processes on one GPU over CUDA IPC.  The
+pipeline runs in fragments of `chunk` bytes through `depth` ring slots
+([L18:c4394]-[L18:c5513 §4.1]); chunk sizes below the message size exercise
+slot reuse and the ack flow control."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import oracle
+from workloads import c1_submatrix, c2_lower_triangle, c3_block_cyclic, c5_particles, fill_bytes
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    os.environ.setdefault("DT_TIMEOUT_MS", "20000")
+    return torch
+
+
+def _loop_check(torch, comm, srec, sorg, sparent, rrec, rorg, rparent, scount=1, rcount=1, seed=3):
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    so, ro = oracle.from_recipe(srec), oracle.from_recipe(rrec)
+    st, rt = dt.from_recipe(srec).commit(), dt.from_recipe(rrec).commit()
+    sh = fill_bytes(sparent, seed)
+    rh = np.full(rparent, 0xA5, dtype=np.uint8)
+    exp = rh.copy()
+    oracle.sendrecv(so, scount, sh, ro, rcount, exp, sorg, rorg)
+    sd = torch.from_numpy(sh).cuda()
+    rd = torch.from_numpy(rh).cuda()
+    comm.sendrecv(sd, scount, st, comm.rank, rd, rcount, rt, comm.rank, sbuf_offset=sorg, rbuf_offset=rorg)
+    torch.cuda.synchronize()
+    comm.check()
+    assert np.array_equal(rd.cpu().numpy(), exp)
+
+
+@pytest.mark.parametrize("chunk,depth", [(64 << 10, 2), (256 << 10, 4), (1 << 20, 2), (4 << 20, 4)])
+def test_loopback_block_cyclic(torch_cuda, chunk, depth):
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth)
+    rec, org, parent = c3_block_cyclic(2048, 64)
+    _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
+    # repeated messages on the same channel reuse the ring (cumulative counters)
+    for s in range(3):
+        _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent, seed=10 + s)
+    comm.free()
+
+
+def test_loopback_different_types(torch_cuda):
+    """Same signature, different layouts (vector <-> contiguous, triangle -> packed;
+    [L26:c4303 §5.2.2]); a receive larger than the message fills a prefix (A12)."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0, chunk_bytes=128 << 10, depth=3)
+    v, vorg, vpar = c1_submatrix(256, 1024, 1, 1)
+    contig = ("contiguous", 256 * 256, ("basic", "DOUBLE"))
+    _loop_check(torch_cuda, comm, v, vorg, vpar, contig, 0, 256 * 256 * 8)
+    _loop_check(torch_cuda, comm, contig, 0, 256 * 256 * 8, v, vorg, vpar)
+    tri, _, tpar = c2_lower_triangle(600)
+    n = 600 * 601 // 2
+    _loop_check(torch_cuda, comm, tri, 0, tpar, ("contiguous", n + 100, ("basic", "DOUBLE")), 0, (n + 100) * 8)
+    # matrix transpose: column-major -> row-major as a vector of blocklength-1 columns ([L26:c4896 §5.2.3])
+    m = 96
+    rows = ("hvector", m, 1, 8, ("vector", m, 1, m, ("basic", "DOUBLE")))
+    cols = ("contiguous", m * m, ("basic", "DOUBLE"))
+    _loop_check(torch_cuda, comm, cols, 0, m * m * 8, rows, 0, m * m * 8)
+    comm.free()
+
+
+def test_loopback_short_blocks(torch_cuda):
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0, chunk_bytes=64 << 10, depth=2)
+    rec, org, parent = c5_particles(1 << 20)
+    _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
+    comm.free()
+
+
+def test_truncation_detected(torch_cuda):
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0, chunk_bytes=64 << 10, depth=2)
+    big = dt.Type.basic("DOUBLE").contiguous(1000).commit()
+    small = dt.Type.basic("DOUBLE").contiguous(999).commit()
+    s = torch.zeros(8000, dtype=torch.uint8, device="cuda")
+    r = torch.full((8000,), 0xA5, dtype=torch.uint8, device="cuda")
+    comm.sendrecv(s, 1, big, 0, r, 1, small, 0)
+    torch.cuda.synchronize()
+    with pytest.raises(dt.DTError) as e:
+        comm.check()
+    assert e.value.name == "DT_ERR_TRUNCATE"
+    assert torch.all(r == 0xA5)
+    # the channel stays usable afterwards
+    s2 = torch.arange(8000, dtype=torch.int64, device="cuda").to(torch.uint8)
+    comm.sendrecv(s2, 1, small, 0, r, 1, small, 0)
+    torch.cuda.synchronize()
+    comm.check()
+    assert torch.equal(r[:7992], s2[:7992])
+    comm.free()
+
+
+def test_loopback_halo_all_faces(torch_cuda):
+    """1-rank periodic halo: the 12 transfers of one exchange in one group."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import FACES, face_box, make_plan
+    n, h = 64, 1
+    L = n + 2 * h
+    comm = dt.Comm(0, 1, 0, chunk_bytes=16 << 10, depth=2)
+    plan = make_plan(0, n, h, dims=(1, 1, 1))
+    A = np.full((L, L, L), 0xA5A5A5A5, dtype=np.uint32)
+    z, y, x = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
+    A[h:h + n, h:h + n, h:h + n] = (z * 1000000 + y * 1000 + x).astype(np.uint32)
+    buf = torch.from_numpy(A.view(np.uint8).reshape(-1).copy()).cuda()
+    plan.exchange(comm, buf)
+    torch.cuda.synchronize()
+    comm.check()
+    B = buf.cpu().numpy().view(np.uint32).reshape(L, L, L)
+    for f in FACES:
+        sub, st = face_box(f, n, h, ghost=True)
+        zz, yy, xx = np.meshgrid(*[np.arange(s, s + k) for s, k in zip(st, sub)], indexing="ij")
+        exp = (((zz - h) % n) * 1000000 + ((yy - h) % n) * 1000 + ((xx - h) % n)).astype(np.uint32)
+        assert np.array_equal(B[zz, yy, xx], exp), f
+    comm.free()
+
+
+def test_nccl_mode_loopback(torch_cuda):
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    try:
+        nid = dt.Comm.nccl_unique_id()
+    except dt.DTError as e:
+        pytest.skip(f"NCCL unavailable: {e}")
+    comm = dt.Comm(0, 1, 0, chunk_bytes=256 << 10, depth=2, mode=dt.XFER_NCCL, nccl_id=nid)
+    rec, org, parent = c3_block_cyclic(1024, 64)
+    _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
+    comm.free()
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _ipc_worker(rank, port, q):
+    try:
+        import torch
+        import torch.distributed as tdist
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        os.environ.setdefault("DT_TIMEOUT_MS", "60000")
+        tdist.init_process_group("gloo", rank=rank, world_size=2)
+        torch.cuda.set_device(0)
+        from paper_conf_hpdc_wubvjd16_b200 import dt
+        comm = dt.Comm.from_process_group(device=0, chunk_bytes=256 << 10, depth=2, ctas=4)
+        rec, org, parent = c2_lower_triangle(1024)
+        t = dt.from_recipe(rec).commit()
+        mine = fill_bytes(parent, 100 + rank)
+        other = fill_bytes(parent, 100 + (1 - rank))
+        sd = torch.from_numpy(mine).cuda()
+        rd = torch.full((parent,), 0xA5, dtype=torch.uint8, device="cuda")
+        comm.sendrecv(sd, 1, t, 1 - rank, rd, 1, t, 1 - rank)
+        torch.cuda.synchronize()
+        comm.check()
+        exp = np.full(parent, 0xA5, dtype=np.uint8)
+        ot = oracle.from_recipe(rec)
+        oracle.sendrecv(ot, 1, other, ot, 1, exp)
+        ok = bool(np.array_equal(rd.cpu().numpy(), exp))
+        tdist.barrier()
+        comm.free()
+        q.put((rank, ok))
+        tdist.destroy_process_group()
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, traceback.format_exc() + repr(e)))
+
+
+def test_two_processes_one_gpu_ipc(torch_cuda):
+    """Two ranks (processes) exchange triangles through IPC-mapped rings on one GPU."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_ipc_worker, args=(r, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = [q.get(timeout=300) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+    for rank, ok in res:
+        assert ok is True, (rank, ok)
