@@ -119,9 +119,11 @@ template <int POL>
 __device__ __forceinline__ void warp_copy(uint8_t* dst, const uint8_t* src, int64_t n, int lane) {
   if (n <= 0) return;
   const unsigned rel = (unsigned)(((uintptr_t)src - (uintptr_t)dst) & 15);
-  if (rel == 0) warp_copy_v<POL, uint4, 4>(dst, src, n, lane);
-  else if ((rel & 7) == 0) warp_copy_v<POL, uint2, 8>(dst, src, n, lane);
-  else if ((rel & 3) == 0) warp_copy_v<POL, unsigned int, 8>(dst, src, n, lane);
+  // 4 KiB in flight per warp and iteration for the 16/8-byte paths (memory-level
+  // parallelism: ~40 warps/SM x 4 KiB covers the loaded HBM latency)
+  if (rel == 0) warp_copy_v<POL, uint4, 8>(dst, src, n, lane);
+  else if ((rel & 7) == 0) warp_copy_v<POL, uint2, 16>(dst, src, n, lane);
+  else if ((rel & 3) == 0) warp_copy_v<POL, unsigned int, 16>(dst, src, n, lane);
   else if ((rel & 1) == 0) warp_copy_v<POL, unsigned short, 8>(dst, src, n, lane);
   else warp_copy_v<POL, unsigned char, 8>(dst, src, n, lane);
 }

@@ -99,7 +99,7 @@ __global__ void __launch_bounds__(kScanNT) k_scan_add(int64_t* out, const int64_
 
 // --------------------------------------------------------------- standalone kernels
 template <bool UNPACK, bool SINGLE>
-__global__ void __launch_bounds__(256) k_seg(const KP P) {
+__global__ void __launch_bounds__(256, 3) k_seg(const KP P) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t p = P.pos + gw * P.per_warp;
@@ -304,6 +304,17 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   return 1;
 }
 
+static int seg_occupancy(bool unpack, bool single) {
+  static int occ[2][2] = {{0, 0}, {0, 0}};
+  int& o = occ[unpack][single];
+  if (!o) {
+    const void* f = unpack ? (single ? (const void*)k_seg<true, true> : (const void*)k_seg<true, false>)
+                           : (single ? (const void*)k_seg<false, true> : (const void*)k_seg<false, false>);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, f, 256, 0) != cudaSuccess || o < 1) o = 4;
+  }
+  return o;
+}
+
 template <bool UNPACK>
 static void launch_word(const KP& P, int64_t g, bool vec16, unsigned grid, size_t smem, cudaStream_t s) {
 #define LW(G, VW) k_word<UNPACK, G, VW><<<grid, 256, smem, s>>>(P)
@@ -358,14 +369,16 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
   if (kind == 0) return DT_OK;
   const int sms = num_sms();
   if (kind == 1) {
-    const int64_t max_warps = (int64_t)sms * 8 * 8;  // 8 CTAs x 8 warps per SM
+    // exactly one wave of resident CTAs (no tail wave), at least ~4 KiB per warp
+    const bool single = P.nblocks == 1;
+    const int occ = seg_occupancy(unpack, single);
+    const int64_t max_warps = (int64_t)sms * occ * 8;
     int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
     int64_t per = (len + nw - 1) / nw;
     per = (per + 511) & ~int64_t(511);
     nw = (len + per - 1) / per;
     P.per_warp = per;
     unsigned grid = (unsigned)((nw + 7) / 8);
-    const bool single = P.nblocks == 1;
     if (unpack) {
       if (single) k_seg<true, true><<<grid, 256, 0, s>>>(P);
       else k_seg<true, false><<<grid, 256, 0, s>>>(P);

@@ -1,0 +1,81 @@
+#!/usr/bin/env python
+"""Kernel-level sweep over the paper's workloads (tuning aid, not the driver bench).
+
+For each config: pack and unpack GB/s (payload read + written, 2*size per
+kernel) with the L2 flushed before every launch, next to a contiguous device
+copy of the same bytes measured in the same run (the paper's "C" / cudaMemcpy
+practical-peak comparator, [L22:c3205 §5.1]).  Prints one JSON line per config.
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--configs", default="C1,C1b,C2,C3,C4x,C4y,C4z,C5_64M,C5_1G,C5b_64M,V4K,V8K,V16K,T16K")
+    ap.add_argument("--reps", type=int, default=20)
+    args = ap.parse_args()
+    import numpy as np
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    import workloads as W
+    mk = {
+        "C1": lambda: W.c1_submatrix(), "C1b": lambda: W.c1_submatrix(r0=1, c0=1),
+        "C2": lambda: W.c2_lower_triangle(), "C3": lambda: W.c3_block_cyclic(),
+        "C4x": lambda: W.c4_face("x-"), "C4y": lambda: W.c4_face("y-"), "C4z": lambda: W.c4_face("z-"),
+        "C5_64M": lambda: W.c5_particles(64 << 20), "C5_1G": lambda: W.c5_particles(1 << 30),
+        "C5b_64M": lambda: W.c5b_irregular(64 << 20),
+        "V4K": lambda: W.c1_submatrix(4096, 8192), "V8K": lambda: W.c1_submatrix(8192, 16384),
+        "V16K": lambda: W.c1_submatrix(16384, 16384),
+        "T16K": lambda: W.c2_lower_triangle(16384), "Tstair8K": lambda: W.stair_triangle(8192, 256),
+    }
+    dev = torch.device("cuda")
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    flush = torch.empty(2 * l2, dtype=torch.uint8, device=dev)
+    s = torch.cuda.current_stream()
+    for name in args.configs.split(","):
+        rec, org, parent = mk[name]()
+        t = dt.from_recipe(rec).commit()
+        n = t.size
+        src = torch.empty(parent, dtype=torch.uint8, device=dev)
+        src.random_(0, 256)
+        pk = torch.empty(n, dtype=torch.uint8, device=dev)
+        dst = torch.empty(parent, dtype=torch.uint8, device=dev)
+        a = torch.empty(n, dtype=torch.uint8, device=dev)
+        b = torch.empty(n, dtype=torch.uint8, device=dev)
+
+        def timeit(fn):
+            ts = []
+            for i in range(args.reps + 3):
+                flush.fill_(i & 0xFF)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                fn()
+                e1.record(s)
+                torch.cuda.synchronize()
+                if i >= 3:
+                    ts.append(e0.elapsed_time(e1))
+            return statistics.median(ts)
+
+        tp = timeit(lambda: dt.pack(t, 1, src, pk, origin_offset=org, stream=s))
+        tu = timeit(lambda: dt.unpack(t, 1, pk, dst, origin_offset=org, stream=s))
+        tc = timeit(lambda: b.copy_(a))
+        kind, g = t.plan(1, src.data_ptr() + org, pk.data_ptr(), 0, n)
+        gb = lambda ms: round(2 * n / (ms * 1e-3) / 1e9, 1)
+        print(json.dumps({"config": name, "bytes": n, "kernel": kind, "gran": g, "pack_us": round(tp * 1e3, 2),
+                          "unpack_us": round(tu * 1e3, 2), "copy_us": round(tc * 1e3, 2), "pack_gbs": gb(tp),
+                          "unpack_gbs": gb(tu), "copy_gbs": gb(tc),
+                          "pack_vs_copy": round(tc / tp, 3), "unpack_vs_copy": round(tc / tu, 3)}), flush=True)
+        del src, pk, dst, a, b
+        torch.cuda.empty_cache()
+
+
+if __name__ == "__main__":
+    main()
