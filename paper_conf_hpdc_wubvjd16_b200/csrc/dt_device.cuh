@@ -115,17 +115,100 @@ __device__ __forceinline__ void warp_copy_v(uint8_t* __restrict__ dst, const uin
   if (lane < tail) dst[nv * W + lane] = src[nv * W + lane];
 }
 
+// 16 output bytes = bytes [R, R+16) of the 32-byte window a|b (R = 1..15).
+template <int R>
+__device__ __forceinline__ uint4 realign(const uint4& a, const uint4& b) {
+  const unsigned w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+  constexpr int ws = R / 4, bs = R % 4;
+  uint4 o;
+  if (bs == 0) {
+    o.x = w[ws]; o.y = w[ws + 1]; o.z = w[ws + 2]; o.w = w[ws + 3];
+  } else {
+    o.x = __funnelshift_r(w[ws], w[ws + 1], 8 * bs);
+    o.y = __funnelshift_r(w[ws + 1], w[ws + 2], 8 * bs);
+    o.z = __funnelshift_r(w[ws + 2], w[ws + 3], 8 * bs);
+    o.w = __funnelshift_r(w[ws + 3], w[ws + 4], 8 * bs);
+  }
+  return o;
+}
+
+// Relatively misaligned copy with full 16-byte accesses on both sides: the
+// destination is peeled to 16 B, the source is read as aligned 16-byte vectors
+// A_i, and output vector i = bytes [R, R+16) of A_i|A_{i+1}; A_{i+1} comes from
+// the neighbouring lane by warp shuffle (lane 31 takes lane 0's next vector), so
+// every source byte is loaded once.  R = (src - dst) mod 16 is a template
+// parameter: the word-aligned cases need 1-3 shuffles per vector, none of the
+// byte juggling of the paper's 8-byte prologue/epilogue scheme.
+template <int POL, int R, int U>
+__device__ __forceinline__ void warp_copy_realign(uint8_t* __restrict__ dst, const uint8_t* __restrict__ src,
+                                                  int64_t n, int lane) {
+  int64_t head = (int64_t)((0 - (uintptr_t)dst) & 15);
+  if (head > n) head = n;
+  if (lane < head) dst[lane] = src[lane];
+  dst += head;
+  src += head;
+  n -= head;
+  const int64_t nv = n / 16;
+  uint4* d = reinterpret_cast<uint4*>(dst);
+  const uint4* A = reinterpret_cast<const uint4*>(src - R);  // (src - R) is 16-byte aligned
+  constexpr int NWORD = (R + 15) / 4 - 3;  // words of the next vector that are needed (1..4)
+  const int nb = (lane + 1) & 31;
+  int64_t base = 0;
+  for (; base + 32 * U <= nv; base += 32 * U) {
+    uint4 a[U + 1];
+#pragma unroll
+    for (int u = 0; u < U; u++) a[u] = ldv<POL>(A + base + lane + 32 * u);
+    a[U] = lane == 0 ? ldv<POL>(A + base + 32 * U) : make_uint4(0, 0, 0, 0);
+    uint4 rot[U + 1];
+#pragma unroll
+    for (int u = 0; u <= U; u++) {
+      rot[u].x = __shfl_sync(0xffffffffu, a[u].x, nb);
+      if (NWORD > 1) rot[u].y = __shfl_sync(0xffffffffu, a[u].y, nb);
+      if (NWORD > 2) rot[u].z = __shfl_sync(0xffffffffu, a[u].z, nb);
+      if (NWORD > 3) rot[u].w = __shfl_sync(0xffffffffu, a[u].w, nb);
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const uint4 nx = lane == 31 ? rot[u + 1] : rot[u];
+      stv(d + base + lane + 32 * u, realign<R>(a[u], nx));
+    }
+  }
+  for (int64_t i = base + lane; i < nv; i += 32) stv(d + i, realign<R>(ldv<POL>(A + i), ldv<POL>(A + i + 1)));
+  const int64_t tail = n - nv * 16;
+  if (lane < tail) dst[nv * 16 + lane] = src[nv * 16 + lane];
+}
+
 template <int POL>
 __device__ __forceinline__ void warp_copy(uint8_t* dst, const uint8_t* src, int64_t n, int lane) {
   if (n <= 0) return;
   const unsigned rel = (unsigned)(((uintptr_t)src - (uintptr_t)dst) & 15);
-  // 4 KiB in flight per warp and iteration for the 16/8-byte paths (memory-level
-  // parallelism: ~40 warps/SM x 4 KiB covers the loaded HBM latency)
-  if (rel == 0) warp_copy_v<POL, uint4, 8>(dst, src, n, lane);
-  else if ((rel & 7) == 0) warp_copy_v<POL, uint2, 16>(dst, src, n, lane);
-  else if ((rel & 3) == 0) warp_copy_v<POL, unsigned int, 16>(dst, src, n, lane);
-  else if ((rel & 1) == 0) warp_copy_v<POL, unsigned short, 8>(dst, src, n, lane);
-  else warp_copy_v<POL, unsigned char, 8>(dst, src, n, lane);
+  // 4 KiB in flight per warp and iteration (memory-level parallelism: ~24-40
+  // warps/SM x 4 KiB covers the loaded HBM latency).  Short segments take the
+  // plain path (the realigning loop needs >= 32 vectors to pay off).
+  if (rel == 0) { warp_copy_v<POL, uint4, 8>(dst, src, n, lane); return; }
+  if (n < 1024) {
+    if ((rel & 7) == 0) warp_copy_v<POL, uint2, 8>(dst, src, n, lane);
+    else if ((rel & 3) == 0) warp_copy_v<POL, unsigned int, 8>(dst, src, n, lane);
+    else warp_copy_v<POL, unsigned char, 8>(dst, src, n, lane);
+    return;
+  }
+  switch (rel) {
+    case 8: warp_copy_realign<POL, 8, 4>(dst, src, n, lane); break;
+    case 4: warp_copy_realign<POL, 4, 4>(dst, src, n, lane); break;
+    case 12: warp_copy_realign<POL, 12, 4>(dst, src, n, lane); break;
+    case 1: warp_copy_realign<POL, 1, 4>(dst, src, n, lane); break;
+    case 2: warp_copy_realign<POL, 2, 4>(dst, src, n, lane); break;
+    case 3: warp_copy_realign<POL, 3, 4>(dst, src, n, lane); break;
+    case 5: warp_copy_realign<POL, 5, 4>(dst, src, n, lane); break;
+    case 6: warp_copy_realign<POL, 6, 4>(dst, src, n, lane); break;
+    case 7: warp_copy_realign<POL, 7, 4>(dst, src, n, lane); break;
+    case 9: warp_copy_realign<POL, 9, 4>(dst, src, n, lane); break;
+    case 10: warp_copy_realign<POL, 10, 4>(dst, src, n, lane); break;
+    case 11: warp_copy_realign<POL, 11, 4>(dst, src, n, lane); break;
+    case 13: warp_copy_realign<POL, 13, 4>(dst, src, n, lane); break;
+    case 14: warp_copy_realign<POL, 14, 4>(dst, src, n, lane); break;
+    default: warp_copy_realign<POL, 15, 4>(dst, src, n, lane); break;
+  }
 }
 
 // largest b with boff[b] <= q (boff strictly increasing, boff[0] == 0): 32-ary
