@@ -24,7 +24,7 @@ def _sources():
 
 
 def _deps():
-    out = _sources() + [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith(".h")]
+    out = _sources() + [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".h", ".cuh"))]
     out.append(os.path.join(ROOT, "include", "dt.h"))
     out.append(os.path.abspath(__file__))
     return out

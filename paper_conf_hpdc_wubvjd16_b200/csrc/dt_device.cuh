@@ -110,7 +110,14 @@ __device__ __forceinline__ void warp_copy_v(uint8_t* __restrict__ dst, const uin
 #pragma unroll
     for (int u = 0; u < U; u++) stv(d + i + 32 * u, v[u]);
   }
-  for (; i < nv; i += 32) stv(d + i, ldv<POL>(s + i));
+  if (i < nv) {  // remainder: one predicated batch, all loads in flight together
+    V v[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) v[u] = ldv<POL>(s + min(i + 32 * u, nv - 1));
+#pragma unroll
+    for (int u = 0; u < U; u++)
+      if (i + 32 * u < nv) stv(d + i + 32 * u, v[u]);
+  }
   const int64_t tail = n - nv * W;
   if (lane < tail) dst[nv * W + lane] = src[nv * W + lane];
 }
@@ -173,7 +180,18 @@ __device__ __forceinline__ void warp_copy_realign(uint8_t* __restrict__ dst, con
       stv(d + base + lane + 32 * u, realign<R>(a[u], nx));
     }
   }
-  for (int64_t i = base + lane; i < nv; i += 32) stv(d + i, realign<R>(ldv<POL>(A + i), ldv<POL>(A + i + 1)));
+  for (int64_t i = base + lane; i < nv; i += 32 * U) {  // remainder (< 32*U vectors): one predicated batch
+    uint4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {  // clamped (always valid) addresses keep the arrays in registers
+      const int64_t j = min(i + 32 * u, nv - 1);
+      a[u] = ldv<POL>(A + j);
+      b[u] = ldv<POL>(A + j + 1);
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++)
+      if (i + 32 * u < nv) stv(d + i + 32 * u, realign<R>(a[u], b[u]));
+  }
   const int64_t tail = n - nv * 16;
   if (lane < tail) dst[nv * 16 + lane] = src[nv * 16 + lane];
 }
@@ -271,46 +289,64 @@ template <> struct WordT<16> { typedef uint4 T; };
 // Threads tid, tid+nthr, ... each handle one VW-byte vector of the packed
 // stream [P.pos, P.pos+P.len) (which must be G-aligned and G-granular); wt is
 // the template's word table in shared memory.
-template <bool UNPACK, int G, int VW, int POL>
+// NV vectors per thread and iteration: every load of the batch is issued before
+// the first store, so a thread keeps NV*VW bytes in flight.
+template <bool UNPACK, int G, int VW, int POL, int NV = 2>
 __device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64_t tid, int64_t nthr) {
   typedef typename WordT<G>::T W;
   typedef typename WordT<VW>::T VT;
   constexpr int NW = VW / G;
   const int64_t nvec = (P.len + VW - 1) / VW;
   const int64_t end = P.pos + P.len;
-  for (int64_t v = tid; v < nvec; v += nthr) {
-    const int64_t s0 = P.pos + v * VW;
-    uint64_t e = fdiv((uint64_t)s0, P.ftsize);
-    int w = (int)((s0 - (int64_t)e * P.tsize) / G);
-    int64_t ed = elem_disp(P, e);
-    const int64_t rem = (end - s0) / G;
-    const int nvalid = rem < NW ? (int)rem : NW;
-    union {
-      VT vec;
-      W word[NW];
-    } u;
-    if (UNPACK) {
-      if (nvalid == NW) u.vec = ldv<POL>(reinterpret_cast<const VT*>(P.c + v * VW));
-      else
-        for (int k = 0; k < nvalid; k++) u.word[k] = reinterpret_cast<const W*>(P.c + v * VW)[k];
+  union U {
+    VT vec;
+    W word[NW];
+  };
+  for (int64_t v0 = tid; v0 < nvec; v0 += nthr * NV) {
+    U u[NV];
+    int nvalid[NV];
+    int64_t ed[NV];
+    uint64_t e[NV];
+    int w[NV];
+#pragma unroll
+    for (int j = 0; j < NV; j++) {
+      const int64_t v = v0 + (int64_t)j * nthr;
+      const int64_t s0 = P.pos + v * VW;
+      const int64_t rem = v < nvec ? (end - s0) / G : 0;
+      nvalid[j] = rem < NW ? (int)rem : NW;
+      e[j] = fdiv((uint64_t)s0, P.ftsize);
+      w[j] = (int)((s0 - (int64_t)e[j] * P.tsize) / G);
+      ed[j] = nvalid[j] > 0 ? elem_disp(P, e[j]) : 0;
+      if (UNPACK) {
+        if (nvalid[j] == NW) u[j].vec = ldv<POL>(reinterpret_cast<const VT*>(P.c + v * VW));
+        else
+          for (int k = 0; k < nvalid[j]; k++) u[j].word[k] = reinterpret_cast<const W*>(P.c + v * VW)[k];
+      }
     }
 #pragma unroll
-    for (int k = 0; k < NW; k++) {
-      if (k < nvalid) {
-        W* a = reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed + wt[w]);
-        if (UNPACK) *a = u.word[k];
-        else u.word[k] = ldv<POL>(a);
-        if (++w == P.nwords && k + 1 < nvalid) {
-          w = 0;
-          ++e;
-          ed = elem_disp(P, e);
+    for (int j = 0; j < NV; j++) {
+#pragma unroll
+      for (int k = 0; k < NW; k++) {
+        if (k < nvalid[j]) {
+          W* a = reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed[j] + wt[w[j]]);
+          if (UNPACK) *a = u[j].word[k];
+          else u[j].word[k] = ldv<POL>(a);
+          if (++w[j] == P.nwords && k + 1 < nvalid[j]) {
+            w[j] = 0;
+            ++e[j];
+            ed[j] = elem_disp(P, e[j]);
+          }
         }
       }
     }
     if (!UNPACK) {
-      if (nvalid == NW) stv(reinterpret_cast<VT*>(P.c + v * VW), u.vec);
-      else
-        for (int k = 0; k < nvalid; k++) reinterpret_cast<W*>(P.c + v * VW)[k] = u.word[k];
+#pragma unroll
+      for (int j = 0; j < NV; j++) {
+        const int64_t v = v0 + (int64_t)j * nthr;
+        if (nvalid[j] == NW) stv(reinterpret_cast<VT*>(P.c + v * VW), u[j].vec);
+        else
+          for (int k = 0; k < nvalid[j]; k++) reinterpret_cast<W*>(P.c + v * VW)[k] = u[j].word[k];
+      }
     }
   }
 }

@@ -37,7 +37,14 @@ struct Level {
 struct Form {
   std::vector<Level> lv;           // outermost first
   std::vector<int64_t> bd, bl;     // template blocks (bytes), typemap order
-  int64_t tsize() const { int64_t s = 0; for (auto x : bl) s += x; return s; }
+  // per-call planning must stay O(levels): O(n) facts are computed once and cached
+  mutable int64_t gran_cache = -1, tsize_cache = -1;
+  mutable int fits32_cache = -1;
+  int64_t tsize() const {
+    if (tsize_cache < 0) { int64_t s = 0; for (auto x : bl) s += x; tsize_cache = s; }
+    return tsize_cache;
+  }
+  void invalidate() const { gran_cache = tsize_cache = -1; fits32_cache = -1; }
   int64_t nelem() const { int64_t n = 1; for (auto& l : lv) n *= l.cnt; return n; }
   bool empty() const { return bl.empty(); }
 };

@@ -254,8 +254,11 @@ void build_levels(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t cou
 }
 
 static bool template_fits_int32(const Form& f) {
+  if (f.fits32_cache >= 0) return f.fits32_cache == 1;
+  f.fits32_cache = 0;
   for (size_t b = 0; b < f.bd.size(); b++)
     if (f.bd[b] < INT32_MIN || f.bd[b] + f.bl[b] > INT32_MAX) return false;
+  f.fits32_cache = 1;
   return true;
 }
 
@@ -300,7 +303,11 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   g = std::min(g, lowp2((uint64_t)len));
   *gran = g;
   const double mean = (double)ts / (double)nb;
-  if (mean < 256.0 && ts / g <= kMaxWordTable && ts % g == 0 && template_fits_int32(f)) return 2;
+  const bool word_ok = ts / g <= kMaxWordTable && ts % g == 0 && template_fits_int32(f);
+  static const int force = getenv("DT_FORCE_KERNEL") ? atoi(getenv("DT_FORCE_KERNEL")) : 0;  // tuning aid
+  if (force == 2 && word_ok) return 2;
+  if (force == 1) return 1;
+  if (mean < 256.0 && word_ok) return 2;
   return 1;
 }
 

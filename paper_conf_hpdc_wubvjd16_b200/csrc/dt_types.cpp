@@ -326,6 +326,7 @@ namespace dt {
 
 static void shift_form(Form& f, int64_t s) {
   for (auto& d : f.bd) d += s;
+  f.invalidate();
 }
 static void prepend_regular(Form& f, int64_t cnt, int64_t stride) {
   Level l;
@@ -354,6 +355,7 @@ static void merge_template(Form& f) {
 }
 
 void normalize(Form& f) {
+  f.invalidate();
   merge_template(f);
   if (f.bl.empty()) { f.lv.clear(); return; }
   for (auto& l : f.lv)
@@ -437,12 +439,14 @@ static int64_t low_pow2(int64_t x) {
 }
 
 int64_t form_granularity(const Form& f) {
+  if (f.gran_cache >= 0) return f.gran_cache;
   int64_t g = 16;
   for (size_t i = 0; i < f.bd.size(); i++) g = std::min(g, std::min(low_pow2(f.bd[i]), low_pow2(f.bl[i])));
   for (auto& l : f.lv) {
     if (l.is_list()) for (auto x : *l.table) g = std::min(g, low_pow2(x));
     else g = std::min(g, low_pow2(l.stride));
   }
+  f.gran_cache = g;
   return g;
 }
 
