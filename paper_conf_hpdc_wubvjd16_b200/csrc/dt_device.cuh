@@ -48,6 +48,7 @@ struct KP {
   const int64_t* table[kMaxLevels];
   FastDiv fcnt[kMaxLevels];
   FastDiv ftsize;
+  FastDiv fnb;  // division by nblocks (short-block window kernel)
   int64_t per_warp;
   const int32_t* wtab;
 };
@@ -348,6 +349,86 @@ __device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64
           for (int k = 0; k < nvalid[j]; k++) reinterpret_cast<W*>(P.c + v * VW)[k] = u[j].word[k];
       }
     }
+  }
+}
+
+// Short blocks under a large template (irregular hindexed, C5b): a warp walks its
+// stream slice in 512-byte windows.  For each window, lanes take one block each
+// (32 per round, block starts from boff) and write the source address of every
+// G-byte word their block contributes to the window into a per-warp shared
+// table; then each lane moves its 16 output bytes: G-byte gathers from the
+// table's addresses and one coalesced 16-byte store (unpack: the reverse).
+constexpr int kBlkWin = 512;
+template <bool UNPACK, int G, int POL>
+__device__ __forceinline__ void blk_range(const KP& P, int64_t p0, const int64_t p1, int lane, int64_t* sa) {
+  typedef typename WordT<G>::T W;
+  const FastDiv& fnb = P.fnb;
+  constexpr int NWL = 16 / G;  // words per lane
+  if (p0 >= p1) return;
+  uint64_t ce = fdiv((uint64_t)p0, P.ftsize);
+  int64_t cb = warp_find_block(P.boff, P.nblocks, p0 - (int64_t)ce * P.tsize, lane);
+  const uint64_t nel = P.nblocks ? (uint64_t)((P.pos + P.len + P.tsize - 1) / P.tsize) : 0;
+  for (int64_t q = p0; q < p1; q += kBlkWin) {
+    const int64_t qe = min(q + kBlkWin, p1);
+    while (true) {
+      int64_t lb = cb + lane;
+      uint64_t le = ce;
+      if (lb >= P.nblocks) {
+        const uint64_t k = fdiv((uint64_t)lb, fnb);
+        le += k;
+        lb -= (int64_t)k * P.nblocks;
+      }
+      int64_t start = INT64_MAX, len = 0;
+      if (le < nel) {
+        start = (int64_t)le * P.tsize + __ldg(P.boff + lb);
+        len = __ldg(P.bl + lb);
+      }
+      const int64_t a = max(start, q), z = min(start + len, qe);
+      if (a < z) {
+        const int64_t base = (int64_t)(uintptr_t)P.nc + elem_disp(P, le) + __ldg(P.bd + lb) - start;
+        for (int64_t x = a; x < z; x += G) sa[(x - q) / G] = base + x;
+      }
+      const bool reach = start != INT64_MAX && start + len >= qe;
+      if (__any_sync(0xffffffffu, reach || start == INT64_MAX)) {
+        const unsigned before = __ballot_sync(0xffffffffu, start != INT64_MAX && start + len <= qe);
+        cb += __popc(before);
+        break;
+      }
+      cb += 32;
+    }
+    if (cb >= P.nblocks) {
+      const uint64_t k = fdiv((uint64_t)cb, fnb);
+      ce += k;
+      cb -= (int64_t)k * P.nblocks;
+    }
+    __syncwarp();
+    const int64_t x0 = q + (int64_t)lane * 16;
+    const int64_t remw = x0 >= qe ? 0 : (qe - x0) / G;
+    const int nvalid = remw < NWL ? (int)remw : NWL;
+    uint8_t* cp = P.c + (x0 - P.pos);
+    union {
+      uint4 vec;
+      W word[NWL];
+    } u;
+    if (UNPACK) {
+      if (nvalid == NWL) u.vec = ldv<POL>(reinterpret_cast<const uint4*>(cp));
+      else
+        for (int k = 0; k < nvalid; k++) u.word[k] = reinterpret_cast<const W*>(cp)[k];
+    }
+#pragma unroll
+    for (int k = 0; k < NWL; k++) {
+      if (k < nvalid) {
+        W* a = reinterpret_cast<W*>(sa[lane * NWL + k]);
+        if (UNPACK) *a = u.word[k];
+        else u.word[k] = ldv<POL>(a);
+      }
+    }
+    if (!UNPACK) {
+      if (nvalid == NWL) stv(reinterpret_cast<uint4*>(cp), u.vec);
+      else
+        for (int k = 0; k < nvalid; k++) reinterpret_cast<W*>(cp)[k] = u.word[k];
+    }
+    __syncwarp();
   }
 }
 

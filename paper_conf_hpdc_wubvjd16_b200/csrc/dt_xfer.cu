@@ -633,9 +633,6 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.n = n;
       X.chunk = c->o.chunk_bytes;
       X.depth = c->o.depth;
-      X.cta0 = cta;
-      X.ncta = G;
-      cta += G;
       uint64_t* pf = c->peer_flags[p.dest];
       X.ring = c->peer_ring[p.dest] + c->ring_off(c->rank, ch);
       X.ready = pf + c->ready_idx(c->rank, ch, 0);
@@ -662,9 +659,6 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.n = cap;
       X.chunk = c->o.chunk_bytes;
       X.depth = c->o.depth;
-      X.cta0 = cta;
-      X.ncta = G;
-      cta += G;
       uint64_t* pf = c->peer_flags[p.source];
       X.ring = c->ring + c->ring_off(p.source, ch);
       X.ready = c->flags + c->ready_idx(p.source, ch, 0);
@@ -682,6 +676,18 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   }
   if (nops == 0) return DT_OK;
   A.nops = nops;
+  // every CTA must be co-resident: fit the per-op CTA count to the occupancy
+  int occ = 0;
+  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_xfer, 256, smem));
+  int sms = 0, dev = 0;
+  CU(cudaGetDevice(&dev));
+  CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  const int per_op = std::max(1, std::min(G, occ * sms / nops));
+  for (int i = 0; i < nops; i++) {
+    A.ops[i].cta0 = cta;
+    A.ops[i].ncta = per_op;
+    cta += per_op;
+  }
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
