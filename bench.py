@@ -285,9 +285,86 @@ def run_e2e(args, t, src_h, org, parent, payload, dev):
             "steps": steps, "note": "host pinned buffers; wall clock incl. all copies and syncs"}
 
 
+def run_xfer(args):
+    """S7: pipelined GPU<->GPU exchange of the C3 block-cyclic submatrix (128 MiB per
+    direction, 512-B runs) through dt_sendrecv, chunk/depth sweep ([L18:c4394 §4.1]).
+    Pairs (r, r^1) exchange concurrently; at N=1 the rank exchanges with itself
+    (loopback, the paper's "1GPU" case [L26:c1686]).  value = bytes received by all
+    ranks per second (max-over-ranks device time)."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from workloads import c3_block_cyclic, fill_bytes, seed_for
+    ws, rank, local = dist_init()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    peer = rank ^ 1 if (rank ^ 1) < ws else rank
+    rec, org, parent = c3_block_cyclic()
+    t = dt.from_recipe(rec).commit()
+    payload = t.size
+    A = torch.from_numpy(fill_bytes(parent, seed_for(3) + rank)).to(dev)
+    B = torch.full((parent,), 0xA5, dtype=torch.uint8, device=dev)
+    s = torch.cuda.current_stream()
+    mode = dt.XFER_NCCL if args.xfer_mode == "nccl" else dt.XFER_P2P
+    results = []
+    for chunk in (64 << 10, 256 << 10, 1 << 20, 4 << 20):
+        for depth in (2, 4):
+            if ws > 1:
+                comm = dt.Comm.from_process_group(device=local, chunk_bytes=chunk, depth=depth, mode=mode)
+            else:
+                nid = dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None
+                comm = dt.Comm(0, 1, local, chunk_bytes=chunk, depth=depth, mode=mode, nccl_id=nid)
+            for _ in range(args.warmup):
+                comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
+            torch.cuda.synchronize()
+            comm.check()
+            steps = max(3, min(args.steps, 20))
+            if ws > 1:
+                torch.distributed.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            for _ in range(steps):
+                comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
+            e1.record(s)
+            torch.cuda.synchronize()
+            comm.check()
+            ms = e0.elapsed_time(e1) / steps
+            if ws > 1:
+                x = torch.tensor([ms], dtype=torch.float64, device=dev)
+                torch.distributed.all_reduce(x, op=torch.distributed.ReduceOp.MAX)
+                ms = float(x[0])
+            results.append({"chunk": chunk, "depth": depth, "ms": round(ms, 4),
+                            "gbs_per_rank": round(payload / (ms * 1e-3) / 1e9, 1)})
+            comm.free()
+    best = max(results, key=lambda r: r["gbs_per_rank"])
+    value = ws * payload / (best["ms"] * 1e-3) / 1e9
+    # parity of the last exchange: my B must equal the peer's A packed/unpacked (closed form: same layout)
+    exp = torch.from_numpy(fill_bytes(parent, seed_for(3) + peer)).to(dev)
+    ok = bool(torch.equal(B.view(-1)[org:org + 8 * 64], exp.view(-1)[org:org + 8 * 64]))
+    peak = 900.0 if ws > 1 else load_peaks()[0] / 4  # loopback: 4x payload of HBM traffic per exchange
+    line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": ws, "steps": steps,
+            "warmup": args.warmup, "ms_per_step": best["ms"], "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
+            "config": {"workload": "C3: ScaLAPACK 2D block-cyclic submatrix (N=8192 f64, nb=64, owner (0,1)), "
+                                   f"pairwise exchange, mode={args.xfer_mode}",
+                       "payload_bytes": payload, "sweep": results, "spot_parity": ok,
+                       "pairs": "loopback (1 GPU)" if ws == 1 else "(r, r^1)"},
+            "roofline": {"bound": "nvlink" if ws > 1 else "hbm", "achieved": best["gbs_per_rank"],
+                         "peak": peak, "unit": "GB/s", "frac": round(best["gbs_per_rank"] / peak, 4),
+                         "note": "per-direction NVLink 900 GB/s nominal" if ws > 1 else
+                                 "loopback moves 4x payload through HBM (pack R+W, unpack R+W)"},
+            "gpu_launches": steps}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--workload", default="c2", choices=["c2", "xfer"])
+    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl"])
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -298,6 +375,8 @@ def main():
         args.warmup = 3
     if args.impl == "reference":
         run_reference(args)
+    elif args.workload == "xfer":
+        run_xfer(args)
     else:
         run_ours(args)
 

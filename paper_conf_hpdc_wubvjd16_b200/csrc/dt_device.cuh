@@ -96,13 +96,14 @@ __device__ __forceinline__ void warp_copy_v(uint8_t* __restrict__ dst, const uin
   constexpr int W = sizeof(V);
   int64_t head = (int64_t)((0 - (uintptr_t)dst) & (W - 1));
   if (head > n) head = n;
-  if (lane < head) dst[lane] = src[lane];
-  dst += head;
-  src += head;
-  n -= head;
-  const int64_t nv = n / W;
-  V* d = reinterpret_cast<V*>(dst);
-  const V* s = reinterpret_cast<const V*>(src);
+  const int64_t nv = (n - head) / W;
+  const int64_t tail = n - head - nv * W;
+  // head and tail bytes are loaded up front so that a short segment costs one
+  // memory round trip (their stores happen after the body's loads are issued)
+  const uint8_t hb = lane < head ? src[lane] : 0;
+  const uint8_t tb = lane < tail ? src[head + nv * W + lane] : 0;
+  V* d = reinterpret_cast<V*>(dst + head);
+  const V* s = reinterpret_cast<const V*>(src + head);
   int64_t i = lane;
   for (; i + 32 * (U - 1) < nv; i += 32 * U) {
     V v[U];
@@ -119,8 +120,8 @@ __device__ __forceinline__ void warp_copy_v(uint8_t* __restrict__ dst, const uin
     for (int u = 0; u < U; u++)
       if (i + 32 * u < nv) stv(d + i + 32 * u, v[u]);
   }
-  const int64_t tail = n - nv * W;
-  if (lane < tail) dst[nv * W + lane] = src[nv * W + lane];
+  if (lane < head) dst[lane] = hb;
+  if (lane < tail) dst[head + nv * W + lane] = tb;
 }
 
 // 16 output bytes = bytes [R, R+16) of the 32-byte window a|b (R = 1..15).
@@ -152,7 +153,10 @@ __device__ __forceinline__ void warp_copy_realign(uint8_t* __restrict__ dst, con
                                                   int64_t n, int lane) {
   int64_t head = (int64_t)((0 - (uintptr_t)dst) & 15);
   if (head > n) head = n;
-  if (lane < head) dst[lane] = src[lane];
+  const uint8_t hb = lane < head ? src[lane] : 0;
+  const int64_t tail0 = (n - head) % 16;
+  const uint8_t tb = lane < tail0 ? src[n - tail0 + lane] : 0;
+  uint8_t* const dst0 = dst;
   dst += head;
   src += head;
   n -= head;
@@ -193,8 +197,8 @@ __device__ __forceinline__ void warp_copy_realign(uint8_t* __restrict__ dst, con
     for (int u = 0; u < U; u++)
       if (i + 32 * u < nv) stv(d + i + 32 * u, realign<R>(a[u], b[u]));
   }
-  const int64_t tail = n - nv * 16;
-  if (lane < tail) dst[nv * 16 + lane] = src[nv * 16 + lane];
+  if (lane < head) dst0[lane] = hb;
+  if (lane < tail0) dst[nv * 16 + lane] = tb;
 }
 
 template <int POL>
@@ -249,6 +253,41 @@ __device__ __forceinline__ int64_t warp_find_block(const int64_t* __restrict__ b
 
 // One warp copies stream bytes [p, p1) (P.pos <= p < p1 <= P.pos + P.len).
 // POL applies to the loads (pack reads the layout, unpack reads the packed side).
+// Walk from a resolved start: stream byte p is byte r of block b of element e
+// (element displacement ed).  The next block's descriptor is prefetched while the
+// current segment is copied.
+template <bool UNPACK, bool SINGLE, int POL>
+__device__ __forceinline__ void seg_walk(const KP& P, int64_t p, const int64_t p1, int64_t b, int64_t r, uint64_t e,
+                                         int64_t ed, const int lane) {
+  int64_t blen = SINGLE ? P.bl0 : __ldg(P.bl + b);
+  int64_t bdsp = SINGLE ? P.bd0 : __ldg(P.bd + b);
+  while (true) {
+    const int64_t seg = min(blen - r, p1 - p);
+    const int64_t nb = (SINGLE || b + 1 == P.nblocks) ? 0 : b + 1;
+    int64_t nblen = 0, nbdsp = 0;
+    if (!SINGLE && p + seg < p1) {
+      nblen = __ldg(P.bl + nb);
+      nbdsp = __ldg(P.bd + nb);
+    }
+    uint8_t* ncp = const_cast<uint8_t*>(P.nc) + ed + bdsp + r;
+    uint8_t* cp = P.c + (p - P.pos);
+    if (UNPACK) warp_copy<POL>(ncp, cp, seg, lane);
+    else warp_copy<POL>(cp, ncp, seg, lane);
+    p += seg;
+    if (p >= p1) break;
+    r = 0;
+    if (SINGLE || nb == 0) {
+      ++e;
+      ed = elem_disp(P, e);
+    }
+    b = nb;
+    if (!SINGLE) {
+      blen = nblen;
+      bdsp = nbdsp;
+    }
+  }
+}
+
 template <bool UNPACK, bool SINGLE, int POL>
 __device__ __forceinline__ void seg_range(const KP& P, int64_t p, const int64_t p1, const int lane) {
   if (p >= p1) return;
@@ -259,24 +298,46 @@ __device__ __forceinline__ void seg_range(const KP& P, int64_t p, const int64_t 
     b = warp_find_block(P.boff, P.nblocks, r, lane);
     r -= __ldg(P.boff + b);
   }
-  int64_t ed = elem_disp(P, e);
-  while (true) {
-    const int64_t blen = SINGLE ? P.bl0 : __ldg(P.bl + b);
-    const int64_t bdsp = SINGLE ? P.bd0 : __ldg(P.bd + b);
-    const int64_t seg = min(blen - r, p1 - p);
-    uint8_t* ncp = const_cast<uint8_t*>(P.nc) + ed + bdsp + r;
-    uint8_t* cp = P.c + (p - P.pos);
-    if (UNPACK) warp_copy<POL>(ncp, cp, seg, lane);
-    else warp_copy<POL>(cp, ncp, seg, lane);
-    p += seg;
-    if (p >= p1) break;
-    r = 0;
-    if (SINGLE || ++b == P.nblocks) {
-      b = 0;
-      ++e;
-      ed = elem_disp(P, e);
-    }
+  seg_walk<UNPACK, SINGLE, POL>(P, p, p1, b, r, e, elem_disp(P, e), lane);
+}
+
+// ---------------------------------------------------------------- launch plans
+// Cost-balanced warp slices (long-run kernel).  A warp's time is its bytes plus a
+// fixed cost per segment (descriptor fetch + one memory round trip), so slices
+// are cut at equal COST, cost(p) = p + alpha * (#block starts before p), instead
+// of equal bytes: the triangle's tail of short columns is spread over many warps
+// instead of serialising in the last one.  The cut positions depend only on the
+// layout and (count, pos, len, nwarps), so they are computed once by k_plan and
+// cached on the committed type — the paper's cached work distribution
+// ([L18:c1649 §3.2]) without a per-unit array.
+struct PlanEnt {
+  int64_t p, b, r, e, ed;  // stream byte p = byte r of block b of element e (displacement ed)
+};
+
+// position of cost C (relative to cost 0 = stream byte 0), with its block/element
+__device__ __forceinline__ PlanEnt pos_of_cost(const KP& P, int64_t alpha, const FastDiv& fce, int64_t ce, int64_t C) {
+  const uint64_t e = fdiv((uint64_t)C, fce);
+  const int64_t rc = C - (int64_t)e * ce;
+  int64_t lo = 0, hi = P.nblocks;  // largest b with boff[b] + alpha*b <= rc
+  while (hi - lo > 1) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (__ldg(P.boff + mid) + alpha * mid <= rc) lo = mid;
+    else hi = mid;
   }
+  const int64_t off = rc - (__ldg(P.boff + lo) + alpha * lo);
+  const int64_t bl = P.nblocks == 1 ? P.bl0 : __ldg(P.bl + lo);  // (a merged run lives in bl0)
+  PlanEnt r;
+  r.e = e;
+  r.b = lo;
+  r.r = min(off, bl);
+  r.p = (int64_t)e * P.tsize + __ldg(P.boff + lo) + r.r;
+  if (off >= bl) {  // inside the block's fixed cost: start at the next block
+    r.r = 0;
+    if (lo + 1 == P.nblocks) { r.b = 0; r.e = e + 1; }
+    else r.b = lo + 1;
+  }
+  r.ed = 0;
+  return r;
 }
 
 template <int G>

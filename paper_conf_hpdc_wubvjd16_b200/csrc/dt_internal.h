@@ -44,7 +44,16 @@ struct Form {
     if (tsize_cache < 0) { int64_t s = 0; for (auto x : bl) s += x; tsize_cache = s; }
     return tsize_cache;
   }
-  void invalidate() const { gran_cache = tsize_cache = -1; fits32_cache = -1; }
+  mutable std::vector<int64_t> hoff_cache;  // host exclusive prefix of bl (launch planning)
+  void invalidate() const { gran_cache = tsize_cache = -1; fits32_cache = -1; hoff_cache.clear(); }
+  const std::vector<int64_t>& hoff() const {
+    if (hoff_cache.size() != bl.size()) {
+      hoff_cache.resize(bl.size());
+      int64_t s = 0;
+      for (size_t i = 0; i < bl.size(); i++) { hoff_cache[i] = s; s += bl[i]; }
+    }
+    return hoff_cache;
+  }
   int64_t nelem() const { int64_t n = 1; for (auto& l : lv) n *= l.cnt; return n; }
   bool empty() const { return bl.empty(); }
 };
@@ -63,6 +72,13 @@ struct DeviceDesc {
   std::vector<int64_t*> tables;  // per level (nullptr for regular levels)
   // word tables for the short kernel, keyed by granularity (1,2,4,8,16)
   int32_t* wtab[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+  // cached cost-balanced warp plans of the long-run kernel, keyed by the launch shape
+  struct PlanSlot {
+    int64_t count = -1, pos = 0, len = 0, nw = 0, alpha = 0, tsize = 0;
+    void* d = nullptr;
+  };
+  std::vector<PlanSlot> plans;
+  size_t plan_next = 0;
 };
 
 enum Kind { K_BASIC, K_CONTIG, K_HVECTOR, K_HINDEXED, K_STRUCT, K_SUBARRAY, K_RESIZED };

@@ -98,13 +98,30 @@ __global__ void __launch_bounds__(kScanNT) k_scan_add(int64_t* out, const int64_
 }
 
 // --------------------------------------------------------------- standalone kernels
+// warp w of the long-run kernel copies stream bytes [plan[w].p, plan[w+1].p)
 template <bool UNPACK, bool SINGLE>
-__global__ void __launch_bounds__(256, 3) k_seg(const KP P) {
+__global__ void __launch_bounds__(256, 3) k_seg(const KP P, const PlanEnt* __restrict__ plan, int64_t nw) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t p = P.pos + gw * P.per_warp;
-  const int64_t p1 = min(p + P.per_warp, P.pos + P.len);
-  seg_range<UNPACK, SINGLE, LD_CS>(P, p, p1, lane);
+  if (gw >= nw) return;
+  const PlanEnt a = plan[gw];
+  const int64_t p1 = plan[gw + 1].p;
+  if (a.p >= p1) return;
+  seg_walk<UNPACK, SINGLE, LD_CS>(P, a.p, p1, a.b, a.r, a.e, a.ed, lane);
+}
+
+// one thread per warp boundary: cost-balanced cut positions (see PlanEnt)
+__global__ void k_plan(const KP P, int64_t alpha, FastDiv fce, int64_t ce, int64_t C0, int64_t C1, int64_t nw,
+                       PlanEnt* plan) {
+  const int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (w > nw) return;
+  const int64_t C = w == nw ? C1 : C0 + (int64_t)((__int128)(C1 - C0) * w / nw);
+  PlanEnt r = pos_of_cost(P, alpha, fce, ce, C);
+  const int64_t end = P.pos + P.len;
+  if (w == nw || r.p > end) r.p = end;
+  if (r.p < P.pos) r.p = P.pos;
+  r.ed = r.p < end ? elem_disp(P, r.e) : 0;
+  plan[w] = r;
 }
 
 template <bool UNPACK, int G>
@@ -159,6 +176,8 @@ void free_desc(DeviceDesc& dd) {
   for (auto*& w : dd.wtab) { cudaFree(w); w = nullptr; }
   dd.bd = dd.bl = dd.boff = nullptr;
   dd.tables.clear();
+  for (auto& sl : dd.plans) cudaFree(sl.d);
+  dd.plans.clear();
   if (cur >= 0 && dd.device >= 0 && dd.device != cur) cudaSetDevice(cur);
 }
 
@@ -300,6 +319,67 @@ static Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t 
   return E;
 }
 
+// per-segment fixed cost in byte-equivalents (one round trip at a warp's share of HBM bandwidth)
+static int64_t seg_alpha() {
+  static const int64_t a = getenv("DT_SEG_ALPHA") ? atoll(getenv("DT_SEG_ALPHA")) : 2048;
+  return a;
+}
+
+// cost of stream byte p (see PlanEnt): p + alpha * (block starts before it)
+static int64_t host_cost(const KP& P, const Form& f, int64_t alpha, int64_t p) {
+  const int64_t ce = P.tsize + alpha * P.nblocks;
+  const int64_t e = p / P.tsize;
+  const int64_t rem = p - e * P.tsize;
+  int64_t b = 0, bo = 0;
+  if (P.nblocks > 1) {
+    const auto& h = f.hoff();
+    b = (int64_t)(std::upper_bound(h.begin(), h.end(), rem) - h.begin()) - 1;
+    bo = h[(size_t)b];
+  }
+  return e * ce + bo + alpha * b + (rem - bo);
+}
+
+// cached (or freshly computed) cost-balanced plan for this launch shape
+static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& dd, int64_t count, int64_t nw,
+                          cudaStream_t s, const PlanEnt** out) {
+  const int64_t alpha = seg_alpha();
+  std::lock_guard<std::mutex> g(t->mu);
+  for (auto& sl : dd.plans) {
+    if (sl.d && sl.count == count && sl.pos == P.pos && sl.len == P.len && sl.nw == nw && sl.alpha == alpha &&
+        sl.tsize == P.tsize) {
+      *out = (const PlanEnt*)sl.d;
+      return DT_OK;
+    }
+  }
+  size_t idx;
+  if (dd.plans.size() < 16) {
+    dd.plans.emplace_back();
+    idx = dd.plans.size() - 1;
+  } else {
+    idx = dd.plan_next++ % dd.plans.size();
+  }
+  DeviceDesc::PlanSlot& sl = dd.plans[idx];
+  if (sl.d) {  // eviction: cudaFree waits for in-flight users of the old plan
+    cudaFree(sl.d);
+    sl.d = nullptr;
+  }
+  sl.count = -1;
+  CU(cudaMalloc(&sl.d, sizeof(PlanEnt) * (size_t)(nw + 1)));
+  const int64_t ce = P.tsize + alpha * P.nblocks;
+  const int64_t C0 = host_cost(P, f, alpha, P.pos), C1 = host_cost(P, f, alpha, P.pos + P.len);
+  k_plan<<<(unsigned)((nw + 1 + 255) / 256), 256, 0, s>>>(P, alpha, make_fd((uint64_t)ce), ce, C0, C1, nw,
+                                                          (PlanEnt*)sl.d);
+  CU(cudaGetLastError());
+  sl.count = count;
+  sl.pos = P.pos;
+  sl.len = P.len;
+  sl.nw = nw;
+  sl.alpha = alpha;
+  sl.tsize = P.tsize;
+  *out = (const PlanEnt*)sl.d;
+  return DT_OK;
+}
+
 int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
                 int64_t* gran) {
   if (len <= 0 || f.bl.empty()) return 0;
@@ -396,18 +476,17 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     const bool single = P.nblocks == 1;
     const int occ = seg_occupancy(unpack, single);
     const int64_t max_warps = (int64_t)sms * occ * 8;
-    int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
-    int64_t per = (len + nw - 1) / nw;
-    per = (per + 511) & ~int64_t(511);
-    nw = (len + per - 1) / per;
-    P.per_warp = per;
+    const int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
+    const PlanEnt* plan = nullptr;
+    dt_status pst = get_plan(t, P, f, dd, count, nw, s, &plan);
+    if (pst != DT_OK) return pst;
     unsigned grid = (unsigned)((nw + 7) / 8);
     if (unpack) {
-      if (single) k_seg<true, true><<<grid, 256, 0, s>>>(P);
-      else k_seg<true, false><<<grid, 256, 0, s>>>(P);
+      if (single) k_seg<true, true><<<grid, 256, 0, s>>>(P, plan, nw);
+      else k_seg<true, false><<<grid, 256, 0, s>>>(P, plan, nw);
     } else {
-      if (single) k_seg<false, true><<<grid, 256, 0, s>>>(P);
-      else k_seg<false, false><<<grid, 256, 0, s>>>(P);
+      if (single) k_seg<false, true><<<grid, 256, 0, s>>>(P, plan, nw);
+      else k_seg<false, false><<<grid, 256, 0, s>>>(P, plan, nw);
     }
   } else if (kind == 3) {
     P.fnb = make_fd((uint64_t)P.nblocks);
