@@ -140,8 +140,8 @@ __global__ void __launch_bounds__(256) k_word(const KP P) {
   extern __shared__ int32_t wt[];
   for (int i = threadIdx.x; i < P.nwords; i += blockDim.x) wt[i] = P.wtab[i];
   __syncthreads();
-  word_range<UNPACK, G, VW, LD_CS>(P, wt, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
-                                   (int64_t)gridDim.x * blockDim.x);
+  word_range<UNPACK, G, VW, LD_CS, (G >= 4 ? 4 : 2)>(P, wt, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                                                     (int64_t)gridDim.x * blockDim.x);
 }
 // --------------------------------------------------------------- host side
 static int g_num_sms = 0;
@@ -516,9 +516,14 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     const bool vec16 = (((uintptr_t)c) & 15) == 0;
     const int64_t vw = vec16 ? 16 : g;
     const int64_t nvec = (len + vw - 1) / vw;
-    const int64_t maxg = (int64_t)sms * 8;
-    unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(maxg, (nvec + 255) / 256));
     size_t smem = sizeof(int32_t) * (size_t)P.nwords;
+    // one wave of resident CTAs (grid-stride loop inside)
+    static int occ_w = 0;
+    if (!occ_w && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_w, k_word<false, 4, 16>, 256, 4096) !=
+                       cudaSuccess || occ_w < 1))
+      occ_w = 4;
+    const int64_t maxg = (int64_t)sms * occ_w;
+    unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(maxg, (nvec + 255) / 256));
     if (unpack) launch_word<true>(P, g, vec16, grid, smem, s);
     else launch_word<false>(P, g, vec16, grid, smem, s);
   }

@@ -38,7 +38,8 @@
 namespace dt {
 
 constexpr int kMaxOps = 16;
-constexpr int kMaxCh = 6;  // concurrent messages per (pair, direction) inside one group
+constexpr int kMaxCh = 6;   // concurrent messages per (pair, direction) inside one group
+constexpr int kMaxSub = 64; // sub-rings (one per sending CTA) per message
 constexpr uint64_t kAbort = 1ull << 63;
 
 struct XOp {
@@ -96,7 +97,7 @@ __device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeo
   int ns = 32;
   while (true) {
     __nanosleep(ns);
-    if (ns < 1024) ns <<= 1;
+    if (ns < 256) ns <<= 1;
     v = ld_acquire_sys(p);
     if (pred(v)) { *out = v; return true; }
     if ((int64_t)(gtimer() - t0) > timeout_ns) {
@@ -140,7 +141,7 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int
 __global__ void __launch_bounds__(256) k_xfer(const __grid_constant__ XArgs A) {
   extern __shared__ int32_t wt[];
   __shared__ uint64_t s_val;
-  __shared__ int s_stop;
+  __shared__ int s_stop, s_gs;
   int op = 0;
   for (int i = 0; i < A.nops; i++)
     if ((int)blockIdx.x >= A.ops[i].cta0 && (int)blockIdx.x < A.ops[i].cta0 + A.ops[i].ncta) op = i;
@@ -153,11 +154,19 @@ __global__ void __launch_bounds__(256) k_xfer(const __grid_constant__ XArgs A) {
   if (threadIdx.x == 0) s_stop = 0;
   __syncthreads();
 
+  // Sub-rings: step k of the message covers stream bytes [kC, (k+1)C); sub-ring
+  // js in [0, gs) carries [kC + js*Cs, kC + (js+1)*Cs), Cs = C/gs, through its own
+  // D slots and flags, so every CTA pipelines on its own (no cross-CTA wait per
+  // fragment).  The sender runs one CTA per sub-ring; receiver CTA j serves
+  // sub-rings j, j+ncta, ...
   int64_t n = X.n;
+  int gs;
   if (X.role == 0) {
-    // ---- send role: header, wait for "go" (receiver-driven, [L20:c3973])
+    gs = X.ncta;
+    // ---- send role: header {seq, nbytes, gs}, wait for "go" (receiver-driven, [L20:c3973])
     if (j == 0 && threadIdx.x == 0) {
       st_release_sys(X.hdr + 1, (uint64_t)n);
+      st_release_sys(X.hdr + 2, (uint64_t)gs);
       st_release_sys(X.hdr, X.seq);
     }
     if (threadIdx.x == 0) {
@@ -168,10 +177,8 @@ __global__ void __launch_bounds__(256) k_xfer(const __grid_constant__ XArgs A) {
       if (s_stop == 1 && j == 0) atomicCAS(X.err, 0, XERR_TRUNCATE);
     }
     __syncthreads();
-    if (s_stop) {
-      if (s_stop == 1 && j == 0 && (int)threadIdx.x < D) X.base_out[threadIdx.x] = X.base_in[threadIdx.x];
-      return;
-    }
+    if (s_stop == 2) return;
+    if (s_stop == 1) n = 0;  // aborted: move nothing, carry the bases over
   } else {
     // ---- recv role: read the header, check capacity, send "go"
     if (threadIdx.x == 0) {
@@ -179,60 +186,69 @@ __global__ void __launch_bounds__(256) k_xfer(const __grid_constant__ XArgs A) {
       const uint64_t seq = X.seq;
       bool ok = spin(X.hdr, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v);
       s_val = ok ? ld_acquire_sys(X.hdr + 1) : 0;
-      s_stop = ok ? 0 : 1;
+      s_gs = ok ? (int)ld_acquire_sys(X.hdr + 2) : 1;
+      s_stop = ok ? 0 : 2;
     }
     __syncthreads();
-    if (s_stop) return;
+    if (s_stop == 2) return;
     n = (int64_t)s_val;
+    gs = s_gs;
     if (n > X.n) {
       if (j == 0 && threadIdx.x == 0) {
         atomicCAS(X.err, 0, XERR_TRUNCATE);
         st_release_sys(X.go, X.seq | kAbort);
       }
-      if (j == 0 && (int)threadIdx.x < D) X.base_out[threadIdx.x] = X.base_in[threadIdx.x];
-      return;
+      n = 0;
+    } else if (j == 0 && threadIdx.x == 0) {
+      st_release_sys(X.go, X.seq);
     }
-    if (j == 0 && threadIdx.x == 0) st_release_sys(X.go, X.seq);
   }
 
+  const int64_t Cs = C / gs;
   const int64_t K = (n + C - 1) / C;
   for (int64_t k = 0; k < K; k++) {
     const int slot = (int)(k % D);
     const int64_t round = k / D;
-    const int64_t clen = min(C, n - k * C);
-    int64_t sub = (clen + X.ncta - 1) / X.ncta;
-    sub = (sub + 511) & ~int64_t(511);
-    const int64_t lo = (int64_t)j * sub;
-    if (lo >= clen) continue;
-    const int64_t len = min(sub, clen - lo);
-    uint8_t* sl = X.ring + (int64_t)slot * C - k * C;  // so that stream byte k*C lands at slot start
-    const uint64_t base = X.base_in[slot] + (uint64_t)round * (uint64_t)C;
-    if (threadIdx.x == 0) {
-      uint64_t v;
-      bool ok;
-      if (X.role == 0) ok = spin(X.ack + slot, [base](uint64_t x) { return x >= base; }, A.timeout_ns, X.err, &v);
-      else {
-        const uint64_t need = base + (uint64_t)clen;
-        ok = spin(X.ready + slot, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v);
+    for (int js = j; js < gs; js += X.ncta) {
+      const int64_t off = k * C + (int64_t)js * Cs;
+      if (off >= n) continue;
+      const int64_t len = min(Cs, n - off);
+      const int fi = js * D + slot;  // flag / base index of (sub-ring, slot)
+      uint8_t* sl = X.ring + (int64_t)fi * Cs - off;  // stream byte `off` lands at the slot start
+      const uint64_t base = X.base_in[fi] + (uint64_t)round * (uint64_t)Cs;
+      if (threadIdx.x == 0) {
+        uint64_t v;
+        bool ok;
+        if (X.role == 0) ok = spin(X.ack + fi, [base](uint64_t x) { return x >= base; }, A.timeout_ns, X.err, &v);
+        else {
+          const uint64_t need = base + (uint64_t)len;
+          ok = spin(X.ready + fi, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v);
+        }
+        s_stop = ok ? 0 : 2;
       }
-      s_stop = ok ? 0 : 1;
-    }
-    __syncthreads();
-    if (s_stop) return;
-    if (X.role == 0) cta_chunk<false>(X, X.P, sl, k * C + lo, len, wt);
-    else cta_chunk<true>(X, X.P, sl, k * C + lo, len, wt);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence_system();
-      red_release_sys_add(X.role == 0 ? X.ready + slot : X.ack + slot, (uint64_t)len);
+      __syncthreads();
+      if (s_stop) return;
+      if (X.role == 0) cta_chunk<false>(X, X.P, sl, off, len, wt);
+      else cta_chunk<true>(X, X.P, sl, off, len, wt);
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence_system();
+        red_release_sys_add(X.role == 0 ? X.ready + fi : X.ack + fi, (uint64_t)len);
+      }
     }
   }
-  // cumulative per-slot bytes after this message (read by the next message's kernel)
-  if (j == 0 && (int)threadIdx.x < D) {
-    const int s = threadIdx.x;
-    uint64_t add = 0;
-    for (int64_t k = s; k < K; k += D) add += (uint64_t)min(C, n - k * C);
-    X.base_out[s] = X.base_in[s] + add;
+  // cumulative per-(sub-ring, slot) bytes after this message (read by the next
+  // message's kernel from the other parity); every sub-ring is carried over
+  for (int js = j; js < kMaxSub; js += X.ncta) {
+    for (int s = threadIdx.x; s < D; s += blockDim.x) {
+      uint64_t add = 0;
+      if (js < gs)
+        for (int64_t k = s; k < K; k += D) {
+          const int64_t off = k * C + (int64_t)js * Cs;
+          if (off < n) add += (uint64_t)min(Cs, n - off);
+        }
+      X.base_out[js * D + s] = X.base_in[js * D + s] + add;
+    }
   }
 }
 
@@ -331,17 +347,20 @@ struct dt_comm_s {
   uint8_t* rstage = nullptr; // recv staging
   int64_t* szbuf = nullptr;  // device size handshake buffers [2][kMaxOps]
   int64_t* szhost = nullptr; // pinned
-  // layout helpers
-  size_t ready_idx(int src, int ch, int slot) const { return ((size_t)src * nch + ch) * o.depth + slot; }
-  size_t hdr_idx(int src, int ch) const { return (size_t)nranks * nch * o.depth + ((size_t)src * nch + ch) * 2; }
-  size_t ack_idx(int dst, int ch, int slot) const {
-    return (size_t)nranks * nch * (o.depth + 2) + ((size_t)dst * nch + ch) * o.depth + slot;
-  }
-  size_t go_idx(int dst, int ch) const { return (size_t)nranks * nch * (2 * o.depth + 2) + (size_t)dst * nch + ch; }
-  size_t err_idx() const { return (size_t)nranks * nch * (2 * o.depth + 3); }
+  // layout helpers (uint64 flag words): per (peer, channel) kMaxSub*depth ready
+  // counters, a 4-word header {seq, nbytes, sub-rings, -}, kMaxSub*depth ack
+  // counters and a go word; then one error word.  The ring of a (source,
+  // channel) pair is depth*chunk bytes, split among the sender's sub-rings.
+  size_t per() const { return (size_t)kMaxSub * o.depth; }
+  size_t pairs() const { return (size_t)nranks * nch; }
+  size_t ready_idx(int src, int ch) const { return ((size_t)src * nch + ch) * per(); }
+  size_t hdr_idx(int src, int ch) const { return pairs() * per() + ((size_t)src * nch + ch) * 4; }
+  size_t ack_idx(int dst, int ch) const { return pairs() * (per() + 4) + ((size_t)dst * nch + ch) * per(); }
+  size_t go_idx(int dst, int ch) const { return pairs() * (2 * per() + 4) + (size_t)dst * nch + ch; }
+  size_t err_idx() const { return pairs() * (2 * per() + 5); }
   size_t ring_off(int src, int ch) const { return (((size_t)src * nch + ch) * o.depth) * (size_t)o.chunk_bytes; }
   uint64_t* base(int parity, int dir, int peer, int ch) const {
-    return bases + ((((size_t)parity * 2 + dir) * nranks + peer) * nch + ch) * o.depth;
+    return bases + ((((size_t)parity * 2 + dir) * nranks + peer) * nch + ch) * per();
   }
 };
 
@@ -423,7 +442,7 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
     e = cudaMalloc(&c->ring, c->ring_bytes);
     if (e == cudaSuccess) e = cudaMalloc(&c->flags, c->flag_words * 8);
     if (e == cudaSuccess) e = cudaMemset(c->flags, 0, c->flag_words * 8);
-    const size_t nb = (size_t)2 * 2 * nranks * c->nch * c->o.depth;
+    const size_t nb = (size_t)2 * 2 * c->pairs() * c->per();
     if (e == cudaSuccess) e = cudaMalloc(&c->bases, nb * 8);
     if (e == cudaSuccess) e = cudaMemset(c->bases, 0, nb * 8);
     if (e != cudaSuccess) {
@@ -609,7 +628,7 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   return DT_OK;
 }
 
-static int default_ctas(const dt_comm_s* c) { return c->o.ctas > 0 ? c->o.ctas : 16; }
+static int default_ctas(const dt_comm_s* c) { return c->o.ctas > 0 ? c->o.ctas : 32; }
 
 static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cudaStream_t s) {
   XArgs A;
@@ -635,9 +654,9 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.depth = c->o.depth;
       uint64_t* pf = c->peer_flags[p.dest];
       X.ring = c->peer_ring[p.dest] + c->ring_off(c->rank, ch);
-      X.ready = pf + c->ready_idx(c->rank, ch, 0);
+      X.ready = pf + c->ready_idx(c->rank, ch);
       X.hdr = pf + c->hdr_idx(c->rank, ch);
-      X.ack = c->flags + c->ack_idx(p.dest, ch, 0);
+      X.ack = c->flags + c->ack_idx(p.dest, ch);
       X.go = c->flags + c->go_idx(p.dest, ch);
       uint64_t& sq = c->send_seq[(size_t)p.dest * c->nch + ch];
       const int par = (int)(sq & 1);
@@ -661,9 +680,9 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.depth = c->o.depth;
       uint64_t* pf = c->peer_flags[p.source];
       X.ring = c->ring + c->ring_off(p.source, ch);
-      X.ready = c->flags + c->ready_idx(p.source, ch, 0);
+      X.ready = c->flags + c->ready_idx(p.source, ch);
       X.hdr = c->flags + c->hdr_idx(p.source, ch);
-      X.ack = pf + c->ack_idx(c->rank, ch, 0);
+      X.ack = pf + c->ack_idx(c->rank, ch);
       X.go = pf + c->go_idx(c->rank, ch);
       uint64_t& sq = c->recv_seq[(size_t)p.source * c->nch + ch];
       const int par = (int)(sq & 1);
@@ -684,9 +703,16 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
   const int per_op = std::max(1, std::min(G, occ * sms / nops));
   for (int i = 0; i < nops; i++) {
+    int n_i = per_op;
+    if (A.ops[i].role == 0) {  // one CTA per sub-ring; a sub-ring slot is C/gs bytes, a multiple of 512
+      const int64_t C = A.ops[i].chunk;
+      int g = 1;
+      while (g * 2 <= per_op && g * 2 <= kMaxSub && C % ((int64_t)g * 2 * 512) == 0) g *= 2;
+      n_i = g;
+    }
     A.ops[i].cta0 = cta;
-    A.ops[i].ncta = per_op;
-    cta += per_op;
+    A.ops[i].ncta = n_i;
+    cta += n_i;
   }
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
