@@ -119,12 +119,13 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int
     const int64_t body = len - len % X.g;
     KP Q = P;
     Q.len = body;
+    // few CTAs carry the whole transfer: keep 4 vectors per thread in flight (512 threads: 32 KiB/CTA)
     switch (X.g) {
-      case 1: word_range<UNPACK, 1, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
-      case 2: word_range<UNPACK, 2, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
-      case 4: word_range<UNPACK, 4, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
-      case 8: word_range<UNPACK, 8, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
-      default: word_range<UNPACK, 16, 16, POL>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 1: word_range<UNPACK, 1, 16, POL, 2>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 2: word_range<UNPACK, 2, 16, POL, 2>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 4: word_range<UNPACK, 4, 16, POL, 4>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 8: word_range<UNPACK, 8, 16, POL, 4>(Q, wt, threadIdx.x, blockDim.x); break;
+      default: word_range<UNPACK, 16, 16, POL, 4>(Q, wt, threadIdx.x, blockDim.x); break;
     }
     if (body < len && threadIdx.x < 32)  // ragged tail (< G bytes): one warp walks it
       seg_range<UNPACK, false, POL>(P, lo + body, lo + len, threadIdx.x & 31);
@@ -138,7 +139,8 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int
   else seg_range<UNPACK, false, POL>(P, a, b, lane);
 }
 
-__global__ void __launch_bounds__(256) k_xfer(const __grid_constant__ XArgs A) {
+constexpr int kXferThreads = 512;
+__global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
   extern __shared__ int32_t wt[];
   __shared__ uint64_t s_val;
   __shared__ int s_stop, s_gs;
@@ -697,7 +699,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   A.nops = nops;
   // every CTA must be co-resident: fit the per-op CTA count to the occupancy
   int occ = 0;
-  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_xfer, 256, smem));
+  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_xfer, kXferThreads, smem));
   int sms = 0, dev = 0;
   CU(cudaGetDevice(&dev));
   CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
@@ -717,7 +719,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
-  CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(256), args, smem, s));
+  CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
   return DT_OK;
 }
 
