@@ -307,13 +307,15 @@ def run_xfer(args):
     s = torch.cuda.current_stream()
     mode = dt.XFER_NCCL if args.xfer_mode == "nccl" else dt.XFER_P2P
     results = []
-    for chunk in (64 << 10, 256 << 10, 1 << 20, 4 << 20):
-        for depth in (2, 4):
+    for chunk in [int(x) << 10 for x in args.xfer_chunks_kib.split(",")]:
+        for depth in [int(x) for x in args.xfer_depths.split(",")]:
             if ws > 1:
-                comm = dt.Comm.from_process_group(device=local, chunk_bytes=chunk, depth=depth, mode=mode)
+                comm = dt.Comm.from_process_group(device=local, chunk_bytes=chunk, depth=depth, mode=mode,
+                                                  ctas=args.xfer_ctas)
             else:
                 nid = dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None
-                comm = dt.Comm(0, 1, local, chunk_bytes=chunk, depth=depth, mode=mode, nccl_id=nid)
+                comm = dt.Comm(0, 1, local, chunk_bytes=chunk, depth=depth, mode=mode, nccl_id=nid,
+                               ctas=args.xfer_ctas)
             for _ in range(args.warmup):
                 comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
             torch.cuda.synchronize()
@@ -365,6 +367,9 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--workload", default="c2", choices=["c2", "xfer"])
     ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl"])
+    ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
+    ap.add_argument("--xfer-depths", default="2,4")
+    ap.add_argument("--xfer-ctas", type=int, default=0, help="CTAs per direction (0 = library default)")
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])

@@ -64,7 +64,7 @@ struct XOp {
 
 struct XArgs {
   int32_t nops;
-  int32_t pad;
+  int32_t flags;  // tuning switches (DT_XFER_FLAGS): bit0 = no sys fence before the flag, bit1 = no sleep in polls
   int64_t timeout_ns;
   XOp ops[kMaxOps];
 };
@@ -90,13 +90,14 @@ enum { XERR_TIMEOUT = 1, XERR_TRUNCATE = 2 };
 
 // spin until pred(*p) holds; false on timeout (sets *err)
 template <typename Pred>
-__device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeout_ns, int32_t* err, uint64_t* out) {
+__device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeout_ns, int32_t* err, uint64_t* out,
+                                     bool sleep = true) {
   uint64_t v = ld_acquire_sys(p);
   if (pred(v)) { *out = v; return true; }
   const uint64_t t0 = gtimer();
   int ns = 32;
   while (true) {
-    __nanosleep(ns);
+    if (sleep) __nanosleep(ns);
     if (ns < 256) ns <<= 1;
     v = ld_acquire_sys(p);
     if (pred(v)) { *out = v; return true; }
@@ -221,10 +222,12 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       if (threadIdx.x == 0) {
         uint64_t v;
         bool ok;
-        if (X.role == 0) ok = spin(X.ack + fi, [base](uint64_t x) { return x >= base; }, A.timeout_ns, X.err, &v);
+        const bool sl_ok = !(A.flags & 2);
+        if (X.role == 0)
+          ok = spin(X.ack + fi, [base](uint64_t x) { return x >= base; }, A.timeout_ns, X.err, &v, sl_ok);
         else {
           const uint64_t need = base + (uint64_t)len;
-          ok = spin(X.ready + fi, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v);
+          ok = spin(X.ready + fi, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v, sl_ok);
         }
         s_stop = ok ? 0 : 2;
       }
@@ -234,7 +237,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       else cta_chunk<true>(X, X.P, sl, off, len, wt);
       __syncthreads();
       if (threadIdx.x == 0) {
-        __threadfence_system();
+        if (!(A.flags & 1)) __threadfence_system();
         red_release_sys_add(X.role == 0 ? X.ready + fi : X.ack + fi, (uint64_t)len);
       }
     }
@@ -637,6 +640,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   std::memset(&A, 0, sizeof(A));
   const char* to = getenv("DT_TIMEOUT_MS");
   A.timeout_ns = (int64_t)(to ? atoll(to) : 30000) * 1000000ll;
+  A.flags = getenv("DT_XFER_FLAGS") ? atoi(getenv("DT_XFER_FLAGS")) : 0;
   int nops = 0, cta = 0;
   size_t smem = 0;
   std::vector<int> sch(c->nranks, 0), rch(c->nranks, 0);

@@ -48,6 +48,11 @@ def main():
         flush_rd.sum()
     s = torch.cuda.current_stream()
     for name in args.configs.split(","):
+        if name.startswith("F8:"):  # Fig. 8 sweep: F8:<nblocks>:<block bytes>, gap = block
+            _, nb, bs = name.split(":")
+            nb, bs = int(nb), int(bs)
+            mk[name] = (lambda nb=nb, bs=bs: (("vector", nb, bs // 8, 2 * bs // 8, ("basic", "DOUBLE")), 0,
+                                              2 * bs * nb))
         rec, org, parent = mk[name]()
         t = dt.from_recipe(rec).commit()
         n = t.size
@@ -76,10 +81,23 @@ def main():
         tc = timeit(lambda: b.copy_(a))
         kind, g = t.plan(1, src.data_ptr() + org, pk.data_ptr(), 0, n)
         gb = lambda ms: round(2 * n / (ms * 1e-3) / 1e9, 1)
-        print(json.dumps({"config": name, "bytes": n, "kernel": kind, "gran": g, "pack_us": round(tp * 1e3, 2),
-                          "unpack_us": round(tu * 1e3, 2), "copy_us": round(tc * 1e3, 2), "pack_gbs": gb(tp),
-                          "unpack_gbs": gb(tu), "copy_gbs": gb(tc),
-                          "pack_vs_copy": round(tc / tp, 3), "unpack_vs_copy": round(tc / tu, 3)}), flush=True)
+        row = {"config": name, "bytes": n, "kernel": kind, "gran": g, "pack_us": round(tp * 1e3, 2),
+               "unpack_us": round(tu * 1e3, 2), "copy_us": round(tc * 1e3, 2), "pack_gbs": gb(tp),
+               "unpack_gbs": gb(tu), "copy_gbs": gb(tc),
+               "pack_vs_copy": round(tc / tp, 3), "unpack_vs_copy": round(tc / tu, 3)}
+        if rec[0] == "vector" and rec[4][0] == "basic":
+            # f4 diagnostic (Fig. 8, [L24:c4075 §5.1]): cudaMemcpy2D of the same vector, device to device
+            from cuda.bindings import runtime as cudart
+            es = {"DOUBLE": 8, "FLOAT": 4, "INT32": 4}.get(rec[4][1], 8)
+            width, height, spitch = rec[2] * es, rec[1], rec[3] * es
+
+            def m2d():
+                cudart.cudaMemcpy2DAsync(pk.data_ptr(), width, src.data_ptr() + org, spitch, width, height,
+                                         cudart.cudaMemcpyKind.cudaMemcpyDeviceToDevice, s.cuda_stream)
+            tm = timeit(m2d)
+            row.update({"memcpy2d_us": round(tm * 1e3, 2), "memcpy2d_gbs": gb(tm),
+                        "pack_vs_memcpy2d": round(tm / tp, 3)})
+        print(json.dumps(row), flush=True)
         del src, pk, dst, a, b
         torch.cuda.empty_cache()
 
