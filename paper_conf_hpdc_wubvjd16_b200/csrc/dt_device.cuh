@@ -413,6 +413,173 @@ __device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64
   }
 }
 
+// ---------------------------------------------------------------- async staging
+// cp.async (LDGSTS) gathers G-byte words straight into shared memory without
+// holding them in registers, so a CTA keeps tens of KiB in flight; the
+// contiguous side moves with TMA bulk copies (cp.async.bulk, UBLKCP): one
+// instruction per tile.  This is the shared-memory/TMA staging of short runs.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+template <int G>
+__device__ __forceinline__ void cp_async(void* smem, const void* gmem) {
+  if (G == 16)
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+  else
+    asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(smem_u32(smem)), "l"(gmem), "n"(G) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ void bulk_store(void* gmem, const void* smem, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gmem), "r"(smem_u32(smem)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void mbar_init(uint64_t* m, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(m)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* m, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(m)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* smem, const void* gmem, uint32_t bytes, uint64_t* m) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(smem)),
+               "l"(gmem), "r"(bytes), "r"(smem_u32(m))
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* m, uint32_t parity) {
+  asm volatile(
+      "{\n.reg .pred p;\nWAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(m)),
+      "r"(parity)
+      : "memory");
+}
+
+constexpr int kStageTile = 16384, kStageBufs = 3;
+
+// Word iterator: thread walks stream words x, x+S, x+2S, ... keeping (element,
+// offset) incrementally (one fast division at the start of a tile).
+struct WordIt {
+  uint64_t e;
+  int64_t q, ed;
+};
+
+// Pack stream bytes [lo, hi) (lo - P.pos and P.c 16-byte aligned) of a G-granular
+// template through shared memory: per tile, every thread cp.async-gathers its
+// words into the tile buffer; the finished tile leaves with one bulk store.
+template <int G>
+__device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64_t lo, int64_t hi, uint8_t* sbuf) {
+  constexpr int T = kStageTile, NB = kStageBufs;
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  const int64_t ntiles = (hi - lo + T - 1) / T;
+  for (int64_t t = 0; t <= ntiles; t++) {
+    if (t < ntiles) {
+      uint8_t* buf = sbuf + (t % NB) * T;
+      if (tid == 0) bulk_wait_read<NB - 2>();  // the store that last read this buffer is done reading
+      __syncthreads();
+      const int64_t s0 = lo + t * T;
+      const int64_t nw = (hi - s0 < T ? hi - s0 : (int64_t)T) / G;
+      int64_t i = tid;
+      if (i < nw) {
+        const int64_t x0 = s0 + i * G;
+        WordIt it;
+        it.e = fdiv((uint64_t)x0, P.ftsize);
+        it.q = x0 - (int64_t)it.e * P.tsize;
+        it.ed = elem_disp(P, it.e);
+        const int64_t S = (int64_t)nthr * G;
+        const int64_t Se = S / P.tsize, Sq = S - Se * P.tsize;
+        while (true) {
+          cp_async<G>(buf + i * G, P.nc + it.ed + wt[it.q / G]);
+          i += nthr;
+          if (i >= nw) break;
+          it.q += Sq;
+          uint64_t ne = it.e + Se;
+          if (it.q >= P.tsize) { it.q -= P.tsize; ne++; }
+          if (ne != it.e) { it.e = ne; it.ed = elem_disp(P, ne); }
+        }
+      }
+      cp_async_commit();
+    }
+    if (t >= 1) {
+      if (t < ntiles) cp_async_wait<1>();
+      else cp_async_wait<0>();
+      __syncthreads();
+      if (tid == 0) {
+        const int64_t s1 = lo + (t - 1) * T;
+        const int64_t tl = hi - s1 < T ? hi - s1 : (int64_t)T;
+        const uint8_t* buf = sbuf + ((t - 1) % NB) * T;
+        fence_proxy_async();
+        if (tl >= 16) {
+          bulk_store(P.c + (s1 - P.pos), buf, (uint32_t)(tl & ~int64_t(15)));
+          bulk_commit();
+        }
+        for (int64_t k = tl & ~int64_t(15); k < tl; k++) P.c[s1 - P.pos + k] = buf[k];  // ragged tail
+      }
+    }
+  }
+  if (tid == 0) bulk_wait_all();
+}
+
+// Unpack: tiles of the contiguous stream arrive by TMA bulk loads (NB in flight,
+// mbarrier completion), then every thread scatters its words from shared memory.
+template <int G>
+__device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int64_t lo, int64_t hi, uint8_t* sbuf,
+                                             uint64_t* mbar) {
+  typedef typename WordT<G>::T W;
+  constexpr int T = kStageTile, NB = kStageBufs;
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  const int64_t ntiles = (hi - lo + T - 1) / T;
+  if (tid == 0) {
+    for (int b = 0; b < NB; b++) mbar_init(mbar + b, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](int64_t t) {
+    const int64_t s = lo + t * T;
+    const uint32_t bytes = (uint32_t)((hi - s < T ? hi - s : (int64_t)T) & ~int64_t(15));
+    uint64_t* m = mbar + (t % NB);
+    mbar_expect_tx(m, bytes);
+    if (bytes) bulk_load(sbuf + (t % NB) * T, P.c + (s - P.pos), bytes, m);
+  };
+  if (tid == 0)
+    for (int64_t t = 0; t < NB && t < ntiles; t++) issue(t);
+  for (int64_t t = 0; t < ntiles; t++) {
+    const uint8_t* buf = sbuf + (t % NB) * T;
+    mbar_wait(mbar + (t % NB), (uint32_t)((t / NB) & 1));
+    const int64_t s0 = lo + t * T;
+    const int64_t tl = hi - s0 < T ? hi - s0 : (int64_t)T;
+    const int64_t nw = tl / G, full = (tl & ~int64_t(15)) / G;
+    int64_t i = tid;
+    if (i < nw) {
+      const int64_t x0 = s0 + i * G;
+      WordIt it;
+      it.e = fdiv((uint64_t)x0, P.ftsize);
+      it.q = x0 - (int64_t)it.e * P.tsize;
+      it.ed = elem_disp(P, it.e);
+      const int64_t S = (int64_t)nthr * G;
+      const int64_t Se = S / P.tsize, Sq = S - Se * P.tsize;
+      while (true) {
+        const W v = i < full ? *reinterpret_cast<const W*>(buf + i * G)
+                             : *reinterpret_cast<const W*>(P.c + (s0 + i * G - P.pos));  // ragged tail
+        *reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + it.ed + wt[it.q / G]) = v;
+        i += nthr;
+        if (i >= nw) break;
+        it.q += Sq;
+        uint64_t ne = it.e + Se;
+        if (it.q >= P.tsize) { it.q -= P.tsize; ne++; }
+        if (ne != it.e) { it.e = ne; it.ed = elem_disp(P, ne); }
+      }
+    }
+    __syncthreads();  // buffer consumed
+    if (tid == 0 && t + NB < ntiles) issue(t + NB);
+  }
+}
+
 // Short blocks under a large template (irregular hindexed, C5b): a warp walks its
 // stream slice in 512-byte windows.  For each window, lanes take one block each
 // (32 per round, block starts from boff) and write the source address of every

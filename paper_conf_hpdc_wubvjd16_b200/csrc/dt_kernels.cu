@@ -135,6 +135,25 @@ __global__ void __launch_bounds__(256) k_blk(const KP P) {
   blk_range<UNPACK, G, LD_CS>(P, p, p1, lane, sa);
 }
 
+// shared-memory staged pack/unpack (cp.async gathers / TMA bulk), CTA c owns a
+// contiguous run of 16 KiB tiles of the stream
+template <bool UNPACK, int G>
+__global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
+  extern __shared__ __align__(128) uint8_t smem_stage[];
+  __shared__ uint64_t mbar[kStageBufs];
+  uint8_t* sbuf = smem_stage;
+  int32_t* wt = reinterpret_cast<int32_t*>(smem_stage + kStageBufs * kStageTile);
+  for (int i = threadIdx.x; i < P.nwords; i += blockDim.x) wt[i] = P.wtab[i];
+  __syncthreads();
+  const int64_t t0 = ntiles * blockIdx.x / gridDim.x, t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
+  const int64_t end = P.pos + P.len;
+  const int64_t lo = P.pos + t0 * kStageTile;
+  const int64_t hi = P.pos + t1 * kStageTile < end ? P.pos + t1 * kStageTile : end;
+  if (lo >= hi) return;
+  if (UNPACK) stage_unpack<G>(P, wt, lo, hi, sbuf, mbar);
+  else stage_pack<G>(P, wt, lo, hi, sbuf);
+}
+
 template <bool UNPACK, int G, int VW>
 __global__ void __launch_bounds__(256) k_word(const KP P) {
   extern __shared__ int32_t wt[];
@@ -395,10 +414,13 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   *gran = g;
   const double mean = (double)ts / (double)nb;
   const bool word_ok = ts / g <= kMaxWordTable && ts % g == 0 && template_fits_int32(f);
-  static const int force = getenv("DT_FORCE_KERNEL") ? atoi(getenv("DT_FORCE_KERNEL")) : 0;  // tuning aid
+  const char* fk = getenv("DT_FORCE_KERNEL");  // tuning / test aid: force a kernel family when applicable
+  const int force = fk ? atoi(fk) : 0;
   const bool blk_ok = (c_addr & 15) == 0 && ts % g == 0;
+  const bool stage_ok = word_ok && g >= 4 && (c_addr & 15) == 0;
   if (force == 2 && word_ok) return 2;
   if (force == 3 && blk_ok) return 3;
+  if (force == 4 && stage_ok) return 4;
   if (force == 1) return 1;
   // word kernel: short blocks, or co-aligned runs up to 1 KiB (one 16-byte word per
   // thread-vector beats a warp per 512-byte run: C3 0.71 vs 0.44 of copy, measured)
@@ -488,6 +510,33 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
       if (single) k_seg<false, true><<<grid, 256, 0, s>>>(P, plan, nw);
       else k_seg<false, false><<<grid, 256, 0, s>>>(P, plan, nw);
     }
+  } else if (kind == 4) {
+    const int32_t* wt = nullptr;
+    dt_status st = ensure_wtab(f, dd, g, &wt);
+    if (st != DT_OK) return st;
+    P.wtab = wt;
+    P.nwords = (int32_t)(f.tsize() / g);
+    const size_t smem = (size_t)kStageBufs * kStageTile + sizeof(int32_t) * (size_t)P.nwords;
+    const int64_t ntiles = (len + kStageTile - 1) / kStageTile;
+    static bool attr_set = false;
+    if (!attr_set) {
+      const void* fs[] = {(const void*)k_stage<false, 4>, (const void*)k_stage<false, 8>,
+                          (const void*)k_stage<false, 16>, (const void*)k_stage<true, 4>,
+                          (const void*)k_stage<true, 8>, (const void*)k_stage<true, 16>};
+      for (const void* fp : fs) cudaFuncSetAttribute(fp, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+      attr_set = true;
+    }
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage<false, 4>, 256, smem) != cudaSuccess || occ < 1)
+      occ = 1;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
+#define LS(U, G) k_stage<U, G><<<grid, 256, smem, s>>>(P, ntiles)
+    if (unpack) {
+      switch (g) { case 4: LS(true, 4); break; case 8: LS(true, 8); break; default: LS(true, 16); break; }
+    } else {
+      switch (g) { case 4: LS(false, 4); break; case 8: LS(false, 8); break; default: LS(false, 16); break; }
+    }
+#undef LS
   } else if (kind == 3) {
     P.fnb = make_fd((uint64_t)P.nblocks);
     const int64_t max_warps = (int64_t)sms * 4 * 8;

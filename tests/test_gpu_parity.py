@@ -170,6 +170,24 @@ def test_random_tiny_types(torch_cuda):
                 raise
 
 
+@pytest.mark.parametrize("kind", ["1", "2", "3", "4"])
+@pytest.mark.parametrize("name", ["C1b", "C2s", "C3s", "C4x", "C4y", "C5", "C5b", "ctg"])
+def test_every_kernel_family(torch_cuda, kind, name, monkeypatch):
+    """Every kernel family (1 warp segments, 2 word table, 3 block windows, 4 smem/TMA
+    staging) on every workload it accepts, forced through DT_FORCE_KERNEL, with
+    ragged pos/len (the planner falls back when a family does not apply)."""
+    mk = {"C1b": lambda: c1_submatrix(256, 1024, 1, 1), "C2s": lambda: c2_lower_triangle(700),
+          "C3s": lambda: c3_block_cyclic(1024, 64), "C4x": lambda: c4_face("x+", 96),
+          "C4y": lambda: c4_face("y-", 96, 1, True), "C5": lambda: c5_particles(1 << 20),
+          "C5b": lambda: c5b_irregular(1 << 20), "ctg": lambda: (("contiguous", 3000, ("basic", "INT32")), 0, 12000)}
+    rec, org, parent = mk[name]()
+    monkeypatch.setenv("DT_FORCE_KERNEL", kind)
+    size = oracle.from_recipe(rec).size
+    check_pack_unpack(torch_cuda, rec, org, parent)
+    check_pack_unpack(torch_cuda, rec, org, parent, count=2, pos=48, nbytes=2 * size - 48 - 16)
+    check_pack_unpack(torch_cuda, rec, org, parent, pos=20, nbytes=size - 37)
+
+
 def test_unpack_rejects_overlap(torch_cuda):
     import torch
     from paper_conf_hpdc_wubvjd16_b200 import dt
