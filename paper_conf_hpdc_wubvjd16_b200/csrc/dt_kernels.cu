@@ -422,9 +422,10 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   if (force == 3 && blk_ok) return 3;
   if (force == 4 && stage_ok) return 4;
   if (force == 1) return 1;
-  // word kernel: short blocks, or co-aligned runs up to 1 KiB (one 16-byte word per
-  // thread-vector beats a warp per 512-byte run: C3 0.71 vs 0.44 of copy, measured)
-  if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return 2;
+  // short blocks / co-aligned runs up to 1 KiB: with >= 8-byte words the smem/TMA
+  // staged kernel wins (C3 pack 0.78 of copy vs 0.66 word table vs 0.44 warp
+  // segments; measured), with 4-byte words the register word kernel does
+  if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return stage_ok && g >= 8 ? 4 : 2;
   if (mean < 128.0 && blk_ok) return 3;
   return 1;
 }

@@ -64,7 +64,9 @@ struct XOp {
 
 struct XArgs {
   int32_t nops;
-  int32_t flags;  // tuning switches (DT_XFER_FLAGS): bit0 = no sys fence before the flag, bit1 = no sleep in polls
+  int32_t wt_off;  // byte offset of the word table in dynamic smem (after the staging buffers)
+  int32_t flags;
+  int32_t pad2;  // tuning switches (DT_XFER_FLAGS): bit0 = no sys fence before the flag, bit1 = no sleep in polls
   int64_t timeout_ns;
   XOp ops[kMaxOps];
 };
@@ -111,11 +113,24 @@ __device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeo
 // pack or unpack stream bytes [lo, lo+len) of the current chunk with this CTA.
 template <bool UNPACK>
 __device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int64_t lo, int64_t len,
-                                          const int32_t* wt) {
+                                          const int32_t* wt, uint8_t* sbuf, uint64_t* mbar) {
   P.c = slot + lo;  // slot maps stream byte 0 of the message (see caller)
   P.pos = lo;
   P.len = len;
   constexpr int POL = UNPACK ? LD_CG : LD_CS;  // ring slots are rewritten by the peer: bypass L1
+  if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
+    switch (X.g) {
+      case 8:
+        if (UNPACK) stage_unpack<8>(P, wt, lo, lo + len, sbuf, mbar);
+        else stage_pack<8>(P, wt, lo, lo + len, sbuf);
+        break;
+      default:
+        if (UNPACK) stage_unpack<16>(P, wt, lo, lo + len, sbuf, mbar);
+        else stage_pack<16>(P, wt, lo, lo + len, sbuf);
+        break;
+    }
+    return;
+  }
   if (X.kind == 2) {
     const int64_t body = len - len % X.g;
     KP Q = P;
@@ -142,7 +157,11 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int
 
 constexpr int kXferThreads = 512;
 __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
-  extern __shared__ int32_t wt[];
+  // dynamic smem: [staging buffers (if any op stages)] [word table]
+  extern __shared__ __align__(128) uint8_t xsm[];
+  __shared__ uint64_t mbar[kStageBufs];
+  uint8_t* sbuf = xsm;
+  int32_t* wt = reinterpret_cast<int32_t*>(xsm + A.wt_off);
   __shared__ uint64_t s_val;
   __shared__ int s_stop, s_gs;
   int op = 0;
@@ -151,6 +170,8 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   const XOp& X = A.ops[op];
   const int j = (int)blockIdx.x - X.cta0;
   if (X.kind == 2)
+    for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
+  if (X.kind == 4)
     for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
   const int64_t C = X.chunk;
   const int D = X.depth;
@@ -233,8 +254,8 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       }
       __syncthreads();
       if (s_stop) return;
-      if (X.role == 0) cta_chunk<false>(X, X.P, sl, off, len, wt);
-      else cta_chunk<true>(X, X.P, sl, off, len, wt);
+      if (X.role == 0) cta_chunk<false>(X, X.P, sl, off, len, wt, sbuf, mbar);
+      else cta_chunk<true>(X, X.P, sl, off, len, wt, sbuf, mbar);
       __syncthreads();
       if (threadIdx.x == 0) {
         if (!(A.flags & 1)) __threadfence_system();
@@ -619,11 +640,12 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   int64_t g = 1;
   // chunk starts are multiples of `chunk` (a multiple of 512) and ring slots are aligned
   int kind = plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
-  if (kind == 2 && lowp2u((uint64_t)chunk) < g) kind = 1;
-  X.kind = kind == 2 ? 2 : 1;
+  if ((kind == 2 || kind == 4) && lowp2u((uint64_t)chunk) < g) kind = 1;
+  if (kind == 4 && g < 8) kind = 2;
+  X.kind = (kind == 2 || kind == 4) ? kind : 1;  // the block-window kernel (3) is not used inside the pipeline
   X.single = P.nblocks == 1;
   X.g = (int32_t)g;
-  if (X.kind == 2) {
+  if (X.kind == 2 || X.kind == 4) {
     const int32_t* wt = nullptr;
     st = ensure_wtab_pub(f, *dd, g, &wt);
     if (st != DT_OK) return st;
@@ -643,6 +665,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   A.flags = getenv("DT_XFER_FLAGS") ? atoi(getenv("DT_XFER_FLAGS")) : 0;
   int nops = 0, cta = 0;
   size_t smem = 0;
+  bool any_stage = false;
   std::vector<int> sch(c->nranks, 0), rch(c->nranks, 0);
   const int G = default_ctas(c);
   for (const auto& p : ops) {
@@ -670,7 +693,8 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.base_out = c->base(par ^ 1, 0, p.dest, ch);
       X.seq = ++sq;
       X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
-      if (X.kind == 2) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+      if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+      any_stage = any_stage || X.kind == 4;
     }
     if (p.source >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
@@ -696,11 +720,15 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.base_out = c->base(par ^ 1, 1, p.source, ch);
       X.seq = ++sq;
       X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
-      if (X.kind == 2) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+      if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+      any_stage = any_stage || X.kind == 4;
     }
   }
   if (nops == 0) return DT_OK;
   A.nops = nops;
+  A.wt_off = any_stage ? kStageBufs * kStageTile : 0;
+  smem += (size_t)A.wt_off;
+  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA must be co-resident: fit the per-op CTA count to the occupancy
   int occ = 0;
   CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_xfer, kXferThreads, smem));
@@ -720,7 +748,6 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
     A.ops[i].ncta = n_i;
     cta += n_i;
   }
-  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
   CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
