@@ -460,7 +460,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* m, uint32_t parity) {
       : "memory");
 }
 
-constexpr int kStageTile = 16384, kStageBufs = 3;
+constexpr int kStageTile = 16384;
+constexpr int kStageBufs = 4;      // standalone kernels (several CTAs per SM)
+constexpr int kXferStageBufs = 8;  // transfer kernel (one CTA per SM carries a whole sub-ring)
 
 // Word iterator: thread walks stream words x, x+S, x+2S, ... keeping (element,
 // offset) incrementally (one fast division at the start of a tile).
@@ -472,15 +474,17 @@ struct WordIt {
 // Pack stream bytes [lo, hi) (lo - P.pos and P.c 16-byte aligned) of a G-granular
 // template through shared memory: per tile, every thread cp.async-gathers its
 // words into the tile buffer; the finished tile leaves with one bulk store.
-template <int G>
+// NB tile buffers: NB-1 tiles of gathers in flight while the oldest finished tile
+// is stored, so a CTA keeps (NB-1)*16 KiB of loads outstanding.
+template <int G, int NB>
 __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64_t lo, int64_t hi, uint8_t* sbuf) {
-  constexpr int T = kStageTile, NB = kStageBufs;
+  constexpr int T = kStageTile, L = NB - 1;
   const int tid = threadIdx.x, nthr = blockDim.x;
   const int64_t ntiles = (hi - lo + T - 1) / T;
-  for (int64_t t = 0; t <= ntiles; t++) {
+  for (int64_t t = 0; t < ntiles + L - 1; t++) {
     if (t < ntiles) {
       uint8_t* buf = sbuf + (t % NB) * T;
-      if (tid == 0) bulk_wait_read<NB - 2>();  // the store that last read this buffer is done reading
+      if (tid == 0) bulk_wait_read<1>();  // the store that last read this buffer (tile t-NB) is done reading
       __syncthreads();
       const int64_t s0 = lo + t * T;
       const int64_t nw = (hi - s0 < T ? hi - s0 : (int64_t)T) / G;
@@ -503,16 +507,16 @@ __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64
           if (ne != it.e) { it.e = ne; it.ed = elem_disp(P, ne); }
         }
       }
-      cp_async_commit();
     }
-    if (t >= 1) {
-      if (t < ntiles) cp_async_wait<1>();
-      else cp_async_wait<0>();
+    cp_async_commit();  // (an empty group in the drain iterations keeps the group count uniform)
+    const int64_t u = t - (L - 1);  // oldest tile in flight: store it once its gathers landed
+    if (u >= 0) {
+      cp_async_wait<L - 1>();
       __syncthreads();
       if (tid == 0) {
-        const int64_t s1 = lo + (t - 1) * T;
+        const int64_t s1 = lo + u * T;
         const int64_t tl = hi - s1 < T ? hi - s1 : (int64_t)T;
-        const uint8_t* buf = sbuf + ((t - 1) % NB) * T;
+        const uint8_t* buf = sbuf + (u % NB) * T;
         fence_proxy_async();
         if (tl >= 16) {
           bulk_store(P.c + (s1 - P.pos), buf, (uint32_t)(tl & ~int64_t(15)));
@@ -527,11 +531,11 @@ __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64
 
 // Unpack: tiles of the contiguous stream arrive by TMA bulk loads (NB in flight,
 // mbarrier completion), then every thread scatters its words from shared memory.
-template <int G>
+template <int G, int NB>
 __device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int64_t lo, int64_t hi, uint8_t* sbuf,
                                              uint64_t* mbar) {
   typedef typename WordT<G>::T W;
-  constexpr int T = kStageTile, NB = kStageBufs;
+  constexpr int T = kStageTile;
   const int tid = threadIdx.x, nthr = blockDim.x;
   const int64_t ntiles = (hi - lo + T - 1) / T;
   if (tid == 0) {

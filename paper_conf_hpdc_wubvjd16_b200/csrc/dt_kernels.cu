@@ -150,8 +150,8 @@ __global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
   const int64_t lo = P.pos + t0 * kStageTile;
   const int64_t hi = P.pos + t1 * kStageTile < end ? P.pos + t1 * kStageTile : end;
   if (lo >= hi) return;
-  if (UNPACK) stage_unpack<G>(P, wt, lo, hi, sbuf, mbar);
-  else stage_pack<G>(P, wt, lo, hi, sbuf);
+  if (UNPACK) stage_unpack<G, kStageBufs>(P, wt, lo, hi, sbuf, mbar);
+  else stage_pack<G, kStageBufs>(P, wt, lo, hi, sbuf);
 }
 
 template <bool UNPACK, int G, int VW>

@@ -121,12 +121,12 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
     switch (X.g) {
       case 8:
-        if (UNPACK) stage_unpack<8>(P, wt, lo, lo + len, sbuf, mbar);
-        else stage_pack<8>(P, wt, lo, lo + len, sbuf);
+        if (UNPACK) stage_unpack<8, kXferStageBufs>(P, wt, lo, lo + len, sbuf, mbar);
+        else stage_pack<8, kXferStageBufs>(P, wt, lo, lo + len, sbuf);
         break;
       default:
-        if (UNPACK) stage_unpack<16>(P, wt, lo, lo + len, sbuf, mbar);
-        else stage_pack<16>(P, wt, lo, lo + len, sbuf);
+        if (UNPACK) stage_unpack<16, kXferStageBufs>(P, wt, lo, lo + len, sbuf, mbar);
+        else stage_pack<16, kXferStageBufs>(P, wt, lo, lo + len, sbuf);
         break;
     }
     return;
@@ -159,7 +159,7 @@ constexpr int kXferThreads = 512;
 __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
   // dynamic smem: [staging buffers (if any op stages)] [word table]
   extern __shared__ __align__(128) uint8_t xsm[];
-  __shared__ uint64_t mbar[kStageBufs];
+  __shared__ uint64_t mbar[kXferStageBufs];
   uint8_t* sbuf = xsm;
   int32_t* wt = reinterpret_cast<int32_t*>(xsm + A.wt_off);
   __shared__ uint64_t s_val;
@@ -726,7 +726,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   }
   if (nops == 0) return DT_OK;
   A.nops = nops;
-  A.wt_off = any_stage ? kStageBufs * kStageTile : 0;
+  A.wt_off = any_stage ? kXferStageBufs * kStageTile : 0;
   smem += (size_t)A.wt_off;
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA must be co-resident: fit the per-op CTA count to the occupancy
