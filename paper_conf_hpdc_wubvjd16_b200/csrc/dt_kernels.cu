@@ -493,7 +493,10 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
   int64_t g = 1;
   int kind = E.merged ? 1 : plan_kernel(f, L, (uint64_t)(uintptr_t)nc, (uint64_t)(uintptr_t)c, pos, len, &g);
   if (kind == 0) return DT_OK;
-  const int sms = num_sms();
+  // grids are sized in SMs' worth of resident CTAs; DT_MAX_SMS caps it (f3: how few
+  // SMs a pack/unpack needs, e.g. to leave the rest to a co-running application)
+  const char* ms = getenv("DT_MAX_SMS");
+  const int sms = ms && atoi(ms) > 0 ? std::min(num_sms(), atoi(ms)) : num_sms();
   if (kind == 1) {
     // exactly one wave of resident CTAs (no tail wave), at least ~4 KiB per warp
     const bool single = P.nblocks == 1;
