@@ -464,8 +464,42 @@ constexpr int kStageTile = 16384;
 constexpr int kStageBufs = 4;      // standalone kernels (several CTAs per SM)
 constexpr int kXferStageBufs = 8;  // transfer kernel (one CTA per SM carries a whole sub-ring)
 
+// Element iterator: element e = hi*cnt[L] + lo over the innermost level L.  The
+// displacement of the outer nest (hi) is cached; advancing by k elements touches
+// only lo and recomputes the outer part when lo wraps (once per cnt[L] elements).
+struct ElemIt {
+  uint64_t hi;
+  int64_t lo, hid;  // hid = displacement of element hi*cnt[L] without level L's contribution
+  int L;
+  __device__ __forceinline__ void init(const KP& P, uint64_t e) {
+    L = P.nlev - 1;
+    if (L < 0) { hi = e; lo = 0; hid = 0; return; }
+    hi = fdiv(e, P.fcnt[L]);
+    lo = (int64_t)(e - hi * (uint64_t)P.cnt[L]);
+    outer(P);
+  }
+  __device__ __forceinline__ void outer(const KP& P) {
+    const uint64_t e0 = hi * (uint64_t)P.cnt[L];
+    hid = elem_disp(P, e0) - (P.table[L] ? __ldg(P.table[L]) : 0);
+  }
+  __device__ __forceinline__ int64_t disp(const KP& P) const {
+    if (L < 0) return 0;
+    return hid + (P.table[L] ? __ldg(P.table[L] + lo) : lo * P.stride[L]);
+  }
+  __device__ __forceinline__ void advance(const KP& P, int64_t k) {
+    if (L < 0 || k == 0) return;
+    lo += k;
+    if (lo >= P.cnt[L]) {
+      const uint64_t q = fdiv((uint64_t)lo, P.fcnt[L]);
+      hi += q;
+      lo -= (int64_t)q * P.cnt[L];
+      outer(P);
+    }
+  }
+};
+
 // Word iterator: thread walks stream words x, x+S, x+2S, ... keeping (element,
-// offset) incrementally (one fast division at the start of a tile).
+// offset within the element) incrementally (one fast division per tile).
 struct WordIt {
   uint64_t e;
   int64_t q, ed;
@@ -481,6 +515,8 @@ __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64
   constexpr int T = kStageTile, L = NB - 1;
   const int tid = threadIdx.x, nthr = blockDim.x;
   const int64_t ntiles = (hi - lo + T - 1) / T;
+  const int64_t S = (int64_t)nthr * G;  // a thread's stride through the stream: Se elements + Sq bytes
+  const int64_t Se = (int64_t)fdiv((uint64_t)S, P.ftsize), Sq = S - Se * P.tsize;
   for (int64_t t = 0; t < ntiles + L - 1; t++) {
     if (t < ntiles) {
       uint8_t* buf = sbuf + (t % NB) * T;
@@ -491,20 +527,19 @@ __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64
       int64_t i = tid;
       if (i < nw) {
         const int64_t x0 = s0 + i * G;
-        WordIt it;
-        it.e = fdiv((uint64_t)x0, P.ftsize);
-        it.q = x0 - (int64_t)it.e * P.tsize;
-        it.ed = elem_disp(P, it.e);
-        const int64_t S = (int64_t)nthr * G;
-        const int64_t Se = S / P.tsize, Sq = S - Se * P.tsize;
+        const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
+        int64_t q = x0 - (int64_t)e0 * P.tsize;
+        ElemIt ei;
+        ei.init(P, e0);
+        int64_t ed = ei.disp(P);
         while (true) {
-          cp_async<G>(buf + i * G, P.nc + it.ed + wt[it.q / G]);
+          cp_async<G>(buf + i * G, P.nc + ed + wt[q / G]);
           i += nthr;
           if (i >= nw) break;
-          it.q += Sq;
-          uint64_t ne = it.e + Se;
-          if (it.q >= P.tsize) { it.q -= P.tsize; ne++; }
-          if (ne != it.e) { it.e = ne; it.ed = elem_disp(P, ne); }
+          q += Sq;
+          int64_t k = Se;
+          if (q >= P.tsize) { q -= P.tsize; k++; }
+          if (k) { ei.advance(P, k); ed = ei.disp(P); }
         }
       }
     }
@@ -538,6 +573,8 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int
   constexpr int T = kStageTile;
   const int tid = threadIdx.x, nthr = blockDim.x;
   const int64_t ntiles = (hi - lo + T - 1) / T;
+  const int64_t S = (int64_t)nthr * G;
+  const int64_t Se = (int64_t)fdiv((uint64_t)S, P.ftsize), Sq = S - Se * P.tsize;
   if (tid == 0) {
     for (int b = 0; b < NB; b++) mbar_init(mbar + b, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -561,22 +598,21 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int
     int64_t i = tid;
     if (i < nw) {
       const int64_t x0 = s0 + i * G;
-      WordIt it;
-      it.e = fdiv((uint64_t)x0, P.ftsize);
-      it.q = x0 - (int64_t)it.e * P.tsize;
-      it.ed = elem_disp(P, it.e);
-      const int64_t S = (int64_t)nthr * G;
-      const int64_t Se = S / P.tsize, Sq = S - Se * P.tsize;
+      const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
+      int64_t q = x0 - (int64_t)e0 * P.tsize;
+      ElemIt ei;
+      ei.init(P, e0);
+      int64_t ed = ei.disp(P);
       while (true) {
         const W v = i < full ? *reinterpret_cast<const W*>(buf + i * G)
                              : *reinterpret_cast<const W*>(P.c + (s0 + i * G - P.pos));  // ragged tail
-        *reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + it.ed + wt[it.q / G]) = v;
+        *reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed + wt[q / G]) = v;
         i += nthr;
         if (i >= nw) break;
-        it.q += Sq;
-        uint64_t ne = it.e + Se;
-        if (it.q >= P.tsize) { it.q -= P.tsize; ne++; }
-        if (ne != it.e) { it.e = ne; it.ed = elem_disp(P, ne); }
+        q += Sq;
+        int64_t k = Se;
+        if (q >= P.tsize) { q -= P.tsize; k++; }
+        if (k) { ei.advance(P, k); ed = ei.disp(P); }
       }
     }
     __syncthreads();  // buffer consumed
