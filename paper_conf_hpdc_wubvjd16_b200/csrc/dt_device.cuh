@@ -256,9 +256,10 @@ __device__ __forceinline__ int64_t warp_find_block(const int64_t* __restrict__ b
 // Walk from a resolved start: stream byte p is byte r of block b of element e
 // (element displacement ed).  The next block's descriptor is prefetched while the
 // current segment is copied.
+// cb: packed-side base such that stream byte p lives at cb + p (cb = c - pos).
 template <bool UNPACK, bool SINGLE, int POL>
-__device__ __forceinline__ void seg_walk(const KP& P, int64_t p, const int64_t p1, int64_t b, int64_t r, uint64_t e,
-                                         int64_t ed, const int lane) {
+__device__ __forceinline__ void seg_walk(const KP& P, uint8_t* cb, int64_t p, const int64_t p1, int64_t b, int64_t r,
+                                         uint64_t e, int64_t ed, const int lane) {
   int64_t blen = SINGLE ? P.bl0 : __ldg(P.bl + b);
   int64_t bdsp = SINGLE ? P.bd0 : __ldg(P.bd + b);
   while (true) {
@@ -270,7 +271,7 @@ __device__ __forceinline__ void seg_walk(const KP& P, int64_t p, const int64_t p
       nbdsp = __ldg(P.bd + nb);
     }
     uint8_t* ncp = const_cast<uint8_t*>(P.nc) + ed + bdsp + r;
-    uint8_t* cp = P.c + (p - P.pos);
+    uint8_t* cp = cb + p;
     if (UNPACK) warp_copy<POL>(ncp, cp, seg, lane);
     else warp_copy<POL>(cp, ncp, seg, lane);
     p += seg;
@@ -289,7 +290,7 @@ __device__ __forceinline__ void seg_walk(const KP& P, int64_t p, const int64_t p
 }
 
 template <bool UNPACK, bool SINGLE, int POL>
-__device__ __forceinline__ void seg_range(const KP& P, int64_t p, const int64_t p1, const int lane) {
+__device__ __forceinline__ void seg_range(const KP& P, uint8_t* cb, int64_t p, const int64_t p1, const int lane) {
   if (p >= p1) return;
   uint64_t e = fdiv((uint64_t)p, P.ftsize);
   int64_t r = p - (int64_t)e * P.tsize;
@@ -298,7 +299,7 @@ __device__ __forceinline__ void seg_range(const KP& P, int64_t p, const int64_t 
     b = warp_find_block(P.boff, P.nblocks, r, lane);
     r -= __ldg(P.boff + b);
   }
-  seg_walk<UNPACK, SINGLE, POL>(P, p, p1, b, r, e, elem_disp(P, e), lane);
+  seg_walk<UNPACK, SINGLE, POL>(P, cb, p, p1, b, r, e, elem_disp(P, e), lane);
 }
 
 // ---------------------------------------------------------------- launch plans
@@ -349,17 +350,19 @@ template <> struct WordT<8> { typedef unsigned long long T; };
 template <> struct WordT<16> { typedef uint4 T; };
 
 // Threads tid, tid+nthr, ... each handle one VW-byte vector of the packed
-// stream [P.pos, P.pos+P.len) (which must be G-aligned and G-granular); wt is
-// the template's word table in shared memory.
+// stream [lo, hi) (G-aligned, G-granular; cb + lo VW-aligned); wt is the
+// template's word table in shared memory.
 // NV vectors per thread and iteration: every load of the batch is issued before
 // the first store, so a thread keeps NV*VW bytes in flight.
 template <bool UNPACK, int G, int VW, int POL, int NV = 2>
-__device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64_t tid, int64_t nthr) {
+__device__ __forceinline__ void word_range(const KP& P, uint8_t* cb, const int64_t lo, const int64_t hi,
+                                           const int32_t* wt, int64_t tid, int64_t nthr) {
   typedef typename WordT<G>::T W;
   typedef typename WordT<VW>::T VT;
   constexpr int NW = VW / G;
-  const int64_t nvec = (P.len + VW - 1) / VW;
-  const int64_t end = P.pos + P.len;
+  const int64_t nvec = (hi - lo + VW - 1) / VW;
+  const int64_t end = hi;
+  uint8_t* const cv = cb + lo;  // vector v of the range lives at cv + v*VW
   union U {
     VT vec;
     W word[NW];
@@ -373,16 +376,16 @@ __device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64
 #pragma unroll
     for (int j = 0; j < NV; j++) {
       const int64_t v = v0 + (int64_t)j * nthr;
-      const int64_t s0 = P.pos + v * VW;
+      const int64_t s0 = lo + v * VW;
       const int64_t rem = v < nvec ? (end - s0) / G : 0;
       nvalid[j] = rem < NW ? (int)rem : NW;
       e[j] = fdiv((uint64_t)s0, P.ftsize);
       w[j] = (int)((s0 - (int64_t)e[j] * P.tsize) / G);
       ed[j] = nvalid[j] > 0 ? elem_disp(P, e[j]) : 0;
       if (UNPACK) {
-        if (nvalid[j] == NW) u[j].vec = ldv<POL>(reinterpret_cast<const VT*>(P.c + v * VW));
+        if (nvalid[j] == NW) u[j].vec = ldv<POL>(reinterpret_cast<const VT*>(cv + v * VW));
         else
-          for (int k = 0; k < nvalid[j]; k++) u[j].word[k] = reinterpret_cast<const W*>(P.c + v * VW)[k];
+          for (int k = 0; k < nvalid[j]; k++) u[j].word[k] = reinterpret_cast<const W*>(cv + v * VW)[k];
       }
     }
 #pragma unroll
@@ -405,9 +408,9 @@ __device__ __forceinline__ void word_range(const KP& P, const int32_t* wt, int64
 #pragma unroll
       for (int j = 0; j < NV; j++) {
         const int64_t v = v0 + (int64_t)j * nthr;
-        if (nvalid[j] == NW) stv(reinterpret_cast<VT*>(P.c + v * VW), u[j].vec);
+        if (nvalid[j] == NW) stv(reinterpret_cast<VT*>(cv + v * VW), u[j].vec);
         else
-          for (int k = 0; k < nvalid[j]; k++) reinterpret_cast<W*>(P.c + v * VW)[k] = u[j].word[k];
+          for (int k = 0; k < nvalid[j]; k++) reinterpret_cast<W*>(cv + v * VW)[k] = u[j].word[k];
       }
     }
   }
@@ -511,7 +514,8 @@ struct WordIt {
 // NB tile buffers: NB-1 tiles of gathers in flight while the oldest finished tile
 // is stored, so a CTA keeps (NB-1)*16 KiB of loads outstanding.
 template <int G, int NB>
-__device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64_t lo, int64_t hi, uint8_t* sbuf) {
+__device__ __forceinline__ void stage_pack(const KP& P, uint8_t* cb, const int32_t* wt, int64_t lo, int64_t hi,
+                                           uint8_t* sbuf) {
   constexpr int T = kStageTile, L = NB - 1;
   const int tid = threadIdx.x, nthr = blockDim.x;
   const int64_t ntiles = (hi - lo + T - 1) / T;
@@ -554,10 +558,10 @@ __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64
         const uint8_t* buf = sbuf + (u % NB) * T;
         fence_proxy_async();
         if (tl >= 16) {
-          bulk_store(P.c + (s1 - P.pos), buf, (uint32_t)(tl & ~int64_t(15)));
+          bulk_store(cb + s1, buf, (uint32_t)(tl & ~int64_t(15)));
           bulk_commit();
         }
-        for (int64_t k = tl & ~int64_t(15); k < tl; k++) P.c[s1 - P.pos + k] = buf[k];  // ragged tail
+        for (int64_t k = tl & ~int64_t(15); k < tl; k++) cb[s1 + k] = buf[k];  // ragged tail
       }
     }
   }
@@ -567,8 +571,8 @@ __device__ __forceinline__ void stage_pack(const KP& P, const int32_t* wt, int64
 // Unpack: tiles of the contiguous stream arrive by TMA bulk loads (NB in flight,
 // mbarrier completion), then every thread scatters its words from shared memory.
 template <int G, int NB>
-__device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int64_t lo, int64_t hi, uint8_t* sbuf,
-                                             uint64_t* mbar) {
+__device__ __forceinline__ void stage_unpack(const KP& P, const uint8_t* cb, const int32_t* wt, int64_t lo, int64_t hi,
+                                             uint8_t* sbuf, uint64_t* mbar) {
   typedef typename WordT<G>::T W;
   constexpr int T = kStageTile;
   const int tid = threadIdx.x, nthr = blockDim.x;
@@ -585,7 +589,7 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int
     const uint32_t bytes = (uint32_t)((hi - s < T ? hi - s : (int64_t)T) & ~int64_t(15));
     uint64_t* m = mbar + (t % NB);
     mbar_expect_tx(m, bytes);
-    if (bytes) bulk_load(sbuf + (t % NB) * T, P.c + (s - P.pos), bytes, m);
+    if (bytes) bulk_load(sbuf + (t % NB) * T, cb + s, bytes, m);
   };
   if (tid == 0)
     for (int64_t t = 0; t < NB && t < ntiles; t++) issue(t);
@@ -605,7 +609,7 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int
       int64_t ed = ei.disp(P);
       while (true) {
         const W v = i < full ? *reinterpret_cast<const W*>(buf + i * G)
-                             : *reinterpret_cast<const W*>(P.c + (s0 + i * G - P.pos));  // ragged tail
+                             : *reinterpret_cast<const W*>(cb + s0 + i * G);  // ragged tail
         *reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed + wt[q / G]) = v;
         i += nthr;
         if (i >= nw) break;
@@ -628,14 +632,15 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const int32_t* wt, int
 // table's addresses and one coalesced 16-byte store (unpack: the reverse).
 constexpr int kBlkWin = 512;
 template <bool UNPACK, int G, int POL>
-__device__ __forceinline__ void blk_range(const KP& P, int64_t p0, const int64_t p1, int lane, int64_t* sa) {
+__device__ __forceinline__ void blk_range(const KP& P, uint8_t* cbase, int64_t p0, const int64_t p1, int lane,
+                                          int64_t* sa) {
   typedef typename WordT<G>::T W;
   const FastDiv& fnb = P.fnb;
   constexpr int NWL = 16 / G;  // words per lane
   if (p0 >= p1) return;
   uint64_t ce = fdiv((uint64_t)p0, P.ftsize);
   int64_t cb = warp_find_block(P.boff, P.nblocks, p0 - (int64_t)ce * P.tsize, lane);
-  const uint64_t nel = P.nblocks ? (uint64_t)((P.pos + P.len + P.tsize - 1) / P.tsize) : 0;
+  const uint64_t nel = P.nblocks ? (uint64_t)((p1 + P.tsize - 1) / P.tsize) : 0;  // elements this warp can touch
   for (int64_t q = p0; q < p1; q += kBlkWin) {
     const int64_t qe = min(q + kBlkWin, p1);
     while (true) {
@@ -673,7 +678,7 @@ __device__ __forceinline__ void blk_range(const KP& P, int64_t p0, const int64_t
     const int64_t x0 = q + (int64_t)lane * 16;
     const int64_t remw = x0 >= qe ? 0 : (qe - x0) / G;
     const int nvalid = remw < NWL ? (int)remw : NWL;
-    uint8_t* cp = P.c + (x0 - P.pos);
+    uint8_t* cp = cbase + x0;
     union {
       uint4 vec;
       W word[NWL];

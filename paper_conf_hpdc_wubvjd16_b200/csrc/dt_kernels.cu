@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(256, 3) k_seg(const KP P, const PlanEnt* __res
   const PlanEnt a = plan[gw];
   const int64_t p1 = plan[gw + 1].p;
   if (a.p >= p1) return;
-  seg_walk<UNPACK, SINGLE, LD_CS>(P, a.p, p1, a.b, a.r, a.e, a.ed, lane);
+  seg_walk<UNPACK, SINGLE, LD_CS>(P, P.c - P.pos, a.p, p1, a.b, a.r, a.e, a.ed, lane);
 }
 
 // one thread per warp boundary: cost-balanced cut positions (see PlanEnt)
@@ -132,7 +132,7 @@ __global__ void __launch_bounds__(256) k_blk(const KP P) {
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t p = P.pos + gw * P.per_warp;
   const int64_t p1 = min(p + P.per_warp, P.pos + P.len);
-  blk_range<UNPACK, G, LD_CS>(P, p, p1, lane, sa);
+  blk_range<UNPACK, G, LD_CS>(P, P.c - P.pos, p, p1, lane, sa);
 }
 
 // shared-memory staged pack/unpack (cp.async gathers / TMA bulk), CTA c owns a
@@ -150,8 +150,8 @@ __global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
   const int64_t lo = P.pos + t0 * kStageTile;
   const int64_t hi = P.pos + t1 * kStageTile < end ? P.pos + t1 * kStageTile : end;
   if (lo >= hi) return;
-  if (UNPACK) stage_unpack<G, kStageBufs>(P, wt, lo, hi, sbuf, mbar);
-  else stage_pack<G, kStageBufs>(P, wt, lo, hi, sbuf);
+  if (UNPACK) stage_unpack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf, mbar);
+  else stage_pack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf);
 }
 
 template <bool UNPACK, int G, int VW>
@@ -159,7 +159,8 @@ __global__ void __launch_bounds__(256) k_word(const KP P) {
   extern __shared__ int32_t wt[];
   for (int i = threadIdx.x; i < P.nwords; i += blockDim.x) wt[i] = P.wtab[i];
   __syncthreads();
-  word_range<UNPACK, G, VW, LD_CS, (G >= 4 ? 4 : 2)>(P, wt, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+  word_range<UNPACK, G, VW, LD_CS, (G >= 4 ? 4 : 2)>(P, P.c - P.pos, P.pos, P.pos + P.len, wt,
+                                                     (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                                                      (int64_t)gridDim.x * blockDim.x);
 }
 // --------------------------------------------------------------- host side

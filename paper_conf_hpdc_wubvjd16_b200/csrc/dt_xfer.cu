@@ -111,48 +111,47 @@ __device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeo
 }
 
 // pack or unpack stream bytes [lo, lo+len) of the current chunk with this CTA.
+// cb: the slot base such that stream byte x of the message lives at cb + x.  The
+// op's parameters stay in the grid-constant bank (no per-fragment struct copy).
 template <bool UNPACK>
-__device__ __forceinline__ void cta_chunk(const XOp& X, KP P, uint8_t* slot, int64_t lo, int64_t len,
-                                          const int32_t* wt, uint8_t* sbuf, uint64_t* mbar) {
-  P.c = slot + lo;  // slot maps stream byte 0 of the message (see caller)
-  P.pos = lo;
-  P.len = len;
+__device__ __forceinline__ void cta_chunk(const XOp& X, uint8_t* cb, int64_t lo, int64_t len, const int32_t* wt,
+                                          uint8_t* sbuf, uint64_t* mbar) {
+  const KP& P = X.P;
+  const int64_t hi = lo + len;
   constexpr int POL = UNPACK ? LD_CG : LD_CS;  // ring slots are rewritten by the peer: bypass L1
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
     switch (X.g) {
       case 8:
-        if (UNPACK) stage_unpack<8, kXferStageBufs>(P, wt, lo, lo + len, sbuf, mbar);
-        else stage_pack<8, kXferStageBufs>(P, wt, lo, lo + len, sbuf);
+        if (UNPACK) stage_unpack<8, kXferStageBufs>(P, cb, wt, lo, hi, sbuf, mbar);
+        else stage_pack<8, kXferStageBufs>(P, cb, wt, lo, hi, sbuf);
         break;
       default:
-        if (UNPACK) stage_unpack<16, kXferStageBufs>(P, wt, lo, lo + len, sbuf, mbar);
-        else stage_pack<16, kXferStageBufs>(P, wt, lo, lo + len, sbuf);
+        if (UNPACK) stage_unpack<16, kXferStageBufs>(P, cb, wt, lo, hi, sbuf, mbar);
+        else stage_pack<16, kXferStageBufs>(P, cb, wt, lo, hi, sbuf);
         break;
     }
     return;
   }
   if (X.kind == 2) {
     const int64_t body = len - len % X.g;
-    KP Q = P;
-    Q.len = body;
     // few CTAs carry the whole transfer: keep 4 vectors per thread in flight (512 threads: 32 KiB/CTA)
     switch (X.g) {
-      case 1: word_range<UNPACK, 1, 16, POL, 2>(Q, wt, threadIdx.x, blockDim.x); break;
-      case 2: word_range<UNPACK, 2, 16, POL, 2>(Q, wt, threadIdx.x, blockDim.x); break;
-      case 4: word_range<UNPACK, 4, 16, POL, 4>(Q, wt, threadIdx.x, blockDim.x); break;
-      case 8: word_range<UNPACK, 8, 16, POL, 4>(Q, wt, threadIdx.x, blockDim.x); break;
-      default: word_range<UNPACK, 16, 16, POL, 4>(Q, wt, threadIdx.x, blockDim.x); break;
+      case 1: word_range<UNPACK, 1, 16, POL, 2>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
+      case 2: word_range<UNPACK, 2, 16, POL, 2>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
+      case 4: word_range<UNPACK, 4, 16, POL, 4>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
+      case 8: word_range<UNPACK, 8, 16, POL, 4>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
+      default: word_range<UNPACK, 16, 16, POL, 4>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
     }
     if (body < len && threadIdx.x < 32)  // ragged tail (< G bytes): one warp walks it
-      seg_range<UNPACK, false, POL>(P, lo + body, lo + len, threadIdx.x & 31);
+      seg_range<UNPACK, false, POL>(P, cb, lo + body, hi, threadIdx.x & 31);
     return;
   }
   const int nw = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   int64_t per = (len + nw - 1) / nw;
   per = (per + 127) & ~int64_t(127);
-  const int64_t a = lo + (int64_t)w * per, b = min(a + per, lo + len);
-  if (X.single) seg_range<UNPACK, true, POL>(P, a, b, lane);
-  else seg_range<UNPACK, false, POL>(P, a, b, lane);
+  const int64_t a = lo + (int64_t)w * per, b = min(a + per, hi);
+  if (X.single) seg_range<UNPACK, true, POL>(P, cb, a, b, lane);
+  else seg_range<UNPACK, false, POL>(P, cb, a, b, lane);
 }
 
 constexpr int kXferThreads = 512;
@@ -254,8 +253,8 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       }
       __syncthreads();
       if (s_stop) return;
-      if (X.role == 0) cta_chunk<false>(X, X.P, sl, off, len, wt, sbuf, mbar);
-      else cta_chunk<true>(X, X.P, sl, off, len, wt, sbuf, mbar);
+      if (X.role == 0) cta_chunk<false>(X, sl, off, len, wt, sbuf, mbar);
+      else cta_chunk<true>(X, sl, off, len, wt, sbuf, mbar);
       __syncthreads();
       if (threadIdx.x == 0) {
         if (!(A.flags & 1)) __threadfence_system();
