@@ -521,30 +521,34 @@ __device__ __forceinline__ void stage_pack(const KP& P, uint8_t* cb, const int32
   const int64_t ntiles = (hi - lo + T - 1) / T;
   const int64_t S = (int64_t)nthr * G;  // a thread's stride through the stream: Se elements + Sq bytes
   const int64_t Se = (int64_t)fdiv((uint64_t)S, P.ftsize), Sq = S - Se * P.tsize;
+  // Persistent per-thread word iterator: thread tid handles words tid, tid+nthr, ...
+  // of the whole range (T/G is a multiple of nthr, so this is also its share of
+  // every tile) -- one division and element decomposition per CALL, not per tile.
+  const int64_t nwords = (hi - lo) / G;
+  int64_t q = 0, ed = 0;
+  ElemIt ei;
+  if (tid < nwords) {
+    const int64_t x0 = lo + (int64_t)tid * G;
+    const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
+    q = x0 - (int64_t)e0 * P.tsize;
+    ei.init(P, e0);
+    ed = ei.disp(P);
+  }
+  int64_t iw = tid;  // next word of this thread (index from lo)
   for (int64_t t = 0; t < ntiles + L - 1; t++) {
     if (t < ntiles) {
-      uint8_t* buf = sbuf + (t % NB) * T;
+      uint8_t* buf = sbuf + (t % NB) * T - (t * T);  // word iw lands at buf + iw*G
       if (tid == 0) bulk_wait_read<1>();  // the store that last read this buffer (tile t-NB) is done reading
       __syncthreads();
-      const int64_t s0 = lo + t * T;
-      const int64_t nw = (hi - s0 < T ? hi - s0 : (int64_t)T) / G;
-      int64_t i = tid;
-      if (i < nw) {
-        const int64_t x0 = s0 + i * G;
-        const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
-        int64_t q = x0 - (int64_t)e0 * P.tsize;
-        ElemIt ei;
-        ei.init(P, e0);
-        int64_t ed = ei.disp(P);
-        while (true) {
-          cp_async<G>(buf + i * G, P.nc + ed + wt[q / G]);
-          i += nthr;
-          if (i >= nw) break;
-          q += Sq;
-          int64_t k = Se;
-          if (q >= P.tsize) { q -= P.tsize; k++; }
-          if (k) { ei.advance(P, k); ed = ei.disp(P); }
-        }
+      const int64_t wend = (t + 1) * (T / G) < nwords ? (t + 1) * (T / G) : nwords;
+      while (iw < wend) {
+        cp_async<G>(buf + iw * G, P.nc + ed + wt[q / G]);
+        iw += nthr;
+        if (iw >= nwords) break;
+        q += Sq;
+        int64_t k = Se;
+        if (q >= P.tsize) { q -= P.tsize; k++; }
+        if (k) { ei.advance(P, k); ed = ei.disp(P); }
       }
     }
     cp_async_commit();  // (an empty group in the drain iterations keeps the group count uniform)
@@ -593,31 +597,33 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const uint8_t* cb, con
   };
   if (tid == 0)
     for (int64_t t = 0; t < NB && t < ntiles; t++) issue(t);
+  // persistent per-thread word iterator (see stage_pack)
+  const int64_t nwords = (hi - lo) / G;
+  const int64_t fullw = ((hi - lo) & ~int64_t(15)) / G;  // words delivered through shared memory
+  int64_t q = 0, ed = 0;
+  ElemIt ei;
+  if (tid < nwords) {
+    const int64_t x0 = lo + (int64_t)tid * G;
+    const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
+    q = x0 - (int64_t)e0 * P.tsize;
+    ei.init(P, e0);
+    ed = ei.disp(P);
+  }
+  int64_t iw = tid;
   for (int64_t t = 0; t < ntiles; t++) {
-    const uint8_t* buf = sbuf + (t % NB) * T;
+    const uint8_t* buf = sbuf + (t % NB) * T - t * T;  // word iw of the range at buf + iw*G
     mbar_wait(mbar + (t % NB), (uint32_t)((t / NB) & 1));
-    const int64_t s0 = lo + t * T;
-    const int64_t tl = hi - s0 < T ? hi - s0 : (int64_t)T;
-    const int64_t nw = tl / G, full = (tl & ~int64_t(15)) / G;
-    int64_t i = tid;
-    if (i < nw) {
-      const int64_t x0 = s0 + i * G;
-      const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
-      int64_t q = x0 - (int64_t)e0 * P.tsize;
-      ElemIt ei;
-      ei.init(P, e0);
-      int64_t ed = ei.disp(P);
-      while (true) {
-        const W v = i < full ? *reinterpret_cast<const W*>(buf + i * G)
-                             : *reinterpret_cast<const W*>(cb + s0 + i * G);  // ragged tail
-        *reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed + wt[q / G]) = v;
-        i += nthr;
-        if (i >= nw) break;
-        q += Sq;
-        int64_t k = Se;
-        if (q >= P.tsize) { q -= P.tsize; k++; }
-        if (k) { ei.advance(P, k); ed = ei.disp(P); }
-      }
+    const int64_t wend = (t + 1) * (T / G) < nwords ? (t + 1) * (T / G) : nwords;
+    while (iw < wend) {
+      const W v = iw < fullw ? *reinterpret_cast<const W*>(buf + iw * G)
+                             : *reinterpret_cast<const W*>(cb + lo + iw * G);  // ragged tail (< 16 B)
+      *reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed + wt[q / G]) = v;
+      iw += nthr;
+      if (iw >= nwords) break;
+      q += Sq;
+      int64_t k = Se;
+      if (q >= P.tsize) { q -= P.tsize; k++; }
+      if (k) { ei.advance(P, k); ed = ei.disp(P); }
     }
     __syncthreads();  // buffer consumed
     if (tid == 0 && t + NB < ntiles) issue(t + NB);

@@ -120,15 +120,20 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, uint8_t* cb, int64_t lo,
   const int64_t hi = lo + len;
   constexpr int POL = UNPACK ? LD_CG : LD_CS;  // ring slots are rewritten by the peer: bypass L1
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
+    const int64_t bh = hi - len % X.g;  // words; a ragged tail (< G bytes, last fragment) is walked below
     switch (X.g) {
       case 8:
-        if (UNPACK) stage_unpack<8, kXferStageBufs>(P, cb, wt, lo, hi, sbuf, mbar);
-        else stage_pack<8, kXferStageBufs>(P, cb, wt, lo, hi, sbuf);
+        if (UNPACK) stage_unpack<8, kXferStageBufs>(P, cb, wt, lo, bh, sbuf, mbar);
+        else stage_pack<8, kXferStageBufs>(P, cb, wt, lo, bh, sbuf);
         break;
       default:
-        if (UNPACK) stage_unpack<16, kXferStageBufs>(P, cb, wt, lo, hi, sbuf, mbar);
-        else stage_pack<16, kXferStageBufs>(P, cb, wt, lo, hi, sbuf);
+        if (UNPACK) stage_unpack<16, kXferStageBufs>(P, cb, wt, lo, bh, sbuf, mbar);
+        else stage_pack<16, kXferStageBufs>(P, cb, wt, lo, bh, sbuf);
         break;
+    }
+    if (bh < hi) {
+      __syncthreads();
+      if (threadIdx.x < 32) seg_range<UNPACK, false, POL>(P, cb, bh, hi, threadIdx.x & 31);
     }
     return;
   }

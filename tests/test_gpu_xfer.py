@@ -67,6 +67,9 @@ def test_loopback_different_types(torch_cuda):
     tri, _, tpar = c2_lower_triangle(600)
     n = 600 * 601 // 2
     _loop_check(torch_cuda, comm, tri, 0, tpar, ("contiguous", n + 100, ("basic", "DOUBLE")), 0, (n + 100) * 8)
+    # message not a multiple of the receive layout's word size (ragged tail inside a staged fragment)
+    _loop_check(torch_cuda, comm, ("contiguous", 125, ("basic", "DOUBLE")), 0, 1000,
+                ("vector", 100, 2, 4, ("basic", "DOUBLE")), 0, 3200)
     # matrix transpose: column-major -> row-major as a vector of blocklength-1 columns ([L26:c4896 §5.2.3])
     m = 96
     rows = ("hvector", m, 1, 8, ("vector", m, 1, m, ("basic", "DOUBLE")))
