@@ -624,8 +624,15 @@ static int check_nonoverlap(dt_type_s* t, const Form& f, int64_t count) {
     if (!proven || cnt <= 1) return;
     const int64_t span = hi - lo;
     if (tab) {
-      std::vector<int64_t> s(*tab);
-      std::sort(s.begin(), s.end());
+      // index lists are usually sorted (LAMMPS-style): check in place, sort a copy otherwise
+      std::vector<int64_t> copy;
+      const std::vector<int64_t>* sp = tab;
+      if (!std::is_sorted(tab->begin(), tab->end())) {
+        copy = *tab;
+        std::sort(copy.begin(), copy.end());
+        sp = &copy;
+      }
+      const std::vector<int64_t>& s = *sp;
       for (size_t i = 1; i < s.size(); i++)
         if (s[i] - s[i - 1] < span) { proven = false; return; }
       lo += s.front();

@@ -54,7 +54,11 @@ def main():
             mk[name] = (lambda nb=nb, bs=bs: (("vector", nb, bs // 8, 2 * bs // 8, ("basic", "DOUBLE")), 0,
                                               2 * bs * nb))
         rec, org, parent = mk[name]()
-        t = dt.from_recipe(rec).commit()
+        t = dt.from_recipe(rec)
+        import time as _time
+        c0 = _time.perf_counter()
+        t.commit()  # f2: first-use cost (host flatten + upload + device scan), cached afterwards
+        commit_ms = (_time.perf_counter() - c0) * 1e3
         n = t.size
         src = torch.empty(parent, dtype=torch.uint8, device=dev)
         src.random_(0, 256)
@@ -84,7 +88,8 @@ def main():
         row = {"config": name, "bytes": n, "kernel": kind, "gran": g, "pack_us": round(tp * 1e3, 2),
                "unpack_us": round(tu * 1e3, 2), "copy_us": round(tc * 1e3, 2), "pack_gbs": gb(tp),
                "unpack_gbs": gb(tu), "copy_gbs": gb(tc),
-               "pack_vs_copy": round(tc / tp, 3), "unpack_vs_copy": round(tc / tu, 3)}
+               "pack_vs_copy": round(tc / tp, 3), "unpack_vs_copy": round(tc / tu, 3),
+               "commit_ms": round(commit_ms, 3)}
         if rec[0] == "vector" and rec[4][0] == "basic":
             # f4 diagnostic (Fig. 8, [L24:c4075 §5.1]): cudaMemcpy2D of the same vector, device to device
             from cuda.bindings import runtime as cudart
