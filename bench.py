@@ -315,7 +315,7 @@ def run_xfer(args):
             else:
                 nid = dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None
                 comm = dt.Comm(0, 1, local, chunk_bytes=chunk, depth=depth, mode=mode, nccl_id=nid,
-                               ctas=args.xfer_ctas)
+                               ctas=args.xfer_ctas, ring_loopback=True)  # measure the pipeline itself
             for _ in range(args.warmup):
                 comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
             torch.cuda.synchronize()
@@ -340,6 +340,17 @@ def run_xfer(args):
             comm.free()
     best = max(results, key=lambda r: r["gbs_per_rank"])
     value = ws * payload / (best["ms"] * 1e-3) / 1e9
+    fused = None
+    if ws == 1:  # f1: the same loopback exchange as one fused datatype -> datatype copy (no ring)
+        for _ in range(args.warmup):
+            dt.copy(t, 1, A, t, 1, B, src_offset=org, dst_offset=org)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(10):
+            dt.copy(t, 1, A, t, 1, B, src_offset=org, dst_offset=org)
+        e1.record(s)
+        torch.cuda.synchronize()
+        fused = round(payload / (e0.elapsed_time(e1) / 10 * 1e-3) / 1e9, 1)
     # parity of the last exchange: my B must equal the peer's A packed/unpacked (closed form: same layout)
     exp = torch.from_numpy(fill_bytes(parent, seed_for(3) + peer)).to(dev)
     ok = bool(torch.equal(B.view(-1)[org:org + 8 * 64], exp.view(-1)[org:org + 8 * 64]))
@@ -350,6 +361,7 @@ def run_xfer(args):
             "config": {"workload": "C3: ScaLAPACK 2D block-cyclic submatrix (N=8192 f64, nb=64, owner (0,1)), "
                                    f"pairwise exchange, mode={args.xfer_mode}",
                        "payload_bytes": payload, "sweep": results, "spot_parity": ok,
+                       "fused_loopback_gbs_per_rank": fused,
                        "pairs": "loopback (1 GPU)" if ws == 1 else "(r, r^1)"},
             "roofline": {"bound": "nvlink" if ws > 1 else "hbm", "achieved": best["gbs_per_rank"],
                          "peak": peak, "unit": "GB/s", "frac": round(best["gbs_per_rank"] / peak, 4),

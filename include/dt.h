@@ -122,6 +122,17 @@ dt_status dt_pack_host(dt_t t, int64_t count, const void* origin, void* packed, 
 dt_status dt_unpack_host(dt_t t, int64_t count, const void* packed, void* origin, int64_t pos, int64_t* len,
                          void* stream);
 
+/* Fused datatype -> datatype copy on the current device:
+ * dst' = unpack(rtype, rcount, pack(stype, scount, src)) over the first
+ * scount*size(stype) bytes, without a packed intermediate: every stream byte
+ * goes from its source-layout address (src, D) straight to its
+ * destination-layout address (dst, D).  Signatures may differ (reading A12;
+ * vector <-> contiguous, matrix transpose: [L26:c4303 §5.2.2], [L26:c4896
+ * §5.2.3]); a larger receive fills a prefix.  Errors: DT_ERR_TRUNCATE if the
+ * bytes do not fit, DT_ERR_OVERLAP for an overlapping destination typemap,
+ * DT_ERR_NOT_COMMITTED, DT_ERR_ARG.  Asynchronous on `stream`. */
+dt_status dt_copy(dt_t stype, int64_t scount, const void* src, dt_t rtype, int64_t rcount, void* dst, void* stream);
+
 /* ------------------------------------------------------------------ introspection (host only, no GPU) */
 typedef struct {
   int64_t size, lb, extent, true_lb, true_extent;
@@ -151,7 +162,8 @@ typedef struct {
   int32_t mode;        /* DT_XFER_P2P (pack straight into the peer's ring over NVLink) or
                           DT_XFER_NCCL (double-buffered ncclSend/ncclRecv of packed chunks) */
   int32_t ctas;        /* CTAs per direction for the P2P pipeline kernel; 0 = default      */
-  int32_t reserved;
+  int32_t flags;       /* bit 0: loopback (dest = source = self) through the ring pipeline
+                          instead of the fused datatype -> datatype copy (dt_copy)        */
 } dt_xfer_opts;
 
 /* Create this rank's endpoint on `device`: allocates the receive rings

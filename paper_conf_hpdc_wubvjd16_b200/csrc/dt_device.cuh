@@ -302,6 +302,57 @@ __device__ __forceinline__ void seg_range(const KP& P, uint8_t* cb, int64_t p, c
   seg_walk<UNPACK, SINGLE, POL>(P, cb, p, p1, b, r, e, elem_disp(P, e), lane);
 }
 
+// ---------------------------------------------------------------- fused type -> type
+// f1: stream bytes [p, p1) go from the source layout S straight to
+// the destination layout R, no packed buffer.  Both sides keep a block cursor;
+// each step copies min(rest of S's block, rest of R's block) with the relative
+// alignment machinery of warp_copy.
+struct Cursor {
+  uint64_t e;
+  int64_t b, r, ed, blen, bd;
+};
+__device__ __forceinline__ void cursor_init(const KP& P, Cursor& c, int64_t p, int lane) {
+  c.e = fdiv((uint64_t)p, P.ftsize);
+  c.r = p - (int64_t)c.e * P.tsize;
+  c.b = 0;
+  if (P.nblocks > 1) {
+    c.b = warp_find_block(P.boff, P.nblocks, c.r, lane);
+    c.r -= __ldg(P.boff + c.b);
+  }
+  c.ed = elem_disp(P, c.e);
+  c.blen = P.nblocks == 1 ? P.bl0 : __ldg(P.bl + c.b);
+  c.bd = P.nblocks == 1 ? P.bd0 : __ldg(P.bd + c.b);
+}
+__device__ __forceinline__ void cursor_advance(const KP& P, Cursor& c, int64_t n) {
+  c.r += n;
+  if (c.r < c.blen) return;
+  c.r = 0;
+  if (P.nblocks == 1 || ++c.b == P.nblocks) {
+    c.b = 0;
+    ++c.e;
+    c.ed = elem_disp(P, c.e);
+  }
+  c.blen = P.nblocks == 1 ? P.bl0 : __ldg(P.bl + c.b);
+  c.bd = P.nblocks == 1 ? P.bd0 : __ldg(P.bd + c.b);
+}
+__device__ __forceinline__ void dual_walk(const KP& S, const KP& R, int64_t p, const int64_t p1, int lane) {
+  if (p >= p1) return;
+  Cursor cs, cr;
+  cursor_init(S, cs, p, lane);
+  cursor_init(R, cr, p, lane);
+  while (p < p1) {
+    int64_t seg = min(cs.blen - cs.r, cr.blen - cr.r);
+    seg = min(seg, p1 - p);
+    const uint8_t* src = S.nc + cs.ed + cs.bd + cs.r;
+    uint8_t* dst = const_cast<uint8_t*>(R.nc) + cr.ed + cr.bd + cr.r;
+    warp_copy<LD_CS>(dst, src, seg, lane);
+    p += seg;
+    if (p >= p1) break;
+    cursor_advance(S, cs, seg);
+    cursor_advance(R, cr, seg);
+  }
+}
+
 // ---------------------------------------------------------------- launch plans
 // Cost-balanced warp slices (long-run kernel).  A warp's time is its bytes plus a
 // fixed cost per segment (descriptor fetch + one memory round trip), so slices
@@ -627,6 +678,54 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const uint8_t* cb, con
     }
     __syncthreads();  // buffer consumed
     if (tid == 0 && t + NB < ntiles) issue(t + NB);
+  }
+}
+
+// Fused type -> type copy of G-granular templates: thread tid moves words tid,
+// tid+nthr, ... of [lo, hi): source address from S's word table + element
+// iterator, destination from R's; NV words in flight per thread.
+template <int G, int NV>
+__device__ __forceinline__ void dual_words(const KP& S, const int32_t* wts, const KP& R, const int32_t* wtr,
+                                           int64_t lo, int64_t hi, int64_t tid, int64_t nthr) {
+  typedef typename WordT<G>::T W;
+  const int64_t nwords = (hi - lo) / G;
+  if (tid >= nwords) return;
+  const int64_t St = nthr * G;
+  const int64_t Ses = (int64_t)fdiv((uint64_t)St, S.ftsize), Sqs = St - Ses * S.tsize;
+  const int64_t Ser = (int64_t)fdiv((uint64_t)St, R.ftsize), Sqr = St - Ser * R.tsize;
+  const int64_t x0 = lo + tid * G;
+  uint64_t e = fdiv((uint64_t)x0, S.ftsize);
+  int64_t qs = x0 - (int64_t)e * S.tsize;
+  ElemIt is;
+  is.init(S, e);
+  int64_t eds = is.disp(S);
+  e = fdiv((uint64_t)x0, R.ftsize);
+  int64_t qr = x0 - (int64_t)e * R.tsize;
+  ElemIt ir;
+  ir.init(R, e);
+  int64_t edr = ir.disp(R);
+  for (int64_t w = tid; w < nwords; w += nthr * NV) {
+    W v[NV];
+    W* d[NV];
+#pragma unroll
+    for (int j = 0; j < NV; j++) {
+      if (w + j * nthr < nwords) {
+        v[j] = ldv<LD_CS>(reinterpret_cast<const W*>(S.nc + eds + wts[qs / G]));
+        d[j] = reinterpret_cast<W*>(const_cast<uint8_t*>(R.nc) + edr + wtr[qr / G]);
+        if (w + (j + 1) * nthr >= nwords) continue;  // never step an iterator past the stream
+        qs += Sqs;
+        int64_t k = Ses;
+        if (qs >= S.tsize) { qs -= S.tsize; k++; }
+        if (k) { is.advance(S, k); eds = is.disp(S); }
+        qr += Sqr;
+        k = Ser;
+        if (qr >= R.tsize) { qr -= R.tsize; k++; }
+        if (k) { ir.advance(R, k); edr = ir.disp(R); }
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < NV; j++)
+      if (w + j * nthr < nwords) *d[j] = v[j];
   }
 }
 

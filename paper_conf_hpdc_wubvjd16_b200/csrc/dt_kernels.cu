@@ -154,6 +154,25 @@ __global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
   else stage_pack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf);
 }
 
+// f1: fused type -> type copies (no packed buffer)
+__global__ void __launch_bounds__(256, 3) k_dual_seg(const KP S, const KP R, int64_t n, int64_t per_warp) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t p = gw * per_warp;
+  dual_walk(S, R, p, min(p + per_warp, n), lane);
+}
+
+template <int G>
+__global__ void __launch_bounds__(256) k_dual_word(const KP S, const KP R, int64_t n) {
+  extern __shared__ int32_t wts[];
+  int32_t* wtr = wts + S.nwords;
+  for (int i = threadIdx.x; i < S.nwords; i += blockDim.x) wts[i] = S.wtab[i];
+  for (int i = threadIdx.x; i < R.nwords; i += blockDim.x) wtr[i] = R.wtab[i];
+  __syncthreads();
+  dual_words<G, 4>(S, wts, R, wtr, 0, n, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                   (int64_t)gridDim.x * blockDim.x);
+}
+
 template <bool UNPACK, int G, int VW>
 __global__ void __launch_bounds__(256) k_word(const KP P) {
   extern __shared__ int32_t wt[];
@@ -756,6 +775,135 @@ dt_status dt_pack(dt_t t, int64_t count, const void* origin, void* packed, int64
 dt_status dt_unpack(dt_t t, int64_t count, const void* packed, void* origin, int64_t pos, int64_t* len,
                     void* stream) {
   return pack_common(true, t, count, origin, const_cast<void*>(packed), pos, len, stream);
+}
+
+// f1: fused datatype -> datatype copy on the current device (no packed buffer).
+static dt_status make_kp(dt_type_s* t, int64_t count, const void* nc, int64_t n, KP& P, const Form** fo,
+                         DeviceDesc** ddo) {
+  DeviceDesc* dd = nullptr;
+  dt_status st = ensure_committed_on_device(t, &dd);
+  if (st != DT_OK) return st;
+  const Form& f = get_form(t);
+  KLevels L;
+  build_levels(f, dd, t, count, L);
+  std::memset(&P, 0, sizeof(P));
+  P.nc = (const uint8_t*)nc;
+  P.pos = 0;
+  P.len = n;
+  P.tsize = f.tsize();
+  P.nblocks = (int64_t)f.bl.size();
+  P.bd = dd->bd;
+  P.bl = dd->bl;
+  P.boff = dd->boff;
+  P.bd0 = f.bd[0];
+  P.bl0 = f.bl[0];
+  P.nlev = L.n;
+  for (int i = 0; i < L.n; i++) {
+    P.cnt[i] = L.cnt[i];
+    P.stride[i] = L.stride[i];
+    P.table[i] = L.table[i];
+    P.fcnt[i] = make_fd((uint64_t)L.cnt[i]);
+  }
+  P.ftsize = make_fd((uint64_t)P.tsize);
+  *fo = &f;
+  *ddo = dd;
+  return DT_OK;
+}
+
+static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, int64_t rcount, void* dst,
+                            void* stream) {
+  if (!st || !rt || scount < 0 || rcount < 0) {
+    set_error("dt_copy: bad argument");
+    return DT_ERR_ARG;
+  }
+  if (!st->committed || !rt->committed) {
+    set_error("dt_copy: type not committed");
+    return DT_ERR_NOT_COMMITTED;
+  }
+  const int64_t n = scount * st->size;
+  if (n > rcount * rt->size) {
+    set_error("dt_copy: %lld bytes do not fit a %lld-byte receive layout", (long long)n,
+              (long long)(rcount * rt->size));
+    return DT_ERR_TRUNCATE;
+  }
+  if (n == 0) return DT_OK;
+  if (!src || !dst) {
+    set_error("dt_copy: NULL buffer");
+    return DT_ERR_ARG;
+  }
+  if (g_check_ptrs) {
+    dt_status s1 = check_dev_ptr((const uint8_t*)src + st->true_lb, "source");
+    if (s1 != DT_OK) return s1;
+    s1 = check_dev_ptr((const uint8_t*)dst + rt->true_lb, "destination");
+    if (s1 != DT_OK) return s1;
+  }
+  KP S, R;
+  const Form *fs, *fr;
+  DeviceDesc *ds, *dr;
+  dt_status s1 = make_kp(st, scount, src, n, S, &fs, &ds);
+  if (s1 != DT_OK) return s1;
+  s1 = make_kp(rt, rcount, dst, n, R, &fr, &dr);
+  if (s1 != DT_OK) return s1;
+  {
+    std::lock_guard<std::mutex> g(rt->mu);
+    if (rt->ovl_count != rcount) {
+      rt->ovl_result = check_nonoverlap(rt, *fr, rcount);
+      rt->ovl_count = rcount;
+    }
+    if (rt->ovl_result != 1) {
+      set_error("dt_copy: destination typemap entries overlap");
+      return DT_ERR_OVERLAP;
+    }
+  }
+  cudaStream_t s = (cudaStream_t)stream;
+  KLevels Ls, Lr;
+  build_levels(*fs, ds, st, scount, Ls);
+  build_levels(*fr, dr, rt, rcount, Lr);
+  int64_t gs = 1, gr = 1;
+  plan_kernel(*fs, Ls, (uint64_t)(uintptr_t)src, 0, 0, n, &gs);
+  plan_kernel(*fr, Lr, (uint64_t)(uintptr_t)dst, 0, 0, n, &gr);
+  const int64_t g = std::min(gs, gr);
+  const double ms = (double)S.tsize / (double)S.nblocks, mr = (double)R.tsize / (double)R.nblocks;
+  const bool words_ok = S.tsize % g == 0 && R.tsize % g == 0 && (S.tsize + R.tsize) / g <= kMaxWordTable &&
+                        template_fits_int32(*fs) && template_fits_int32(*fr);
+  const char* fk = getenv("DT_FORCE_KERNEL");
+  const int force = fk ? atoi(fk) : 0;
+  const bool use_words = words_ok && force != 1 && (force == 2 || std::min(ms, mr) < 256.0);
+  const int sms = num_sms();
+  if (use_words) {
+    const int32_t *wa = nullptr, *wb = nullptr;
+    s1 = ensure_wtab(*fs, *ds, g, &wa);
+    if (s1 != DT_OK) return s1;
+    s1 = ensure_wtab(*fr, *dr, g, &wb);
+    if (s1 != DT_OK) return s1;
+    S.wtab = wa;
+    S.nwords = (int32_t)(S.tsize / g);
+    R.wtab = wb;
+    R.nwords = (int32_t)(R.tsize / g);
+    const size_t smem = sizeof(int32_t) * (size_t)(S.nwords + R.nwords);
+    const int64_t nwords = n / g;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * 6, (nwords + 1023) / 1024));
+    switch (g) {
+      case 1: k_dual_word<1><<<grid, 256, smem, s>>>(S, R, n); break;
+      case 2: k_dual_word<2><<<grid, 256, smem, s>>>(S, R, n); break;
+      case 4: k_dual_word<4><<<grid, 256, smem, s>>>(S, R, n); break;
+      case 8: k_dual_word<8><<<grid, 256, smem, s>>>(S, R, n); break;
+      default: k_dual_word<16><<<grid, 256, smem, s>>>(S, R, n); break;
+    }
+  } else {
+    const int64_t nw = std::min<int64_t>((int64_t)sms * 3 * 8, std::max<int64_t>(1, (n + 4095) / 4096));
+    int64_t per = (n + nw - 1) / nw;
+    per = (per + 511) & ~int64_t(511);
+    const int64_t nwr = (n + per - 1) / per;
+    k_dual_seg<<<(unsigned)((nwr + 7) / 8), 256, 0, s>>>(S, R, n, per);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "dt_copy launch");
+  return DT_OK;
+}
+
+dt_status dt_copy(dt_t st, int64_t scount, const void* src, dt_t rt, int64_t rcount, void* dst, void* stream) {
+  return copy_typed(st, scount, src, rt, rcount, dst, stream);
 }
 
 dt_status dt_plan(dt_t t, int64_t count, uint64_t origin_addr, uint64_t packed_addr, int64_t pos, int64_t len,

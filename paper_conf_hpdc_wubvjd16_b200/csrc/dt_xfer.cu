@@ -418,7 +418,7 @@ static void fill_opts(dt_xfer_opts& o, const dt_xfer_opts* in) {
   o.depth = 4;
   o.mode = DT_XFER_P2P;
   o.ctas = 0;
-  o.reserved = 0;
+  o.flags = in ? in->flags : 0;
   if (in) {
     if (in->chunk_bytes > 0) o.chunk_bytes = in->chunk_bytes;
     if (in->depth > 0) o.depth = in->depth;
@@ -885,9 +885,28 @@ static dt_status validate(dt_comm_s* c, const PendingOp& p) {
   return DT_OK;
 }
 
-static dt_status issue(dt_comm_s* c, const std::vector<PendingOp>& ops, void* stream) {
+// Loopback (dest = source = this rank, the paper's "1GPU" case [L26:c1686]) in
+// P2P mode goes through the fused datatype -> datatype copy (f1): no ring, no
+// flags, each byte moves once.  The k-th send-to-self of a call/group matches the
+// k-th receive-from-self.  opts.flags bit 0 keeps loopback on the ring pipeline.
+static dt_status issue(dt_comm_s* c, const std::vector<PendingOp>& ops_in, void* stream) {
   cudaStream_t s = (cudaStream_t)stream;
-  if (c->o.mode == DT_XFER_NCCL) return issue_nccl(c, ops, s);
+  if (c->o.mode == DT_XFER_NCCL) return issue_nccl(c, ops_in, s);
+  if (c->o.flags & 1) return issue_p2p(c, ops_in, s);
+  std::vector<PendingOp> ops = ops_in;
+  std::vector<size_t> sends, recvs;
+  for (size_t i = 0; i < ops.size(); i++) {
+    if (ops[i].dest == c->rank) sends.push_back(i);
+    if (ops[i].source == c->rank) recvs.push_back(i);
+  }
+  for (size_t k = 0; k < std::min(sends.size(), recvs.size()); k++) {
+    PendingOp& a = ops[sends[k]];
+    PendingOp& b = ops[recvs[k]];
+    dt_status st = dt_copy(a.stype, a.scount, a.sbuf, b.rtype, b.rcount, b.rbuf, stream);
+    if (st != DT_OK) return st;
+    a.dest = -1;
+    b.source = -1;
+  }
   return issue_p2p(c, ops, s);
 }
 

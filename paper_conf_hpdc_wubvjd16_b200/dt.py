@@ -38,7 +38,7 @@ class FormInfo(C.Structure):
 
 class XferOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("depth", C.c_int32), ("mode", C.c_int32), ("ctas", C.c_int32),
-                ("reserved", C.c_int32)]
+                ("flags", C.c_int32)]
 
 
 P = C.c_void_p
@@ -64,6 +64,7 @@ _SIGS = {
     "dt_pack": (C.c_int, [P, I64, P, P, I64, PI64, P]),
     "dt_unpack": (C.c_int, [P, I64, P, P, I64, PI64, P]),
     "dt_pack_host": (C.c_int, [P, I64, P, P, I64, PI64, P]),
+    "dt_copy": (C.c_int, [P, I64, P, P, I64, P, P]),
     "dt_unpack_host": (C.c_int, [P, I64, P, P, I64, PI64, P]),
     "dt_get_form": (C.c_int, [P, C.POINTER(FormInfo)]),
     "dt_flatten": (C.c_int, [P, I64, PI64, PI64, I64, PI64]),
@@ -336,8 +337,9 @@ class Comm:
     """dt_comm_t: this rank's endpoint (receive rings + flags, or a NCCL communicator)."""
 
     def __init__(self, rank: int, nranks: int, device: int, chunk_bytes: int = 1 << 20, depth: int = 4,
-                 mode: int = XFER_P2P, ctas: int = 0, nccl_id: bytes | None = None):
-        self.opts = XferOpts(chunk_bytes, depth, mode, ctas, 0)
+                 mode: int = XFER_P2P, ctas: int = 0, nccl_id: bytes | None = None, ring_loopback: bool = False):
+        # ring_loopback: send-to-self goes through the ring pipeline instead of the fused dt_copy
+        self.opts = XferOpts(chunk_bytes, depth, mode, ctas, 1 if ring_loopback else 0)
         self.h = P()
         self.rank, self.nranks = rank, nranks
         idbuf = C.create_string_buffer(nccl_id, 128) if nccl_id else None
@@ -404,3 +406,10 @@ class Comm:
                 _lib.dt_comm_free(C.byref(self.h))
         except Exception:
             pass
+
+
+def copy(stype: Type, scount: int, src, rtype: Type, rcount: int, dst, stream=None, src_offset: int = 0,
+         dst_offset: int = 0) -> None:
+    """dt_copy: fused datatype -> datatype copy on one GPU (no packed buffer)."""
+    _check(lib().dt_copy(stype.h, scount, _ptr(src) + src_offset, rtype.h, rcount, _ptr(dst) + dst_offset,
+                         _stream(stream)))

@@ -44,9 +44,10 @@ def _loop_check(torch, comm, srec, sorg, sparent, rrec, rorg, rparent, scount=1,
 
 
 @pytest.mark.parametrize("chunk,depth", [(64 << 10, 2), (256 << 10, 4), (1 << 20, 2), (4 << 20, 4)])
-def test_loopback_block_cyclic(torch_cuda, chunk, depth):
+@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+def test_loopback_block_cyclic(torch_cuda, chunk, depth, ring):
     from paper_conf_hpdc_wubvjd16_b200 import dt
-    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth)
+    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth, ring_loopback=ring)
     rec, org, parent = c3_block_cyclic(2048, 64)
     _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
     # repeated messages on the same channel reuse the ring (cumulative counters)
@@ -55,11 +56,13 @@ def test_loopback_block_cyclic(torch_cuda, chunk, depth):
     comm.free()
 
 
-def test_loopback_different_types(torch_cuda):
+@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+def test_loopback_different_types(torch_cuda, ring):
     """Same signature, different layouts (vector <-> contiguous, triangle -> packed;
-    [L26:c4303 §5.2.2]); a receive larger than the message fills a prefix (A12)."""
+    [L26:c4303 §5.2.2]); a receive larger than the message fills a prefix (A12).
+    fused = f1, the datatype -> datatype copy without a ring."""
     from paper_conf_hpdc_wubvjd16_b200 import dt
-    comm = dt.Comm(0, 1, 0, chunk_bytes=128 << 10, depth=3)
+    comm = dt.Comm(0, 1, 0, chunk_bytes=128 << 10, depth=3, ring_loopback=ring)
     v, vorg, vpar = c1_submatrix(256, 1024, 1, 1)
     contig = ("contiguous", 256 * 256, ("basic", "DOUBLE"))
     _loop_check(torch_cuda, comm, v, vorg, vpar, contig, 0, 256 * 256 * 8)
@@ -78,9 +81,10 @@ def test_loopback_different_types(torch_cuda):
     comm.free()
 
 
-def test_loopback_short_blocks(torch_cuda):
+@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+def test_loopback_short_blocks(torch_cuda, ring):
     from paper_conf_hpdc_wubvjd16_b200 import dt
-    comm = dt.Comm(0, 1, 0, chunk_bytes=64 << 10, depth=2)
+    comm = dt.Comm(0, 1, 0, chunk_bytes=64 << 10, depth=2, ring_loopback=ring)
     rec, org, parent = c5_particles(1 << 20)
     _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
     comm.free()
@@ -90,7 +94,7 @@ def test_truncation_detected(torch_cuda):
     import torch
 
     from paper_conf_hpdc_wubvjd16_b200 import dt
-    comm = dt.Comm(0, 1, 0, chunk_bytes=64 << 10, depth=2)
+    comm = dt.Comm(0, 1, 0, chunk_bytes=64 << 10, depth=2, ring_loopback=True)
     big = dt.Type.basic("DOUBLE").contiguous(1000).commit()
     small = dt.Type.basic("DOUBLE").contiguous(999).commit()
     s = torch.zeros(8000, dtype=torch.uint8, device="cuda")
@@ -110,7 +114,8 @@ def test_truncation_detected(torch_cuda):
     comm.free()
 
 
-def test_loopback_halo_all_faces(torch_cuda):
+@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+def test_loopback_halo_all_faces(torch_cuda, ring):
     """1-rank periodic halo: the 12 transfers of one exchange in one group."""
     import torch
 
@@ -118,7 +123,7 @@ def test_loopback_halo_all_faces(torch_cuda):
     from paper_conf_hpdc_wubvjd16_b200.halo import FACES, face_box, make_plan
     n, h = 64, 1
     L = n + 2 * h
-    comm = dt.Comm(0, 1, 0, chunk_bytes=16 << 10, depth=2)
+    comm = dt.Comm(0, 1, 0, chunk_bytes=16 << 10, depth=2, ring_loopback=ring)
     plan = make_plan(0, n, h, dims=(1, 1, 1))
     A = np.full((L, L, L), 0xA5A5A5A5, dtype=np.uint32)
     z, y, x = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
@@ -203,3 +208,45 @@ def test_two_processes_one_gpu_ipc(torch_cuda):
         p.join(timeout=60)
     for rank, ok in res:
         assert ok is True, (rank, ok)
+
+
+def test_fused_copy_direct(torch_cuda):
+    """dt_copy (f1) directly: transpose via blocklength-1 vectors ([L26:c4896 §5.2.3]),
+    vector <-> contiguous ([L26:c4303 §5.2.2]), triangle -> block-cyclic-shaped
+    layouts of equal size, both kernel families (forced), truncation, overlap."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    m = 200
+    cases = [
+        (("contiguous", m * m, ("basic", "DOUBLE")), 0, m * m * 8,
+         ("hvector", m, 1, 8, ("vector", m, 1, m, ("basic", "DOUBLE"))), 0, m * m * 8),
+        (c1_submatrix(128, 512, 3, 5)[:3] + (("contiguous", 128 * 128, ("basic", "DOUBLE")), 0, 128 * 128 * 8)),
+        (c2_lower_triangle(257)[:3] + c5_particles(257 * 258 // 2 * 8)[:3]),
+        (c5_particles(56 * 3000)[:3] + (("contiguous", 3000 * 14, ("basic", "INT32")), 0, 3000 * 56)),
+    ]
+    for force in ("", "1", "2"):
+        os.environ["DT_FORCE_KERNEL"] = force
+        for i, (srec, sorg, spar, rrec, rorg, rpar) in enumerate(cases):
+            so, ro = oracle.from_recipe(srec), oracle.from_recipe(rrec)
+            if so.size > ro.size:
+                continue
+            st, rt = dt.from_recipe(srec).commit(), dt.from_recipe(rrec).commit()
+            sh = fill_bytes(spar, 70 + i)
+            exp = np.full(rpar, 0xA5, dtype=np.uint8)
+            oracle.sendrecv(so, 1, sh, ro, 1, exp, sorg, rorg)
+            rd = torch.full((rpar,), 0xA5, dtype=torch.uint8, device="cuda")
+            dt.copy(st, 1, torch.from_numpy(sh).cuda(), rt, 1, rd, src_offset=sorg, dst_offset=rorg)
+            torch.cuda.synchronize()
+            assert np.array_equal(rd.cpu().numpy(), exp), (force, i)
+    os.environ.pop("DT_FORCE_KERNEL", None)
+    a = dt.Type.basic("DOUBLE").contiguous(10).commit()
+    b = dt.Type.basic("DOUBLE").contiguous(9).commit()
+    x = torch.zeros(80, dtype=torch.uint8, device="cuda")
+    with pytest.raises(dt.DTError) as e:
+        dt.copy(a, 1, x, b, 1, x)
+    assert e.value.name == "DT_ERR_TRUNCATE"
+    ov = dt.Type.basic("INT32").vector(4, 3, 2).commit()
+    with pytest.raises(dt.DTError) as e:
+        dt.copy(dt.Type.basic("INT32").contiguous(12).commit(), 1, x, ov, 1, x)
+    assert e.value.name == "DT_ERR_OVERLAP"
