@@ -868,7 +868,8 @@ static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, i
                         template_fits_int32(*fs) && template_fits_int32(*fr);
   const char* fk = getenv("DT_FORCE_KERNEL");
   const int force = fk ? atoi(fk) : 0;
-  const bool use_words = words_ok && force != 1 && (force == 2 || std::min(ms, mr) < 256.0);
+  const double mm = std::min(ms, mr);
+  const bool use_words = words_ok && force != 1 && (force == 2 || mm < 256.0 || (g == 16 && mm < 1024.0));
   const int sms = num_sms();
   if (use_words) {
     const int32_t *wa = nullptr, *wb = nullptr;
