@@ -374,14 +374,78 @@ def run_xfer(args):
         torch.distributed.destroy_process_group()
 
 
+def run_halo(args):
+    """C4: 3D halo exchange of 512^3 f32 per rank (ghost width 1), 6 subarray faces
+    per rank to 3 peers on a periodic grid (2x2x2 at N=8; reading A17), all 12
+    transfers of one exchange in one dt_group.  At N=1 the domain is periodic on
+    itself (every face is a loopback transfer)."""
+    import numpy as np
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import make_plan
+    ws, rank, local = dist_init()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dims = {1: (1, 1, 1), 2: (1, 1, 2), 4: (1, 2, 2), 8: (2, 2, 2)}.get(ws, (1, 1, ws))
+    n, h = 512, 1
+    L = n + 2 * h
+    plan = make_plan(rank, n, h, dims)
+    buf = torch.empty(L * L * L * 4, dtype=torch.uint8, device=dev)
+    buf.view(torch.int32).random_(0, 1 << 30)
+    mode = dt.XFER_NCCL if args.xfer_mode == "nccl" else dt.XFER_P2P
+    kw = dict(chunk_bytes=1 << 20, depth=2, mode=mode, ctas=args.xfer_ctas, ring_loopback=args.ring_loopback)
+    comm = dt.Comm.from_process_group(device=local, **kw) if ws > 1 else \
+        dt.Comm(0, 1, local, nccl_id=dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None, **kw)
+    s = torch.cuda.current_stream()
+    for _ in range(args.warmup):
+        plan.exchange(comm, buf, stream=s)
+    torch.cuda.synchronize()
+    comm.check()
+    ok = None
+    if ws == 1:
+        A = buf.view(torch.int32).view(L, L, L)
+        ok = bool(torch.equal(A[1:-1, 1:-1, 0], A[1:-1, 1:-1, n]) and torch.equal(A[1:-1, 0, 1:-1], A[1:-1, n, 1:-1])
+                  and torch.equal(A[0, 1:-1, 1:-1], A[n, 1:-1, 1:-1]))
+    steps = max(5, min(args.steps, 100))
+    if ws > 1:
+        torch.distributed.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    for _ in range(steps):
+        plan.exchange(comm, buf, stream=s)
+    e1.record(s)
+    torch.cuda.synchronize()
+    comm.check()
+    ms = e0.elapsed_time(e1) / steps
+    if ws > 1:
+        x = torch.tensor([ms], dtype=torch.float64, device=dev)
+        torch.distributed.all_reduce(x, op=torch.distributed.ReduceOp.MAX)
+        ms = float(x[0])
+    face = n * n * h * 4
+    value = ws * 6 * face / (ms * 1e-3) / 1e9
+    line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": ws, "steps": steps,
+            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u8", "data": "synthetic (random f32 bit patterns)",
+            "config": {"workload": f"C4: 3D halo 512^3 f32 per rank, 6 faces x {face} B, grid {dims}, "
+                                   f"mode={args.xfer_mode}", "us_per_exchange": round(ms * 1e3, 2),
+                       "periodic_self_check": ok, "np": np.__version__},
+            "gpu_launches": steps}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        torch.distributed.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--workload", default="c2", choices=["c2", "xfer"])
+    ap.add_argument("--workload", default="c2", choices=["c2", "xfer", "halo"])
     ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl"])
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
     ap.add_argument("--xfer-depths", default="2,4")
     ap.add_argument("--xfer-ctas", type=int, default=0, help="CTAs per direction (0 = library default)")
+    ap.add_argument("--ring-loopback", action="store_true", help="halo at N=1: loopback through the ring pipeline")
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -394,6 +458,8 @@ def main():
         run_reference(args)
     elif args.workload == "xfer":
         run_xfer(args)
+    elif args.workload == "halo":
+        run_halo(args)
     else:
         run_ours(args)
 
