@@ -681,6 +681,75 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const uint8_t* cb, con
   }
 }
 
+// Persistent word cursor of one layout: thread's words tid, tid+nthr, ... of [lo, ..)
+struct WordCursor {
+  int64_t q, ed, Se, Sq;
+  ElemIt ei;
+  __device__ __forceinline__ void init(const KP& P, int64_t x0, int64_t stride_bytes) {
+    const uint64_t e0 = fdiv((uint64_t)x0, P.ftsize);
+    q = x0 - (int64_t)e0 * P.tsize;
+    ei.init(P, e0);
+    ed = ei.disp(P);
+    Se = (int64_t)fdiv((uint64_t)stride_bytes, P.ftsize);
+    Sq = stride_bytes - Se * P.tsize;
+  }
+  __device__ __forceinline__ int64_t addr_off(const int32_t* wt, int G) const { return ed + wt[q / G]; }
+  __device__ __forceinline__ void next(const KP& P) {
+    q += Sq;
+    int64_t k = Se;
+    if (q >= P.tsize) { q -= P.tsize; k++; }
+    if (k) { ei.advance(P, k); ed = ei.disp(P); }
+  }
+};
+
+// Fused type -> type copy staged through shared memory: per 16 KiB tile of the
+// stream, cp.async gathers the words from the source layout S (NB-1 tiles in
+// flight), then the tile is scattered from shared memory to the destination
+// layout R.  Each thread keeps a persistent cursor per layout.
+template <int G, int NB>
+__device__ __forceinline__ void stage_copy(const KP& S, const int32_t* wts, const KP& R, const int32_t* wtr,
+                                           int64_t lo, int64_t hi, uint8_t* sbuf) {
+  typedef typename WordT<G>::T W;
+  constexpr int T = kStageTile, L = NB - 1;
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  const int64_t ntiles = (hi - lo + T - 1) / T;
+  const int64_t nwords = (hi - lo) / G;
+  WordCursor cs, cr;
+  if (tid < nwords) {
+    cs.init(S, lo + (int64_t)tid * G, (int64_t)nthr * G);
+    cr.init(R, lo + (int64_t)tid * G, (int64_t)nthr * G);
+  }
+  int64_t iw = tid, jw = tid;
+  for (int64_t t = 0; t < ntiles + L - 1; t++) {
+    if (t < ntiles) {
+      uint8_t* buf = sbuf + (t % NB) * T - t * T;
+      const int64_t wend = (t + 1) * (T / G) < nwords ? (t + 1) * (T / G) : nwords;
+      while (iw < wend) {
+        cp_async<G>(buf + iw * G, S.nc + cs.addr_off(wts, G));
+        iw += nthr;
+        if (iw >= nwords) break;
+        cs.next(S);
+      }
+    }
+    cp_async_commit();
+    const int64_t u = t - (L - 1);
+    if (u >= 0) {
+      cp_async_wait<L - 1>();
+      __syncthreads();
+      const uint8_t* buf = sbuf + (u % NB) * T - u * T;
+      const int64_t wend = (u + 1) * (T / G) < nwords ? (u + 1) * (T / G) : nwords;
+      while (jw < wend) {
+        *reinterpret_cast<W*>(const_cast<uint8_t*>(R.nc) + cr.addr_off(wtr, G)) =
+            *reinterpret_cast<const W*>(buf + jw * G);
+        jw += nthr;
+        if (jw >= nwords) break;
+        cr.next(R);
+      }
+      __syncthreads();  // tile buffer free for the gather NB tiles later
+    }
+  }
+}
+
 // Fused type -> type copy of G-granular templates: thread tid moves words tid,
 // tid+nthr, ... of [lo, hi): source address from S's word table + element
 // iterator, destination from R's; NV words in flight per thread.

@@ -163,6 +163,20 @@ __global__ void __launch_bounds__(256, 3) k_dual_seg(const KP S, const KP R, int
 }
 
 template <int G>
+__global__ void __launch_bounds__(256) k_dual_stage(const KP S, const KP R, int64_t n, int64_t ntiles) {
+  extern __shared__ __align__(128) uint8_t smem_dual[];
+  uint8_t* sbuf = smem_dual;
+  int32_t* wts = reinterpret_cast<int32_t*>(smem_dual + kStageBufs * kStageTile);
+  int32_t* wtr = wts + S.nwords;
+  for (int i = threadIdx.x; i < S.nwords; i += blockDim.x) wts[i] = S.wtab[i];
+  for (int i = threadIdx.x; i < R.nwords; i += blockDim.x) wtr[i] = R.wtab[i];
+  __syncthreads();
+  const int64_t t0 = ntiles * blockIdx.x / gridDim.x, t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
+  const int64_t lo = t0 * kStageTile, hi = t1 * kStageTile < n ? t1 * kStageTile : n;
+  if (lo < hi) stage_copy<G, kStageBufs>(S, wts, R, wtr, lo, hi, sbuf);
+}
+
+template <int G>
 __global__ void __launch_bounds__(256) k_dual_word(const KP S, const KP R, int64_t n) {
   extern __shared__ int32_t wts[];
   int32_t* wtr = wts + S.nwords;
@@ -883,6 +897,25 @@ static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, i
     R.nwords = (int32_t)(R.tsize / g);
     const size_t smem = sizeof(int32_t) * (size_t)(S.nwords + R.nwords);
     const int64_t nwords = n / g;
+    if (g >= 8 && force != 5) {  // staged: cp.async gathers by S into smem tiles, scatter by R
+      const size_t smem2 = (size_t)kStageBufs * kStageTile + smem;
+      static bool attr = false;
+      if (!attr) {
+        cudaFuncSetAttribute(k_dual_stage<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
+        cudaFuncSetAttribute(k_dual_stage<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
+        attr = true;
+      }
+      int occ = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dual_stage<16>, 256, smem2) != cudaSuccess || occ < 1)
+        occ = 1;
+      const int64_t ntiles = (n + kStageTile - 1) / kStageTile;
+      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
+      if (g == 8) k_dual_stage<8><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
+      else k_dual_stage<16><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return cuda_fail(e, "dt_copy launch");
+      return DT_OK;
+    }
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * 6, (nwords + 1023) / 1024));
     switch (g) {
       case 1: k_dual_word<1><<<grid, 256, smem, s>>>(S, R, n); break;
