@@ -681,6 +681,63 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const uint8_t* cb, con
   }
 }
 
+// Dense-span pack (short blocks inside small, dense records, e.g. C5's 56-of-64-byte
+// particles): per tile of E elements, 16-byte cp.async copies the whole aligned
+// span [a0, a0+spanB) of every element into shared memory (4x fewer, fully
+// aligned requests than 4-byte word gathers), threads compact the template's
+// G-byte words into the packed tile (shared -> shared), one TMA bulk store writes
+// it out.  Requires 16-byte aligned element bases and the full stream (pos = 0).
+template <int G, int NB>
+__device__ __forceinline__ void span_pack(const KP& P, uint8_t* cb, const int32_t* wsp, int64_t a0, int spanB,
+                                          int E, int64_t e_lo, int64_t e_hi, uint8_t* sbuf) {
+  typedef typename WordT<G>::T W;
+  constexpr int L = NB - 1;
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  const int nch = spanB / 16;
+  const int nw = (int)(P.tsize / G);
+  const int64_t stage = (int64_t)E * spanB + (int64_t)E * P.tsize;
+  const int64_t ntiles = (e_hi - e_lo + E - 1) / E;
+  for (int64_t t = 0; t < ntiles + L - 1; t++) {
+    if (t < ntiles) {
+      uint8_t* span = sbuf + (t % NB) * stage;
+      if (tid == 0) bulk_wait_read<1>();
+      __syncthreads();
+      const int64_t e0 = e_lo + t * E;
+      const int ne = (int)(e_hi - e0 < E ? e_hi - e0 : E);
+      for (int k = tid; k < ne * nch; k += nthr) {
+        const int i = k / nch, c = k - i * nch;
+        cp_async<16>(span + i * spanB + 16 * c, P.nc + elem_disp(P, (uint64_t)(e0 + i)) + a0 + 16 * c);
+      }
+    }
+    cp_async_commit();
+    const int64_t u = t - (L - 1);
+    if (u >= 0) {
+      cp_async_wait<L - 1>();
+      __syncthreads();
+      const uint8_t* span = sbuf + (u % NB) * stage;
+      uint8_t* pk = sbuf + (u % NB) * stage + (int64_t)E * spanB;
+      const int64_t e0 = e_lo + u * E;
+      const int ne = (int)(e_hi - e0 < E ? e_hi - e0 : E);
+      for (int w = tid; w < ne * nw; w += nthr) {
+        const int i = w / nw, k = w - i * nw;
+        *reinterpret_cast<W*>(pk + (int64_t)w * G) = *reinterpret_cast<const W*>(span + i * spanB + wsp[k]);
+      }
+      __syncthreads();
+      if (tid == 0) {
+        const int64_t bytes = (int64_t)ne * P.tsize;
+        uint8_t* dst = cb + e0 * P.tsize;
+        fence_proxy_async();
+        if (bytes >= 16) {
+          bulk_store(dst, pk, (uint32_t)(bytes & ~int64_t(15)));
+          bulk_commit();
+        }
+        for (int64_t k = bytes & ~int64_t(15); k < bytes; k++) dst[k] = pk[k];
+      }
+    }
+  }
+  if (tid == 0) bulk_wait_all();
+}
+
 // Persistent word cursor of one layout: thread's words tid, tid+nthr, ... of [lo, ..)
 struct WordCursor {
   int64_t q, ed, Se, Sq;

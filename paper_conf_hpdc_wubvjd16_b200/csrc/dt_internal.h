@@ -38,14 +38,18 @@ struct Form {
   std::vector<Level> lv;           // outermost first
   std::vector<int64_t> bd, bl;     // template blocks (bytes), typemap order
   // per-call planning must stay O(levels): O(n) facts are computed once and cached
-  mutable int64_t gran_cache = -1, tsize_cache = -1;
+  mutable int64_t gran_cache = -1, tsize_cache = -1, lvl_gran_cache = -1;
   mutable int fits32_cache = -1;
   int64_t tsize() const {
     if (tsize_cache < 0) { int64_t s = 0; for (auto x : bl) s += x; tsize_cache = s; }
     return tsize_cache;
   }
   mutable std::vector<int64_t> hoff_cache;  // host exclusive prefix of bl (launch planning)
-  void invalidate() const { gran_cache = tsize_cache = -1; fits32_cache = -1; hoff_cache.clear(); }
+  void invalidate() const {
+    gran_cache = tsize_cache = lvl_gran_cache = -1;
+    fits32_cache = -1;
+    hoff_cache.clear();
+  }
   const std::vector<int64_t>& hoff() const {
     if (hoff_cache.size() != bl.size()) {
       hoff_cache.resize(bl.size());
@@ -62,6 +66,8 @@ void normalize(Form& f);
 // Expand into merged blocks (typemap order).  Returns false if > cap.
 bool expand(const Form& f, std::vector<int64_t>& d, std::vector<int64_t>& l, int64_t cap);
 int64_t form_granularity(const Form& f);
+// largest power of two <= 16 dividing every level stride / list entry (element bases)
+int64_t level_granularity(const Form& f);
 
 // Per-device copy of the descriptor.
 struct DeviceDesc {

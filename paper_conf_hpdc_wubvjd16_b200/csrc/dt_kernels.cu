@@ -154,6 +154,22 @@ __global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
   else stage_pack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf);
 }
 
+// dense-span pack: CTA c owns a contiguous run of E-element tiles
+constexpr int kSpanBufs = 3;
+template <int G>
+__global__ void __launch_bounds__(256) k_span(const KP P, int64_t ntiles, int64_t a0, int spanB, int E,
+                                              int64_t nel) {
+  extern __shared__ __align__(128) uint8_t smem_span[];
+  const int nw = (int)(P.tsize / G);
+  int32_t* wsp = reinterpret_cast<int32_t*>(smem_span);
+  uint8_t* sbuf = smem_span + ((nw * 4 + 127) & ~127);
+  for (int i = threadIdx.x; i < nw; i += blockDim.x) wsp[i] = P.wtab[i] - (int32_t)a0;
+  __syncthreads();
+  const int64_t t0 = ntiles * blockIdx.x / gridDim.x, t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
+  const int64_t e_lo = t0 * E, e_hi = t1 * E < nel ? t1 * E : nel;
+  if (e_lo < e_hi) span_pack<G, kSpanBufs>(P, P.c - P.pos, wsp, a0, spanB, E, e_lo, e_hi, sbuf);
+}
+
 // f1: fused type -> type copies (no packed buffer)
 __global__ void __launch_bounds__(256, 3) k_dual_seg(const KP S, const KP R, int64_t n, int64_t per_warp) {
   const int lane = threadIdx.x & 31;
@@ -531,6 +547,62 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
   // SMs a pack/unpack needs, e.g. to leave the rest to a co-running application)
   const char* ms = getenv("DT_MAX_SMS");
   const int sms = ms && atoi(ms) > 0 ? std::min(num_sms(), atoi(ms)) : num_sms();
+  // dense-span pack: short blocks (word kernels) inside small dense 16-byte-aligned records
+  if (!unpack && (kind == 2 || kind == 4) && !E.merged && pos == 0 && P.tsize > 0 && len % P.tsize == 0) {
+    int64_t tg = 16;  // template word size
+    for (size_t b = 0; b < f.bd.size(); b++) tg = std::min(tg, std::min(lowp2((uint64_t)f.bd[b]), lowp2((uint64_t)f.bl[b])));
+    int64_t lg = level_granularity(f);
+    for (int i = 0; i < L.n; i++)
+      if (!L.table[i]) lg = std::min(lg, lowp2((uint64_t)L.stride[i]));
+    int64_t lo_b = INT64_MAX, hi_b = INT64_MIN;
+    for (size_t b = 0; b < f.bd.size(); b++) {
+      lo_b = std::min(lo_b, f.bd[b]);
+      hi_b = std::max(hi_b, f.bd[b] + f.bl[b]);
+    }
+    const int64_t a0 = lo_b >= 0 ? lo_b & ~int64_t(15) : -((-lo_b + 15) & ~int64_t(15));
+    const int64_t spanB = ((hi_b - a0) + 15) & ~int64_t(15);
+    const char* fk = getenv("DT_FORCE_KERNEL");
+    const bool no_span = fk && atoi(fk) != 5;
+    if (!no_span && tg >= 4 && lg >= 16 && (((uintptr_t)nc) & 15) == 0 && (((uintptr_t)c) & 15) == 0 &&
+        spanB <= 512 && 2 * P.tsize >= spanB && template_fits_int32(f) && P.tsize % tg == 0 &&
+        P.tsize / tg <= kMaxWordTable) {
+      int64_t m = 16;
+      for (int64_t x = P.tsize; m > 1 && x % m; m >>= 1) {
+      }
+      m = 16 / m;  // elements per 16-byte-aligned packed boundary
+      int64_t Ee = std::min<int64_t>(16384 / spanB, 16384 / P.tsize) / m * m;
+      if (Ee >= m) {
+        const int32_t* wt = nullptr;
+        dt_status st = ensure_wtab(f, dd, tg, &wt);
+        if (st != DT_OK) return st;
+        P.wtab = wt;
+        P.nwords = (int32_t)(P.tsize / tg);
+        const int64_t nel = len / P.tsize;
+        const int64_t ntiles = (nel + Ee - 1) / Ee;
+        const size_t smem = (size_t)((P.nwords * 4 + 127) & ~127) +
+                            (size_t)kSpanBufs * (size_t)(Ee * spanB + Ee * P.tsize);
+        static bool attr = false;
+        if (!attr) {
+          cudaFuncSetAttribute(k_span<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+          cudaFuncSetAttribute(k_span<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+          cudaFuncSetAttribute(k_span<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+          attr = true;
+        }
+        int occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_span<4>, 256, smem) != cudaSuccess || occ < 1)
+          occ = 1;
+        const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
+        switch (tg) {
+          case 4: k_span<4><<<grid, 256, smem, s>>>(P, ntiles, a0, (int)spanB, (int)Ee, nel); break;
+          case 8: k_span<8><<<grid, 256, smem, s>>>(P, ntiles, a0, (int)spanB, (int)Ee, nel); break;
+          default: k_span<16><<<grid, 256, smem, s>>>(P, ntiles, a0, (int)spanB, (int)Ee, nel); break;
+        }
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_fail(e, "span kernel launch");
+        return DT_OK;
+      }
+    }
+  }
   if (kind == 1) {
     // exactly one wave of resident CTAs (no tail wave), at least ~4 KiB per warp
     const bool single = P.nblocks == 1;

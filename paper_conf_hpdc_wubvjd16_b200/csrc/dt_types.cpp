@@ -438,6 +438,17 @@ static int64_t low_pow2(int64_t x) {
   return g > 16 ? 16 : g;
 }
 
+int64_t level_granularity(const Form& f) {
+  if (f.lvl_gran_cache >= 0) return f.lvl_gran_cache;
+  int64_t g = 16;
+  for (auto& l : f.lv) {
+    if (l.is_list()) for (auto x : *l.table) g = std::min(g, low_pow2(x));
+    else g = std::min(g, low_pow2(l.stride));
+  }
+  f.lvl_gran_cache = g;
+  return g;
+}
+
 int64_t form_granularity(const Form& f) {
   if (f.gran_cache >= 0) return f.gran_cache;
   int64_t g = 16;

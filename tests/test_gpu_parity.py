@@ -170,7 +170,7 @@ def test_random_tiny_types(torch_cuda):
                 raise
 
 
-@pytest.mark.parametrize("kind", ["1", "2", "3", "4"])
+@pytest.mark.parametrize("kind", ["1", "2", "3", "4", "5"])
 @pytest.mark.parametrize("name", ["C1b", "C2s", "C3s", "C4x", "C4y", "C5", "C5b", "ctg"])
 def test_every_kernel_family(torch_cuda, kind, name, monkeypatch):
     """Every kernel family (1 warp segments, 2 word table, 3 block windows, 4 smem/TMA
