@@ -421,9 +421,13 @@ __device__ __forceinline__ void word_range(const KP& P, uint8_t* cb, const int64
   for (int64_t v0 = tid; v0 < nvec; v0 += nthr * NV) {
     U u[NV];
     int nvalid[NV];
-    int64_t ed[NV];
+    int64_t ed[NV], edn[NV];
     uint64_t e[NV];
     int w[NV];
+    // when an element holds >= VW bytes a vector crosses at most one element
+    // boundary: the next element's displacement (a list-table load for index
+    // lists) is fetched up front instead of on the critical path mid-vector
+    const bool one_cross = P.tsize >= VW;
 #pragma unroll
     for (int j = 0; j < NV; j++) {
       const int64_t v = v0 + (int64_t)j * nthr;
@@ -433,6 +437,7 @@ __device__ __forceinline__ void word_range(const KP& P, uint8_t* cb, const int64
       e[j] = fdiv((uint64_t)s0, P.ftsize);
       w[j] = (int)((s0 - (int64_t)e[j] * P.tsize) / G);
       ed[j] = nvalid[j] > 0 ? elem_disp(P, e[j]) : 0;
+      edn[j] = (one_cross && nvalid[j] > 0 && w[j] + nvalid[j] > P.nwords) ? elem_disp(P, e[j] + 1) : 0;
       if (UNPACK) {
         if (nvalid[j] == NW) u[j].vec = ldv<POL>(reinterpret_cast<const VT*>(cv + v * VW));
         else
@@ -450,7 +455,7 @@ __device__ __forceinline__ void word_range(const KP& P, uint8_t* cb, const int64
           if (++w[j] == P.nwords && k + 1 < nvalid[j]) {
             w[j] = 0;
             ++e[j];
-            ed[j] = elem_disp(P, e[j]);
+            ed[j] = one_cross ? edn[j] : elem_disp(P, e[j]);
           }
         }
       }
