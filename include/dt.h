@@ -150,7 +150,9 @@ dt_status dt_get_form(dt_t t, dt_form_info* out);
  * (host arrays of capacity max); *nblocks = total blocks (may exceed max). */
 dt_status dt_flatten(dt_t t, int64_t count, int64_t* disps, int64_t* lens, int64_t max, int64_t* nblocks);
 /* Which kernel dt_pack would launch for this request: 0 none, 1 warp-segment
- * ("long"), 2 word-table ("short"); *granularity = word size in bytes. */
+ * ("long"), 2 word-table ("short", register staged), 3 block windows (short
+ * blocks under a large template), 4 shared-memory/TMA staging, 6 record spans
+ * (short blocks inside small dense records); *granularity = word size in bytes. */
 dt_status dt_plan(dt_t t, int64_t count, uint64_t origin_addr, uint64_t packed_addr, int64_t pos, int64_t len,
                   int* kernel, int64_t* granularity);
 

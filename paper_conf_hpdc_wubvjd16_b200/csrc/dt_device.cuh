@@ -686,63 +686,6 @@ __device__ __forceinline__ void stage_unpack(const KP& P, const uint8_t* cb, con
   }
 }
 
-// Dense-span pack (short blocks inside small, dense records, e.g. C5's 56-of-64-byte
-// particles): per tile of E elements, 16-byte cp.async copies the whole aligned
-// span [a0, a0+spanB) of every element into shared memory (4x fewer, fully
-// aligned requests than 4-byte word gathers), threads compact the template's
-// G-byte words into the packed tile (shared -> shared), one TMA bulk store writes
-// it out.  Requires 16-byte aligned element bases and the full stream (pos = 0).
-template <int G, int NB>
-__device__ __forceinline__ void span_pack(const KP& P, uint8_t* cb, const int32_t* wsp, int64_t a0, int spanB,
-                                          int E, int64_t e_lo, int64_t e_hi, uint8_t* sbuf) {
-  typedef typename WordT<G>::T W;
-  constexpr int L = NB - 1;
-  const int tid = threadIdx.x, nthr = blockDim.x;
-  const int nch = spanB / 16;
-  const int nw = (int)(P.tsize / G);
-  const int64_t stage = (int64_t)E * spanB + (int64_t)E * P.tsize;
-  const int64_t ntiles = (e_hi - e_lo + E - 1) / E;
-  for (int64_t t = 0; t < ntiles + L - 1; t++) {
-    if (t < ntiles) {
-      uint8_t* span = sbuf + (t % NB) * stage;
-      if (tid == 0) bulk_wait_read<1>();
-      __syncthreads();
-      const int64_t e0 = e_lo + t * E;
-      const int ne = (int)(e_hi - e0 < E ? e_hi - e0 : E);
-      for (int k = tid; k < ne * nch; k += nthr) {
-        const int i = k / nch, c = k - i * nch;
-        cp_async<16>(span + i * spanB + 16 * c, P.nc + elem_disp(P, (uint64_t)(e0 + i)) + a0 + 16 * c);
-      }
-    }
-    cp_async_commit();
-    const int64_t u = t - (L - 1);
-    if (u >= 0) {
-      cp_async_wait<L - 1>();
-      __syncthreads();
-      const uint8_t* span = sbuf + (u % NB) * stage;
-      uint8_t* pk = sbuf + (u % NB) * stage + (int64_t)E * spanB;
-      const int64_t e0 = e_lo + u * E;
-      const int ne = (int)(e_hi - e0 < E ? e_hi - e0 : E);
-      for (int w = tid; w < ne * nw; w += nthr) {
-        const int i = w / nw, k = w - i * nw;
-        *reinterpret_cast<W*>(pk + (int64_t)w * G) = *reinterpret_cast<const W*>(span + i * spanB + wsp[k]);
-      }
-      __syncthreads();
-      if (tid == 0) {
-        const int64_t bytes = (int64_t)ne * P.tsize;
-        uint8_t* dst = cb + e0 * P.tsize;
-        fence_proxy_async();
-        if (bytes >= 16) {
-          bulk_store(dst, pk, (uint32_t)(bytes & ~int64_t(15)));
-          bulk_commit();
-        }
-        for (int64_t k = bytes & ~int64_t(15); k < bytes; k++) dst[k] = pk[k];
-      }
-    }
-  }
-  if (tid == 0) bulk_wait_all();
-}
-
 // Persistent word cursor of one layout: thread's words tid, tid+nthr, ... of [lo, ..)
 struct WordCursor {
   int64_t q, ed, Se, Sq;
@@ -939,6 +882,141 @@ __device__ __forceinline__ void blk_range(const KP& P, uint8_t* cbase, int64_t p
     }
     __syncwarp();
   }
+}
+
+// ---------------------------------------------------------------- record spans
+// Short blocks inside small dense records (C5's 56-of-64-byte particles; any
+// template whose blocks lie in a 16-byte-aligned span of <= 128 B that is at least
+// half payload, with 16-byte-aligned element bases).  A warp moves RB whole
+// records per batch (RB a multiple of 32, so every batch starts on a 16-byte
+// boundary of the packed stream).
+//   pack:   each lane issues its LPL 16-byte loads of the records' spans (all in
+//           flight together; 4 lanes per 64-byte record), parks them in a per-warp
+//           shared buffer, then assembles coalesced 16-byte vectors of the packed
+//           stream from the template words (offset table `omap` in shared memory);
+//   unpack: the packed vectors land in the shared buffer, each lane writes span
+//           chunks: one 16-byte store when the template covers the chunk, G-byte
+//           stores of the covered words otherwise (gap bytes stay untouched).
+// Compared with gathering G-byte words (k_word), every DRAM sector of a record is
+// requested by one 16-byte access instead of 16/G word accesses.
+struct RecGeo {
+  int64_t a0;          // span start relative to the element displacement (16-aligned)
+  int32_t spanB, nch;  // span bytes (multiple of 16, <= 128) and 16-byte chunks
+  int32_t RB, LPL;     // records per warp batch (multiple of 32), chunks per lane (RB*nch/32)
+  int32_t nwr;         // template words per record (tsize / G)
+  int32_t invnch;      // ceil(2^16 / nch): idx / nch = (idx * invnch) >> 16 for idx < 4096
+  int64_t e_lo, e_hi;  // elements touching [pos, pos+len)
+  int64_t b0, nbatch;  // first batch element (multiple of 32) and number of batches
+};
+constexpr int kRecMaxLPL = 8;
+
+template <int G>
+__device__ __forceinline__ void rec_pack_batch(const KP& P, const RecGeo& R, uint8_t* cb, int64_t e0, uint8_t* buf,
+                                               const int64_t* sd, const uint16_t* omap, int lane) {
+  typedef typename WordT<G>::T W;
+  constexpr int NW = 16 / G;
+  const int64_t end = P.pos + P.len;
+  uint4 v[kRecMaxLPL];
+#pragma unroll
+  for (int j = 0; j < kRecMaxLPL; j++) {
+    if (j < R.LPL) {
+      const int idx = lane + 32 * j;
+      const int r = (idx * R.invnch) >> 16, ch = idx - r * R.nch;
+      const int64_t e = e0 + r;
+      if (e >= R.e_lo && e < R.e_hi) v[j] = ldv<LD_CS>(reinterpret_cast<const uint4*>(P.nc + sd[r] + R.a0 + 16 * ch));
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < kRecMaxLPL; j++)
+    if (j < R.LPL) reinterpret_cast<uint4*>(buf)[lane + 32 * j] = v[j];  // (unloaded chunks: never output)
+  __syncwarp();
+  const int nvec = (int)((int64_t)R.RB * P.tsize / 16);  // RB is a multiple of 32: exact
+  const int64_t sb = e0 * P.tsize;
+  for (int vv = lane; vv < nvec; vv += 32) {
+    const int64_t s = sb + 16 * (int64_t)vv;
+    if (s + 16 <= P.pos || s >= end) continue;
+    union {
+      uint4 q;
+      W w[NW];
+    } o;
+#pragma unroll
+    for (int k = 0; k < NW; k++) o.w[k] = *reinterpret_cast<const W*>(buf + omap[vv * NW + k]);
+    if (s >= P.pos && s + 16 <= end) {
+      stv(reinterpret_cast<uint4*>(cb + s), o.q);
+    } else {
+      const uint8_t* ob = reinterpret_cast<const uint8_t*>(&o.q);
+      for (int k = 0; k < 16; k++)
+        if (s + k >= P.pos && s + k < end) cb[s + k] = ob[k];
+    }
+  }
+  __syncwarp();
+}
+
+template <int G>
+__device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, const uint8_t* cb, int64_t e0,
+                                                 uint8_t* buf, const int64_t* sd, const int16_t* umap, int lane) {
+  typedef typename WordT<G>::T W;
+  constexpr int NW = 16 / G;
+  const int64_t end = P.pos + P.len;
+  const int nvec = (int)((int64_t)R.RB * P.tsize / 16);
+  const int64_t sb = e0 * P.tsize;
+  uint4 v[kRecMaxLPL];
+#pragma unroll
+  for (int j = 0; j < kRecMaxLPL; j++) {  // nvec <= RB*spanB/16 = 32*LPL
+    const int vv = lane + 32 * j;
+    const int64_t s = sb + 16 * (int64_t)vv;
+    if (j < R.LPL && vv < nvec && s >= P.pos && s + 16 <= end) v[j] = ldv<LD_CS>(reinterpret_cast<const uint4*>(cb + s));
+  }
+#pragma unroll
+  for (int j = 0; j < kRecMaxLPL; j++) {
+    const int vv = lane + 32 * j;
+    const int64_t s = sb + 16 * (int64_t)vv;
+    if (j < R.LPL && vv < nvec) {
+      if (s >= P.pos && s + 16 <= end) reinterpret_cast<uint4*>(buf)[vv] = v[j];
+      else if (s + 16 > P.pos && s < end)  // ragged ends of the request: in-range words only
+        for (int k = 0; k < 16; k += G)
+          if (s + k >= P.pos && s + k + G <= end)
+            *reinterpret_cast<W*>(buf + 16 * vv + k) = *reinterpret_cast<const W*>(cb + s + k);
+    }
+  }
+  __syncwarp();
+#pragma unroll
+  for (int j = 0; j < kRecMaxLPL; j++) {
+    if (j < R.LPL) {
+      const int idx = lane + 32 * j;
+      const int r = (idx * R.invnch) >> 16, ch = idx - r * R.nch;
+      const int64_t e = e0 + r;
+      if (e >= R.e_lo && e < R.e_hi) {
+        const int64_t rs = e * P.tsize;  // stream byte of the record's first word
+        const bool whole = rs >= P.pos && rs + P.tsize <= end;
+        union {
+          uint4 q;
+          W w[NW];
+        } o;
+        unsigned mask = 0;
+#pragma unroll
+        for (int k = 0; k < NW; k++) {
+          const int m = umap[ch * NW + k];
+          if (m >= 0) {
+            const int64_t x = rs + (int64_t)m * G;
+            if (whole || (x >= P.pos && x + G <= end)) {
+              o.w[k] = *reinterpret_cast<const W*>(buf + (int64_t)r * P.tsize + (int64_t)m * G);
+              mask |= 1u << k;
+            }
+          }
+        }
+        uint8_t* d = const_cast<uint8_t*>(P.nc) + sd[r] + R.a0 + 16 * ch;
+        if (mask == (1u << NW) - 1) {
+          stv(reinterpret_cast<uint4*>(d), o.q);
+        } else {
+#pragma unroll
+          for (int k = 0; k < NW; k++)
+            if (mask & (1u << k)) reinterpret_cast<W*>(d)[k] = o.w[k];
+        }
+      }
+    }
+  }
+  __syncwarp();
 }
 
 }  // namespace dt

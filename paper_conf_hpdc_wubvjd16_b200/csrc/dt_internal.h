@@ -40,6 +40,20 @@ struct Form {
   // per-call planning must stay O(levels): O(n) facts are computed once and cached
   mutable int64_t gran_cache = -1, tsize_cache = -1, lvl_gran_cache = -1;
   mutable int fits32_cache = -1;
+  mutable int64_t span_lo = 0, span_hi = -1;  // cached min bd / max bd+bl (span_hi < span_lo: not computed)
+  void span(int64_t* lo, int64_t* hi) const {
+    if (span_hi < span_lo) {
+      int64_t a = INT64_MAX, b = INT64_MIN;
+      for (size_t i = 0; i < bd.size(); i++) {
+        a = bd[i] < a ? bd[i] : a;
+        b = bd[i] + bl[i] > b ? bd[i] + bl[i] : b;
+      }
+      span_lo = a;
+      span_hi = b;
+    }
+    *lo = span_lo;
+    *hi = span_hi;
+  }
   int64_t tsize() const {
     if (tsize_cache < 0) { int64_t s = 0; for (auto x : bl) s += x; tsize_cache = s; }
     return tsize_cache;
@@ -48,6 +62,8 @@ struct Form {
   void invalidate() const {
     gran_cache = tsize_cache = lvl_gran_cache = -1;
     fits32_cache = -1;
+    span_lo = 0;
+    span_hi = -1;
     hoff_cache.clear();
   }
   const std::vector<int64_t>& hoff() const {

@@ -154,22 +154,6 @@ __global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
   else stage_pack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf);
 }
 
-// dense-span pack: CTA c owns a contiguous run of E-element tiles
-constexpr int kSpanBufs = 3;
-template <int G>
-__global__ void __launch_bounds__(256) k_span(const KP P, int64_t ntiles, int64_t a0, int spanB, int E,
-                                              int64_t nel) {
-  extern __shared__ __align__(128) uint8_t smem_span[];
-  const int nw = (int)(P.tsize / G);
-  int32_t* wsp = reinterpret_cast<int32_t*>(smem_span);
-  uint8_t* sbuf = smem_span + ((nw * 4 + 127) & ~127);
-  for (int i = threadIdx.x; i < nw; i += blockDim.x) wsp[i] = P.wtab[i] - (int32_t)a0;
-  __syncthreads();
-  const int64_t t0 = ntiles * blockIdx.x / gridDim.x, t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
-  const int64_t e_lo = t0 * E, e_hi = t1 * E < nel ? t1 * E : nel;
-  if (e_lo < e_hi) span_pack<G, kSpanBufs>(P, P.c - P.pos, wsp, a0, spanB, E, e_lo, e_hi, sbuf);
-}
-
 // f1: fused type -> type copies (no packed buffer)
 __global__ void __launch_bounds__(256, 3) k_dual_seg(const KP S, const KP R, int64_t n, int64_t per_warp) {
   const int lane = threadIdx.x & 31;
@@ -201,6 +185,43 @@ __global__ void __launch_bounds__(256) k_dual_word(const KP S, const KP R, int64
   __syncthreads();
   dual_words<G, 4>(S, wts, R, wtr, 0, n, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                    (int64_t)gridDim.x * blockDim.x);
+}
+
+// record-span pack/unpack (short blocks in small dense records): warp w takes
+// batches w, w + nwarps, ... of RB records
+template <bool UNPACK, int G>
+__global__ void __launch_bounds__(256, 3) k_rec(const KP P, const RecGeo R) {
+  extern __shared__ __align__(16) uint8_t smem_rec[];
+  const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int bufB = R.RB * R.spanB;
+  uint8_t* buf = smem_rec + w * bufB;
+  int64_t* sd = reinterpret_cast<int64_t*>(smem_rec + nwc * bufB) + w * R.RB;
+  uint16_t* omap = reinterpret_cast<uint16_t*>(smem_rec + nwc * bufB + nwc * R.RB * 8);
+  int16_t* umap = reinterpret_cast<int16_t*>(omap);
+  // maps from the template's G-word table (source offset of packed word k)
+  if (!UNPACK) {
+    const int n = R.RB * R.nwr;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+      const int r = i / R.nwr, k = i - r * R.nwr;
+      omap[i] = (uint16_t)(r * R.spanB + (int)(P.wtab[k] - R.a0));
+    }
+  } else {
+    for (int i = threadIdx.x; i < R.spanB / G; i += blockDim.x) umap[i] = -1;
+    __syncthreads();
+    for (int k = threadIdx.x; k < R.nwr; k += blockDim.x) umap[(int)(P.wtab[k] - R.a0) / G] = (int16_t)k;
+  }
+  __syncthreads();
+  const int64_t nwt = (int64_t)gridDim.x * nwc;
+  for (int64_t b = (int64_t)blockIdx.x * nwc + w; b < R.nbatch; b += nwt) {
+    const int64_t e0 = R.b0 + b * R.RB;
+    for (int i = lane; i < R.RB; i += 32) {
+      const int64_t e = e0 + i;
+      sd[i] = (e >= R.e_lo && e < R.e_hi) ? elem_disp(P, (uint64_t)e) : 0;
+    }
+    __syncwarp();
+    if (UNPACK) rec_unpack_batch<G>(P, R, P.c - P.pos, e0, buf, sd, umap, lane);
+    else rec_pack_batch<G>(P, R, P.c - P.pos, e0, buf, sd, omap, lane);
+  }
 }
 
 template <bool UNPACK, int G, int VW>
@@ -449,6 +470,38 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
   return DT_OK;
 }
 
+// Record-span geometry of a launch (k_rec), or false when it does not apply:
+// G >= 4, 16-byte-aligned element bases and packed side, the template inside a
+// 16-byte-aligned span of <= 128 B that is at least half payload.
+static bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos,
+                         int64_t len, int64_t g, RecGeo* R) {
+  if (g < 4 || f.bl.empty() || len <= 0) return false;
+  if ((nc_addr & 15) || ((c_addr - (uint64_t)pos) & 15)) return false;
+  int64_t lg = level_granularity(f);
+  for (int i = 0; i < L.n; i++)
+    if (!L.table[i]) lg = std::min(lg, lowp2((uint64_t)L.stride[i]));
+  if (lg < 16) return false;
+  if (f.bl.size() > 64) return false;  // (a <= 128-byte span holds few blocks; keeps planning O(1))
+  int64_t lo, hi;
+  f.span(&lo, &hi);
+  const int64_t a0 = lo >= 0 ? lo & ~int64_t(15) : -((-lo + 15) & ~int64_t(15));
+  const int64_t spanB = ((hi - a0) + 15) & ~int64_t(15);
+  const int64_t ts = f.tsize();
+  if (spanB > 128 || 2 * ts < spanB || ts % g) return false;
+  R->a0 = a0;
+  R->spanB = (int32_t)spanB;
+  R->nch = (int32_t)(spanB / 16);
+  R->RB = 32 * (8 / R->nch);
+  R->LPL = R->RB * R->nch / 32;
+  R->nwr = (int32_t)(ts / g);
+  R->invnch = (65536 + R->nch - 1) / R->nch;
+  R->e_lo = pos / ts;
+  R->e_hi = (pos + len + ts - 1) / ts;
+  R->b0 = R->e_lo & ~int64_t(31);
+  R->nbatch = (R->e_hi - R->b0 + R->RB - 1) / R->RB;
+  return true;
+}
+
 int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
                 int64_t* gran) {
   if (len <= 0 || f.bl.empty()) return 0;
@@ -468,6 +521,9 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   const int force = fk ? atoi(fk) : 0;
   const bool blk_ok = (c_addr & 15) == 0 && ts % g == 0;
   const bool stage_ok = word_ok && g >= 4 && (c_addr & 15) == 0;
+  RecGeo rg;
+  const bool rec_ok = rec_geometry(f, L, nc_addr, c_addr, pos, len, g, &rg);
+  if (force == 6 && rec_ok) return 6;
   if (force == 2 && word_ok) return 2;
   if (force == 3 && blk_ok) return 3;
   if (force == 4 && stage_ok) return 4;
@@ -475,6 +531,8 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   // short blocks / co-aligned runs up to 1 KiB: with >= 8-byte words the smem/TMA
   // staged kernel wins (C3 pack 0.78 of copy vs 0.66 word table vs 0.44 warp
   // segments; measured), with 4-byte words the register word kernel does
+  // short blocks in small dense records (C5 particles): whole-record 16-byte loads
+  if (mean < 256.0 && rec_ok && !force) return 6;
   if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return stage_ok && g >= 8 ? 4 : 2;
   if (mean < 128.0 && blk_ok) return 3;
   return 1;
@@ -547,65 +605,40 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
   // SMs a pack/unpack needs, e.g. to leave the rest to a co-running application)
   const char* ms = getenv("DT_MAX_SMS");
   const int sms = ms && atoi(ms) > 0 ? std::min(num_sms(), atoi(ms)) : num_sms();
-  // dense-span pack: short blocks (word kernels) inside small dense 16-byte-aligned records
-  if (!unpack && (kind == 2 || kind == 4) && !E.merged && pos == 0 && P.tsize > 0 && len % P.tsize == 0) {
-    int64_t tg = 16;  // template word size
-    for (size_t b = 0; b < f.bd.size(); b++) tg = std::min(tg, std::min(lowp2((uint64_t)f.bd[b]), lowp2((uint64_t)f.bl[b])));
-    int64_t lg = level_granularity(f);
-    for (int i = 0; i < L.n; i++)
-      if (!L.table[i]) lg = std::min(lg, lowp2((uint64_t)L.stride[i]));
-    int64_t lo_b = INT64_MAX, hi_b = INT64_MIN;
-    for (size_t b = 0; b < f.bd.size(); b++) {
-      lo_b = std::min(lo_b, f.bd[b]);
-      hi_b = std::max(hi_b, f.bd[b] + f.bl[b]);
+  if (kind == 6) {
+    RecGeo R;
+    if (!rec_geometry(f, L, (uint64_t)(uintptr_t)nc, (uint64_t)(uintptr_t)c, pos, len, g, &R)) {
+      set_error("record-span geometry changed between plan and launch");
+      return DT_ERR_ARG;
     }
-    const int64_t a0 = lo_b >= 0 ? lo_b & ~int64_t(15) : -((-lo_b + 15) & ~int64_t(15));
-    const int64_t spanB = ((hi_b - a0) + 15) & ~int64_t(15);
-    // opt-in only: measured slower than the word / staged kernels on C5 (1.22 vs 1.01 ms
-    // pack at 1 GiB) and C3 (78 vs 45 us); kept as kernel family 5 (DT_FORCE_KERNEL=5)
-    const char* fk = getenv("DT_FORCE_KERNEL");
-    const bool no_span = !(fk && atoi(fk) == 5);
-    if (!no_span && tg >= 4 && lg >= 16 && (((uintptr_t)nc) & 15) == 0 && (((uintptr_t)c) & 15) == 0 &&
-        spanB <= 512 && 2 * P.tsize >= spanB && template_fits_int32(f) && P.tsize % tg == 0 &&
-        P.tsize / tg <= kMaxWordTable) {
-      int64_t m = 16;
-      for (int64_t x = P.tsize; m > 1 && x % m; m >>= 1) {
-      }
-      m = 16 / m;  // elements per 16-byte-aligned packed boundary
-      int64_t Ee = std::min<int64_t>(16384 / spanB, 16384 / P.tsize) / m * m;
-      if (Ee >= m) {
-        const int32_t* wt = nullptr;
-        dt_status st = ensure_wtab(f, dd, tg, &wt);
-        if (st != DT_OK) return st;
-        P.wtab = wt;
-        P.nwords = (int32_t)(P.tsize / tg);
-        const int64_t nel = len / P.tsize;
-        const int64_t ntiles = (nel + Ee - 1) / Ee;
-        const size_t smem = (size_t)((P.nwords * 4 + 127) & ~127) +
-                            (size_t)kSpanBufs * (size_t)(Ee * spanB + Ee * P.tsize);
-        static bool attr = false;
-        if (!attr) {
-          cudaFuncSetAttribute(k_span<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-          cudaFuncSetAttribute(k_span<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-          cudaFuncSetAttribute(k_span<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-          attr = true;
-        }
-        int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_span<4>, 256, smem) != cudaSuccess || occ < 1)
-          occ = 1;
-        const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
-        switch (tg) {
-          case 4: k_span<4><<<grid, 256, smem, s>>>(P, ntiles, a0, (int)spanB, (int)Ee, nel); break;
-          case 8: k_span<8><<<grid, 256, smem, s>>>(P, ntiles, a0, (int)spanB, (int)Ee, nel); break;
-          default: k_span<16><<<grid, 256, smem, s>>>(P, ntiles, a0, (int)spanB, (int)Ee, nel); break;
-        }
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return cuda_fail(e, "span kernel launch");
-        return DT_OK;
-      }
+    const int32_t* wt = nullptr;
+    dt_status st = ensure_wtab(f, dd, g, &wt);
+    if (st != DT_OK) return st;
+    P.wtab = wt;
+    P.nwords = R.nwr;
+    const int nwc = 8;
+    const size_t tabB = std::max<size_t>((size_t)R.RB * R.nwr * 2, (size_t)(R.spanB / g) * 2);
+    const size_t smem = (size_t)nwc * R.RB * R.spanB + (size_t)nwc * R.RB * 8 + ((tabB + 15) & ~size_t(15));
+    static bool attr = false;
+    if (!attr) {
+      const void* fs[] = {(const void*)k_rec<false, 4>, (const void*)k_rec<false, 8>, (const void*)k_rec<false, 16>,
+                          (const void*)k_rec<true, 4>,  (const void*)k_rec<true, 8>,  (const void*)k_rec<true, 16>};
+      for (const void* fp : fs) cudaFuncSetAttribute(fp, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024);
+      attr = true;
     }
-  }
-  if (kind == 1) {
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rec<false, 4>, 256, smem) != cudaSuccess || occ < 1)
+      occ = 1;
+    const int64_t need = (R.nbatch + nwc - 1) / nwc;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, need));
+#define LR(U, G) k_rec<U, G><<<grid, 256, smem, s>>>(P, R)
+    if (unpack) {
+      switch (g) { case 4: LR(true, 4); break; case 8: LR(true, 8); break; default: LR(true, 16); break; }
+    } else {
+      switch (g) { case 4: LR(false, 4); break; case 8: LR(false, 8); break; default: LR(false, 16); break; }
+    }
+#undef LR
+  } else if (kind == 1) {
     // exactly one wave of resident CTAs (no tail wave), at least ~4 KiB per warp
     const bool single = P.nblocks == 1;
     const int occ = seg_occupancy(unpack, single);

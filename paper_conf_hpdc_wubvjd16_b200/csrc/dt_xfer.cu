@@ -644,6 +644,7 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   int64_t g = 1;
   // chunk starts are multiples of `chunk` (a multiple of 512) and ring slots are aligned
   int kind = plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
+  if (kind == 6) kind = g >= 8 ? 4 : 2;  // record-span kernel: standalone only (fragments use word gathers)
   if ((kind == 2 || kind == 4) && lowp2u((uint64_t)chunk) < g) kind = 1;
   if (kind == 4 && g < 8) kind = 2;
   X.kind = (kind == 2 || kind == 4) ? kind : 1;  // the block-window kernel (3) is not used inside the pipeline

@@ -104,7 +104,14 @@ def test_plan_selects_kernels():
     k, g = t.plan(1, 0x10000, 0x20000, 0, 1 << 30)
     assert g == 4
     t = dt.from_recipe(c5_particles(56 * 100)[0])
-    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 30) == (2, 4)
+    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 30) == (6, 4)     # dense records: record spans
+    assert t.plan(1, 0x10000, 0x20004, 0, 1 << 30) == (2, 4)     # packed side not 16-B aligned: words
+    assert t.plan(1, 0x10008, 0x20000, 0, 1 << 30) == (2, 4)     # record bases not 16-B aligned: words
+    assert t.plan(1, 0x10000, 0x20000, 32, 4000) == (6, 4)       # 16-B-congruent fragment
+    # sparse records (8 of 32 span bytes) stay on word gathers
+    t = dt.from_recipe(("hvector", 100, 1, 64, ("resized", ("struct", [1, 1], [0, 28], [("basic", "INT32")] * 2),
+                                                0, 64)))
+    assert t.plan(1, 0x10000, 0x20000, 0, 800)[0] == 2
     # byte-granular start position lowers the word size
     assert t.plan(1, 0x10000, 0x20000, 3, 100) == (2, 1)
     # irregular short blocks under a template too large for a word table: window kernel

@@ -170,11 +170,11 @@ def test_random_tiny_types(torch_cuda):
                 raise
 
 
-@pytest.mark.parametrize("kind", ["1", "2", "3", "4", "5"])
+@pytest.mark.parametrize("kind", ["1", "2", "3", "4", "6"])
 @pytest.mark.parametrize("name", ["C1b", "C2s", "C3s", "C4x", "C4y", "C5", "C5b", "ctg"])
 def test_every_kernel_family(torch_cuda, kind, name, monkeypatch):
     """Every kernel family (1 warp segments, 2 word table, 3 block windows, 4 smem/TMA
-    staging) on every workload it accepts, forced through DT_FORCE_KERNEL, with
+    staging, 6 record spans) on every workload it accepts, forced through DT_FORCE_KERNEL, with
     ragged pos/len (the planner falls back when a family does not apply)."""
     mk = {"C1b": lambda: c1_submatrix(256, 1024, 1, 1), "C2s": lambda: c2_lower_triangle(700),
           "C3s": lambda: c3_block_cyclic(1024, 64), "C4x": lambda: c4_face("x+", 96),
@@ -260,3 +260,38 @@ def test_full_size_sampled_c5_large(torch_cuda):
     idx = rec[2][:2000] + 4  # bytes 4..7 of a selected particle are padding: never written
     assert np.all(dst[torch.from_numpy(idx).cuda()].cpu().numpy() == 0xA5)
     del gaps
+
+
+# ------------------------------------------------------------------ record-span kernel (k_rec)
+REC_TYPES = {
+    # C5 particle records (G = 4): blocks (0,4),(8,52) of a 64-byte span
+    "particle": lambda: c5_particles(56 * 3001),
+    # struct{f64@0, f64@16} resized to 32 B, an array of them (G = 8, half payload)
+    "pair8": lambda: (("contiguous", 1500, ("resized", ("struct", [1, 1], [0, 16], [("basic", "DOUBLE")] * 2),
+                                           0, 32)), 0, 1500 * 32),
+    # 16-byte runs at a 48-byte pitch, span 16 (G = 16)
+    "run16": lambda: (("hvector", 2000, 1, 48, ("contiguous", 2, ("basic", "DOUBLE"))), 0, 2000 * 48),
+    # two-level nest of 3-word records (span 16, 12 of 16 bytes), G = 4
+    "nest4": lambda: (("hvector", 37, 1, 16 * 64 + 32, ("hvector", 64, 1, 16, ("contiguous", 3, ("basic", "INT32")))),
+                      0, 37 * (16 * 64 + 32)),
+}
+
+
+@pytest.mark.parametrize("name", sorted(REC_TYPES))
+def test_record_span_kernel(torch_cuda, name):
+    """k_rec is the planner's choice for short blocks in small dense records and is
+    bit-exact for whole streams, counts > 1 and ragged 16-aligned pos / G-granular len
+    (records cut at both ends of a fragment)."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = REC_TYPES[name]()
+    t = dt.from_recipe(rec).commit()
+    assert t.plan(1, 4096, 8192, 0, t.size)[0] == 6
+    size = t.size
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=31)
+    rng = np.random.default_rng(3)
+    for count in (1, 3):
+        total = count * size
+        for _ in range(3):
+            a = int(rng.integers(0, total // 16)) * 16
+            b = int(rng.integers(a // 4, total // 4 + 1)) * 4
+            check_pack_unpack(torch_cuda, rec, org, parent, count=count, pos=a, nbytes=b - a, seed=a)

@@ -20,6 +20,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", default="C1,C1b,C2,C3,C4x,C4y,C4z,C5_64M,C5_1G,C5b_64M,V4K,V8K,V16K,T16K")
     ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--l2fetch", type=int, default=0, help="cudaLimitMaxL2FetchGranularity (bytes) for the run")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -37,6 +38,11 @@ def main():
         "T16K": lambda: W.c2_lower_triangle(16384), "Tstair8K": lambda: W.stair_triangle(8192, 256),
     }
     dev = torch.device("cuda")
+    torch.zeros(1, device=dev)
+    if args.l2fetch:
+        from cuda.bindings import runtime as cudart
+        print(cudart.cudaDeviceSetLimit(cudart.cudaLimit.cudaLimitMaxL2FetchGranularity, args.l2fetch),
+              cudart.cudaDeviceGetLimit(cudart.cudaLimit.cudaLimitMaxL2FetchGranularity), file=sys.stderr)
     l2 = torch.cuda.get_device_properties(dev).L2_cache_size
     flush = torch.empty(2 * l2, dtype=torch.uint8, device=dev)
     flush_rd = torch.zeros(2 * l2 // 4, dtype=torch.int32, device=dev)
