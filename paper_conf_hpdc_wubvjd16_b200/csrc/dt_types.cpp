@@ -162,27 +162,51 @@ dt_status dt_create_vector(int64_t count, int64_t blocklen, int64_t stride, dt_t
   return dt_create_hvector(count, blocklen, stride * old->extent(), old, out);
 }
 
-dt_status dt_create_hindexed(int64_t count, const int64_t* bls, const int64_t* dps, dt_t old, dt_t* out) {
+}  // extern "C"
+
+// hindexed with per-entry blocklens (bls) or one uniform blocklen (bls == nullptr)
+static dt_status create_hindexed(int64_t count, const int64_t* bls, int64_t ubl, const int64_t* dps, dt_t old,
+                                 dt_t* out) {
   CHECK_ARG(old && out, "NULL argument");
   CHECK_ARG(count >= 0, "negative count");
-  CHECK_ARG(count == 0 || (bls && dps), "NULL arrays");
-  for (int64_t i = 0; i < count; i++) CHECK_ARG(bls[i] >= 0, "negative blocklen");
+  CHECK_ARG(count == 0 || dps, "NULL arrays");
+  if (bls) {
+    for (int64_t i = 0; i < count; i++) CHECK_ARG(bls[i] >= 0, "negative blocklen");
+  } else {
+    CHECK_ARG(ubl >= 0, "negative blocklen");
+  }
   auto* t = new dt_type_s;
   t->kind = K_HINDEXED;
   t->count = count;
-  t->bls.assign(bls, bls + count);
+  if (bls) t->bls.assign(bls, bls + count);
+  else t->bls.assign((size_t)count, ubl);
   t->dps.assign(dps, dps + count);
   t->old = retain(old);
+  // every copy is of the same type `old`, so the bounds need only the range of the
+  // shifts over all copies and their number (one pass, no per-entry Bounds update)
   Bounds b;
+  const int64_t e = old->extent();
+  int64_t smin = INT64_MAX, smax = INT64_MIN, ncopies = 0;
   for (int64_t i = 0; i < count; i++) {
-    if (bls[i] == 0) continue;
-    int64_t b0, b1;
-    lin_range(bls[i], old->extent(), b0, b1);
-    b.add(old, dps[i] + b0, dps[i] + b1, bls[i]);
+    const int64_t n = bls ? bls[i] : ubl;
+    if (n == 0) continue;
+    const int64_t last = (n - 1) * e;
+    const int64_t lo = dps[i] + (last < 0 ? last : 0), hi = dps[i] + (last > 0 ? last : 0);
+    smin = lo < smin ? lo : smin;
+    smax = hi > smax ? hi : smax;
+    ncopies += n;
   }
+  if (ncopies > 0) b.add(old, smin, smax, ncopies);
   b.finish(t, false);
   *out = t;
   return DT_OK;
+}
+
+extern "C" {
+
+dt_status dt_create_hindexed(int64_t count, const int64_t* bls, const int64_t* dps, dt_t old, dt_t* out) {
+  CHECK_ARG(count == 0 || bls, "NULL arrays");
+  return create_hindexed(count, bls, 0, dps, old, out);
 }
 
 dt_status dt_create_indexed(int64_t count, const int64_t* bls, const int64_t* d, dt_t old, dt_t* out) {
@@ -197,15 +221,16 @@ dt_status dt_create_indexed(int64_t count, const int64_t* bls, const int64_t* d,
 dt_status dt_create_hindexed_block(int64_t count, int64_t blocklen, const int64_t* dps, dt_t old, dt_t* out) {
   CHECK_ARG(count >= 0 && blocklen >= 0, "negative count/blocklen");
   CHECK_ARG(count == 0 || dps, "NULL arrays");
-  std::vector<int64_t> b(count, blocklen);
-  return dt_create_hindexed(count, b.data(), dps, old, out);
+  return create_hindexed(count, nullptr, blocklen, dps, old, out);
 }
 
 dt_status dt_create_indexed_block(int64_t count, int64_t blocklen, const int64_t* d, dt_t old, dt_t* out) {
   CHECK_ARG(count >= 0 && blocklen >= 0, "negative count/blocklen");
   CHECK_ARG(count == 0 || d, "NULL arrays");
-  std::vector<int64_t> b(count, blocklen);
-  return dt_create_indexed(count, b.data(), d, old, out);
+  CHECK_ARG(old, "NULL argument");
+  std::vector<int64_t> db(d, d + count);
+  for (auto& x : db) x *= old->extent();
+  return create_hindexed(count, nullptr, blocklen, db.data(), old, out);
 }
 
 dt_status dt_create_struct(int64_t count, const int64_t* bls, const int64_t* dps, const dt_t* types, dt_t* out) {
@@ -438,11 +463,18 @@ static int64_t low_pow2(int64_t x) {
   return g > 16 ? 16 : g;
 }
 
+// the lowest set bit of an OR over values is the lowest set bit of any of them
+static int64_t low_pow2_all(const std::vector<int64_t>& v) {
+  uint64_t acc = 0;
+  for (int64_t x : v) acc |= (uint64_t)x;  // (two's complement keeps the low bits of |x|)
+  return low_pow2((int64_t)acc);
+}
+
 int64_t level_granularity(const Form& f) {
   if (f.lvl_gran_cache >= 0) return f.lvl_gran_cache;
   int64_t g = 16;
   for (auto& l : f.lv) {
-    if (l.is_list()) for (auto x : *l.table) g = std::min(g, low_pow2(x));
+    if (l.is_list()) g = std::min(g, low_pow2_all(*l.table));
     else g = std::min(g, low_pow2(l.stride));
   }
   f.lvl_gran_cache = g;
@@ -452,11 +484,8 @@ int64_t level_granularity(const Form& f) {
 int64_t form_granularity(const Form& f) {
   if (f.gran_cache >= 0) return f.gran_cache;
   int64_t g = 16;
-  for (size_t i = 0; i < f.bd.size(); i++) g = std::min(g, std::min(low_pow2(f.bd[i]), low_pow2(f.bl[i])));
-  for (auto& l : f.lv) {
-    if (l.is_list()) for (auto x : *l.table) g = std::min(g, low_pow2(x));
-    else g = std::min(g, low_pow2(l.stride));
-  }
+  g = std::min(g, std::min(low_pow2_all(f.bd), low_pow2_all(f.bl)));
+  g = std::min(g, level_granularity(f));
   f.gran_cache = g;
   return g;
 }
@@ -495,28 +524,37 @@ static Form build_form(const dt_type_s* t) {
       break;
     }
     case K_HINDEXED: {
+      // entries with blocklen 0 contribute nothing; the common case (none) avoids the
+      // filtered copies (a 1 GB index list has ~2e7 entries: first-use cost, f2)
+      const bool all_pos = std::all_of(t->bls.begin(), t->bls.end(), [](int64_t x) { return x > 0; });
       std::vector<int64_t> B, D;
-      for (int64_t i = 0; i < t->count; i++)
-        if (t->bls[i] > 0) { B.push_back(t->bls[i]); D.push_back(t->dps[i]); }
+      if (!all_pos) {
+        for (int64_t i = 0; i < t->count; i++)
+          if (t->bls[i] > 0) { B.push_back(t->bls[i]); D.push_back(t->dps[i]); }
+      }
+      const std::vector<int64_t>& Bv = all_pos ? t->bls : B;
+      const std::vector<int64_t>& Dv = all_pos ? t->dps : D;
       Form sub = build_form(t->old);
       normalize(sub);
-      if (B.empty() || sub.empty()) break;
-      bool uniform = std::all_of(B.begin(), B.end(), [&](int64_t x) { return x == B[0]; });
+      if (Bv.empty() || sub.empty()) break;
+      bool uniform = std::all_of(Bv.begin(), Bv.end(), [&](int64_t x) { return x == Bv[0]; });
       if (uniform) {
         f = sub;
-        prepend_regular(f, B[0], t->old->extent());
-        prepend_list(f, D);
+        prepend_regular(f, Bv[0], t->old->extent());
+        prepend_list(f, Dv);
       } else if (is_simple_run(sub, t->old->extent())) {
         // indexed of a contiguous element: one block per entry (the triangle, C2)
-        for (size_t i = 0; i < B.size(); i++) {
-          f.bd.push_back(D[i] + sub.bd[0]);
-          f.bl.push_back(B[i] * sub.bl[0]);
+        f.bd.resize(Bv.size());
+        f.bl.resize(Bv.size());
+        for (size_t i = 0; i < Bv.size(); i++) {
+          f.bd[i] = Dv[i] + sub.bd[0];
+          f.bl[i] = Bv[i] * sub.bl[0];
         }
       } else {
         int64_t e = t->old->extent();
-        for (size_t i = 0; i < B.size(); i++)
-          for (int64_t j = 0; j < B[i]; j++)
-            if (!append_expanded(f, sub, D[i] + j * e)) throw FlattenError();
+        for (size_t i = 0; i < Bv.size(); i++)
+          for (int64_t j = 0; j < Bv[i]; j++)
+            if (!append_expanded(f, sub, Dv[i] + j * e)) throw FlattenError();
       }
       break;
     }
