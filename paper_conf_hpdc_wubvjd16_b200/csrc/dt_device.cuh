@@ -402,7 +402,7 @@ template <> struct WordT<16> { typedef uint4 T; };
 
 // Threads tid, tid+nthr, ... each handle one VW-byte vector of the packed
 // stream [lo, hi) (G-aligned, G-granular; cb + lo VW-aligned); wt is the
-// template's word table in shared memory.
+// template's word table in shared memory (nullptr for a single-block template).
 // NV vectors per thread and iteration: every load of the batch is issued before
 // the first store, so a thread keeps NV*VW bytes in flight.
 template <bool UNPACK, int G, int VW, int POL, int NV = 2>
@@ -449,7 +449,9 @@ __device__ __forceinline__ void word_range(const KP& P, uint8_t* cb, const int64
 #pragma unroll
       for (int k = 0; k < NW; k++) {
         if (k < nvalid[j]) {
-          W* a = reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed[j] + wt[w[j]]);
+          // (wt == nullptr: single-block template, word k at bd0 + k*G -- no table load)
+          const int64_t wo = wt ? (int64_t)wt[w[j]] : P.bd0 + (int64_t)w[j] * G;
+          W* a = reinterpret_cast<W*>(const_cast<uint8_t*>(P.nc) + ed[j] + wo);
           if (UNPACK) *a = u[j].word[k];
           else u[j].word[k] = ldv<POL>(a);
           if (++w[j] == P.nwords && k + 1 < nvalid[j]) {

@@ -110,6 +110,18 @@ __global__ void __launch_bounds__(256, 3) k_seg(const KP P, const PlanEnt* __res
   seg_walk<UNPACK, SINGLE, LD_CS>(P, P.c - P.pos, a.p, p1, a.b, a.r, a.e, a.ed, lane);
 }
 
+// single-block templates (every block the same length, so cost balance is moot):
+// warp w copies [pos + w*per, ...) resolved arithmetically -- no plan load ahead
+// of the first data load (latency-bound small messages: C1, C4 y/z faces)
+template <bool UNPACK>
+__global__ void __launch_bounds__(256, 3) k_seg_eq(const KP P, int64_t per) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t p = P.pos + gw * per, end = P.pos + P.len;
+  if (p >= end) return;
+  seg_range<UNPACK, true, LD_CS>(P, P.c - P.pos, p, min(p + per, end), lane);
+}
+
 // one thread per warp boundary: cost-balanced cut positions (see PlanEnt)
 __global__ void k_plan(const KP P, int64_t alpha, FastDiv fce, int64_t ce, int64_t C0, int64_t C1, int64_t nw,
                        PlanEnt* plan) {
@@ -227,9 +239,14 @@ __global__ void __launch_bounds__(256, 3) k_rec(const KP P, const RecGeo R) {
 template <bool UNPACK, int G, int VW>
 __global__ void __launch_bounds__(256) k_word(const KP P) {
   extern __shared__ int32_t wt[];
-  for (int i = threadIdx.x; i < P.nwords; i += blockDim.x) wt[i] = P.wtab[i];
-  __syncthreads();
-  word_range<UNPACK, G, VW, LD_CS, (G >= 4 ? 4 : 2)>(P, P.c - P.pos, P.pos, P.pos + P.len, wt,
+  // single-block template: word offsets are arithmetic (no dependent table load
+  // before the first gather -- it matters for latency-bound faces, C4 x)
+  const bool sb = P.nblocks == 1;
+  if (!sb) {
+    for (int i = threadIdx.x; i < P.nwords; i += blockDim.x) wt[i] = P.wtab[i];
+    __syncthreads();
+  }
+  word_range<UNPACK, G, VW, LD_CS, (G >= 4 ? 4 : 2)>(P, P.c - P.pos, P.pos, P.pos + P.len, sb ? nullptr : wt,
                                                      (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
                                                      (int64_t)gridDim.x * blockDim.x);
 }
@@ -638,6 +655,16 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
       switch (g) { case 4: LR(false, 4); break; case 8: LR(false, 8); break; default: LR(false, 16); break; }
     }
 #undef LR
+  } else if (kind == 1 && P.nblocks == 1) {
+    // one wave of resident CTAs, equal 16-byte-multiple slices of >= 1 KiB per warp
+    const int occ = seg_occupancy(unpack, true);
+    const int64_t max_warps = (int64_t)sms * occ * 8;
+    int64_t per = std::max<int64_t>(1024, (len + max_warps - 1) / max_warps);
+    per = (per + 15) & ~int64_t(15);
+    const int64_t nw = (len + per - 1) / per;
+    const unsigned grid = (unsigned)((nw + 7) / 8);
+    if (unpack) k_seg_eq<true><<<grid, 256, 0, s>>>(P, per);
+    else k_seg_eq<false><<<grid, 256, 0, s>>>(P, per);
   } else if (kind == 1) {
     // exactly one wave of resident CTAs (no tail wave), at least ~4 KiB per warp
     const bool single = P.nblocks == 1;
