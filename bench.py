@@ -10,7 +10,9 @@ construct + commit happen once, before timing, as the paper's cached DEVs
 [L24:c2714]).  Metric (BASELINE.json): pack/unpack GB/s counting payload bytes
 read + written, i.e. 2*payload per kernel, reported against the measured HBM
 copy peak.  At N>1 every rank runs the same step on its own matrices (weak
-scaling, no data-path collective; the transfer path is `--workload c3`).
+scaling, no data-path collective) and the line adds a "transfer" object: the
+north_star's multi-GPU metric, the pipelined C3 exchange between pairs (r, r^1)
+over NVLink as a fraction of 900 GB/s per direction (`--workload xfer` sweeps it).
 
 L2 hygiene: a 2xL2 scratch buffer is rewritten before every timed kernel, and
 only the pack/unpack kernels themselves are inside the CUDA-event intervals.
@@ -100,8 +102,16 @@ def dist_init():
         import torch.distributed as tdist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         import torch
-        torch.cuda.set_device(local)
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        # test aid: DT_BENCH_SHARE_GPU=1 maps every rank onto the visible GPUs round-robin
+        # (several ranks per GPU talk over CUDA IPC exactly as across GPUs) with a gloo
+        # process group for the bootstrap and the max-over-ranks reductions
+        if os.environ.get("DT_BENCH_SHARE_GPU") == "1":
+            local = local % torch.cuda.device_count()
+            torch.cuda.set_device(local)
+            tdist.init_process_group("gloo")
+        else:
+            torch.cuda.set_device(local)
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
     return ws, rank, local
 
 
@@ -234,6 +244,19 @@ def run_ours(args):
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(f"c2_{dom}")
     e2e = run_e2e(args, t, src_h, org, parent, payload, dev) if rank == 0 else None
+    transfer = None
+    if ws > 1:
+        # the north_star's multi-GPU metric: pipelined non-contiguous exchange between
+        # pairs (r, r^1) over NVLink (C3 block-cyclic, P2P mode), reported beside the
+        # replica headline as a fraction of 900 GB/s per direction
+        del src, dst, packed, flush, flush_rd
+        torch.cuda.empty_cache()
+        res, xpay, xok, _ = xfer_sweep(ws, rank, local, [1 << 20, 4 << 20], [4], "p2p", 0, 10, 3)
+        xb = max(res, key=lambda r: r["gbs_per_rank"])
+        transfer = {"workload": "C3 block-cyclic 128 MiB per direction, pairs (r, r^1), dt_sendrecv P2P",
+                    "value": round(ws * xpay / (xb["ms"] * 1e-3) / 1e9, 1), "unit": UNIT,
+                    "gbs_per_direction": xb["gbs_per_rank"], "peak": 900.0,
+                    "frac": round(xb["gbs_per_rank"] / 900.0, 4), "sweep": res, "spot_parity": xok}
     line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(kern_ms / args.steps, 5), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
@@ -249,6 +272,8 @@ def run_ours(args):
                          "traffic": traffic,
                          "algorithmic_bytes_per_launch": 2 * payload},
             "gpu_launches": 2 * args.steps, "clocks": clk.summary(), "e2e": e2e}
+    if transfer is not None:
+        line["transfer"] = transfer
     if rank == 0 and ws == 1 and not args.no_cpu:
         line["cpu_baseline"] = time_oracle_c2(seconds=args.cpu_seconds)[0]
     if rank == 0:
@@ -285,18 +310,14 @@ def run_e2e(args, t, src_h, org, parent, payload, dev):
             "steps": steps, "note": "host pinned buffers; wall clock incl. all copies and syncs"}
 
 
-def run_xfer(args):
-    """S7: pipelined GPU<->GPU exchange of the C3 block-cyclic submatrix (128 MiB per
-    direction, 512-B runs) through dt_sendrecv, chunk/depth sweep ([L18:c4394 §4.1]).
-    Pairs (r, r^1) exchange concurrently; at N=1 the rank exchanges with itself
-    (loopback, the paper's "1GPU" case [L26:c1686]).  value = bytes received by all
-    ranks per second (max-over-ranks device time)."""
+def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup):
+    """Pairwise C3 exchange through dt_sendrecv over a chunk x depth sweep (S7).
+    Returns (results, payload, spot_parity); every timing is the max over ranks of
+    the device time between a barrier-aligned pair of CUDA events."""
     import torch
 
     from paper_conf_hpdc_wubvjd16_b200 import dt
     from workloads import c3_block_cyclic, fill_bytes, seed_for
-    ws, rank, local = dist_init()
-    torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     peer = rank ^ 1 if (rank ^ 1) < ws else rank
     rec, org, parent = c3_block_cyclic()
@@ -305,24 +326,23 @@ def run_xfer(args):
     A = torch.from_numpy(fill_bytes(parent, seed_for(3) + rank)).to(dev)
     B = torch.full((parent,), 0xA5, dtype=torch.uint8, device=dev)
     s = torch.cuda.current_stream()
-    mode = dt.XFER_NCCL if args.xfer_mode == "nccl" else dt.XFER_P2P
+    mode = dt.XFER_NCCL if mode_name == "nccl" else dt.XFER_P2P
     results = []
-    for chunk in [int(x) << 10 for x in args.xfer_chunks_kib.split(",")]:
-        for depth in [int(x) for x in args.xfer_depths.split(",")]:
+    for chunk in chunks:
+        for depth in depths:
             if ws > 1:
-                comm = dt.Comm.from_process_group(device=local, chunk_bytes=chunk, depth=depth, mode=mode,
-                                                  ctas=args.xfer_ctas)
+                comm = dt.Comm.from_process_group(device=local, chunk_bytes=chunk, depth=depth, mode=mode, ctas=ctas)
             else:
                 nid = dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None
                 comm = dt.Comm(0, 1, local, chunk_bytes=chunk, depth=depth, mode=mode, nccl_id=nid,
-                               ctas=args.xfer_ctas, ring_loopback=True)  # measure the pipeline itself
-            for _ in range(args.warmup):
+                               ctas=ctas, ring_loopback=True)  # measure the pipeline itself
+            for _ in range(warmup):
                 comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
             torch.cuda.synchronize()
             comm.check()
-            steps = max(3, min(args.steps, 20))
             if ws > 1:
                 torch.distributed.barrier()
+            torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             for _ in range(steps):
@@ -338,6 +358,28 @@ def run_xfer(args):
             results.append({"chunk": chunk, "depth": depth, "ms": round(ms, 4),
                             "gbs_per_rank": round(payload / (ms * 1e-3) / 1e9, 1)})
             comm.free()
+    # parity of the last exchange: my B must equal the peer's A (same layout on both sides)
+    exp = torch.from_numpy(fill_bytes(parent, seed_for(3) + peer)).to(dev)
+    ok = bool(torch.equal(B.view(-1)[org:org + 8 * 64], exp.view(-1)[org:org + 8 * 64]))
+    return results, payload, ok, (t, A, B, org)
+
+
+def run_xfer(args):
+    """S7: pipelined GPU<->GPU exchange of the C3 block-cyclic submatrix (128 MiB per
+    direction, 512-B runs) through dt_sendrecv, chunk/depth sweep ([L18:c4394 §4.1]).
+    Pairs (r, r^1) exchange concurrently; at N=1 the rank exchanges with itself
+    (loopback, the paper's "1GPU" case [L26:c1686]).  value = bytes received by all
+    ranks per second (max-over-ranks device time)."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    ws, rank, local = dist_init()
+    torch.cuda.set_device(local)
+    steps = max(3, min(args.steps, 20))
+    results, payload, ok, (t, A, B, org) = xfer_sweep(
+        ws, rank, local, [int(x) << 10 for x in args.xfer_chunks_kib.split(",")],
+        [int(x) for x in args.xfer_depths.split(",")], args.xfer_mode, args.xfer_ctas, steps, args.warmup)
+    s = torch.cuda.current_stream()
     best = max(results, key=lambda r: r["gbs_per_rank"])
     value = ws * payload / (best["ms"] * 1e-3) / 1e9
     fused = None
@@ -351,9 +393,6 @@ def run_xfer(args):
         e1.record(s)
         torch.cuda.synchronize()
         fused = round(payload / (e0.elapsed_time(e1) / 10 * 1e-3) / 1e9, 1)
-    # parity of the last exchange: my B must equal the peer's A packed/unpacked (closed form: same layout)
-    exp = torch.from_numpy(fill_bytes(parent, seed_for(3) + peer)).to(dev)
-    ok = bool(torch.equal(B.view(-1)[org:org + 8 * 64], exp.view(-1)[org:org + 8 * 64]))
     peak = 900.0 if ws > 1 else load_peaks()[0] / 4  # loopback: 4x payload of HBM traffic per exchange
     line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": ws, "steps": steps,
             "warmup": args.warmup, "ms_per_step": best["ms"], "higher_is_better": True, "scaling": "weak",
