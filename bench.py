@@ -476,10 +476,148 @@ def run_halo(args):
         torch.distributed.destroy_process_group()
 
 
+def sweep_configs(which):
+    """The SURVEY §8(d) 1-GPU table: C1 (+ misaligned), C2, C3, C4 faces, the C5
+    particle sweep 1 KiB..1 GiB (x4 steps), C5b, the V sweep (lda = 2N, reading A3),
+    the T sweep and the stair triangle (reading A4)."""
+    import workloads as W
+    cf = {"C1": lambda: W.c1_submatrix(), "C1b": lambda: W.c1_submatrix(r0=1, c0=1),
+          "C2": lambda: W.c2_lower_triangle(), "C3": lambda: W.c3_block_cyclic(),
+          "C4x": lambda: W.c4_face("x-"), "C4y": lambda: W.c4_face("y-"), "C4z": lambda: W.c4_face("z-"),
+          "C5b_64M": lambda: W.c5b_irregular(64 << 20), "Tstair8K": lambda: W.stair_triangle(8192, 256)}
+    for k in range(11):
+        m = 1 << (10 + 2 * k)
+        cf[f"C5_{m >> 10}K"] = (lambda m=m: W.c5_particles(m))
+    for n in (1024, 2048, 4096, 8192, 16384):
+        cf[f"V{n >> 10}K"] = (lambda n=n: W.c1_submatrix(n, 2 * n))
+        cf[f"T{n >> 10}K"] = (lambda n=n: W.c2_lower_triangle(n))
+    if which == "all":
+        return cf
+    return {k: cf[k] for k in which.split(",")}
+
+
+def sector_bytes(t, count=1):
+    """32-byte DRAM sectors the layout touches (x 32 B): the read floor of a pack
+    (SURVEY §8(d) "sector-aware" fraction).  Host-only flatten of the committed type."""
+    import numpy as np
+    d, ln = t.flatten(count)
+    d, ln = np.asarray(d), np.asarray(ln)
+    o = np.argsort(d, kind="stable")
+    a, b = d[o] // 32, (d[o] + ln[o] - 1) // 32
+    prev = np.maximum.accumulate(np.concatenate([[-1], b[:-1]]))
+    a = np.maximum(a, prev + 1)
+    return int(np.sum(np.maximum(0, b - a + 1))) * 32
+
+
+def run_sweep(args):
+    """`--workload sweep`: one JSON row per SURVEY §8(d) config on one GPU (not the
+    driver's headline line): pack/unpack event-timed after an L2 flush, CUDA-graph
+    replay per call (L2-resident) for small payloads, a same-run contiguous copy,
+    the sector-aware fraction, and the CPU oracle as it stands (single thread and
+    all host cores) on a bounded prefix sample of the same stream."""
+    import numpy as np
+    import torch
+
+    import oracle
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(0)
+    peak = load_peaks()[0]
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    flush = torch.empty(2 * l2, dtype=torch.uint8, device=dev)
+    flush_rd = torch.zeros(2 * l2 // 4, dtype=torch.int32, device=dev)
+    s = torch.cuda.current_stream()
+    cores = len(os.sched_getaffinity(0))
+
+    def timeit(fn, reps):
+        ts = []
+        for i in range(reps + 3):
+            flush.fill_(i & 0xFF)
+            flush_rd.sum()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            fn()
+            e1.record(s)
+            torch.cuda.synchronize()
+            if i >= 3:
+                ts.append(e0.elapsed_time(e1))
+        return statistics.median(ts)
+
+    def graph_us(fn, n=1000):
+        g, gs = torch.cuda.CUDAGraph(), torch.cuda.Stream()
+        fn(gs)  # plans / word tables are created outside the capture
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=gs):
+            for _ in range(n):
+                fn(gs)
+        g.replay()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        g.replay()
+        e1.record(s)
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) * 1e3 / n
+
+    for name, mk in sweep_configs(args.sweep).items():
+        rec, org, parent = mk()
+        t = dt.from_recipe(rec)
+        c0 = time.perf_counter()
+        t.commit()
+        commit_ms = (time.perf_counter() - c0) * 1e3
+        n = t.size
+        src = torch.empty(parent, dtype=torch.uint8, device=dev)
+        src.view(-1)[: parent // 4 * 4].view(torch.int32).random_()
+        pk = torch.empty(n, dtype=torch.uint8, device=dev)
+        dst = torch.full((parent,), 0xA5, dtype=torch.uint8, device=dev)
+        a = torch.empty(n, dtype=torch.uint8, device=dev)
+        b = torch.empty(n, dtype=torch.uint8, device=dev)
+        reps = 20 if n < (256 << 20) else 7
+        pack = lambda st=None: dt.pack(t, 1, src, pk, origin_offset=org, stream=st or s)  # noqa: E731
+        unpack = lambda st=None: dt.unpack(t, 1, pk, dst, origin_offset=org, stream=st or s)  # noqa: E731
+        tp, tu, tc = timeit(pack, reps), timeit(unpack, reps), timeit(lambda: b.copy_(a), reps)
+        kind, gran = t.plan(1, src.data_ptr() + org, pk.data_ptr(), 0, n)
+        gbs = lambda ms: round(2 * n / (ms * 1e-3) / 1e9, 1)  # noqa: E731
+        row = {"config": name, "payload": n, "kernel": kind, "gran": gran, "commit_ms": round(commit_ms, 2),
+               "pack_us": round(tp * 1e3, 2), "unpack_us": round(tu * 1e3, 2), "copy_us": round(tc * 1e3, 2),
+               "pack_gbs": gbs(tp), "unpack_gbs": gbs(tu), "copy_gbs": gbs(tc),
+               "pack_frac_hbm": round(gbs(tp) / peak, 3), "unpack_frac_hbm": round(gbs(tu) / peak, 3),
+               "pack_vs_copy": round(tc / tp, 3), "unpack_vs_copy": round(tc / tu, 3)}
+        if n <= (4 << 20):  # latency-bound sizes: per-call device time amortised over 1000 graph-replayed calls
+            row["graph_pack_us"] = round(graph_us(pack), 3)
+            row["graph_unpack_us"] = round(graph_us(unpack), 3)
+            row["graph_note"] = "1000 calls in one CUDA graph, L2-resident (no flush)"
+        if n <= (1 << 28):
+            sb = sector_bytes(t)
+            row["sector_read_bytes"] = sb
+            row["pack_sector_aware_frac"] = round((sb + n) / (tp * 1e-3) / 1e9 / peak, 3)
+        # CPU oracle as it stands, on a prefix of the same stream (bounded ~1 s per leg)
+        ot = oracle.from_recipe(rec)
+        host = np.empty(parent, dtype=np.uint8)
+        host[: min(parent, 1 << 30)] = 0x5A
+        for label, th in (("oracle_1t", 1), ("oracle_mt", cores)):
+            m = min(n, 1 << 20)
+            while True:
+                c0 = time.perf_counter()
+                out = oracle.pack(ot, 1, host, org, 0, m, threads=th)
+                oracle.unpack(ot, 1, out, host, org, 0, threads=th)
+                el = time.perf_counter() - c0
+                if el > 0.5 or m >= n:
+                    break
+                m = min(n, 4 * m)
+            row[label + "_gbs"] = round(4 * m / el / 1e9, 3)
+            row[label + "_sample_bytes"] = m
+        row["oracle_cores"] = cores
+        print(json.dumps(row), flush=True)
+        del src, pk, dst, a, b, host
+        torch.cuda.empty_cache()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--workload", default="c2", choices=["c2", "xfer", "halo"])
+    ap.add_argument("--workload", default="c2", choices=["c2", "xfer", "halo", "sweep"])
+    ap.add_argument("--sweep", default="all", help="--workload sweep: comma-separated config names or 'all'")
     ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl"])
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
     ap.add_argument("--xfer-depths", default="2,4")
@@ -499,6 +637,8 @@ def main():
         run_xfer(args)
     elif args.workload == "halo":
         run_halo(args)
+    elif args.workload == "sweep":
+        run_sweep(args)
     else:
         run_ours(args)
 
