@@ -328,6 +328,8 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup):
     s = torch.cuda.current_stream()
     mode = dt.XFER_NCCL if mode_name == "nccl" else dt.XFER_P2P
     results = []
+    if mode_name == "direct":  # persistent direct plan: chunk and depth do not apply
+        chunks, depths = [0], [0]
     for chunk in chunks:
         for depth in depths:
             if ws > 1:
@@ -336,20 +338,28 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup):
                 nid = dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None
                 comm = dt.Comm(0, 1, local, chunk_bytes=chunk, depth=depth, mode=mode, nccl_id=nid,
                                ctas=ctas, ring_loopback=True)  # measure the pipeline itself
+            if mode_name == "direct":
+                ops = ([(A.data_ptr() + org, 1, t, peer, 0)], [(B.data_ptr() + org, 1, t, peer, 0)])
+                xp = dt.XPlan.from_process_group(comm, *ops) if ws > 1 else dt.XPlan.local(comm, *ops)
+                one = lambda: xp.start(s)  # noqa: E731
+                chk = xp.check
+            else:
+                one = lambda: comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)  # noqa
+                chk = comm.check
             for _ in range(warmup):
-                comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
+                one()
             torch.cuda.synchronize()
-            comm.check()
+            chk()
             if ws > 1:
                 torch.distributed.barrier()
             torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             for _ in range(steps):
-                comm.sendrecv(A, 1, t, peer, B, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
+                one()
             e1.record(s)
             torch.cuda.synchronize()
-            comm.check()
+            chk()
             ms = e0.elapsed_time(e1) / steps
             if ws > 1:
                 x = torch.tensor([ms], dtype=torch.float64, device=dev)
@@ -357,6 +367,8 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup):
                 ms = float(x[0])
             results.append({"chunk": chunk, "depth": depth, "ms": round(ms, 4),
                             "gbs_per_rank": round(payload / (ms * 1e-3) / 1e9, 1)})
+            if mode_name == "direct":
+                xp.free()
             comm.free()
     # parity of the last exchange: my B must equal the peer's A (same layout on both sides)
     exp = torch.from_numpy(fill_bytes(parent, seed_for(3) + peer)).to(dev)
@@ -393,7 +405,9 @@ def run_xfer(args):
         e1.record(s)
         torch.cuda.synchronize()
         fused = round(payload / (e0.elapsed_time(e1) / 10 * 1e-3) / 1e9, 1)
-    peak = 900.0 if ws > 1 else load_peaks()[0] / 4  # loopback: 4x payload of HBM traffic per exchange
+    # loopback through the ring moves 4x payload through HBM (pack R+W, unpack R+W); a direct
+    # plan (and the fused copy) moves 2x (read once, written once)
+    peak = 900.0 if ws > 1 else load_peaks()[0] / (2 if args.xfer_mode == "direct" else 4)
     line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": ws, "steps": steps,
             "warmup": args.warmup, "ms_per_step": best["ms"], "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
@@ -405,7 +419,7 @@ def run_xfer(args):
             "roofline": {"bound": "nvlink" if ws > 1 else "hbm", "achieved": best["gbs_per_rank"],
                          "peak": peak, "unit": "GB/s", "frac": round(best["gbs_per_rank"] / peak, 4),
                          "note": "per-direction NVLink 900 GB/s nominal" if ws > 1 else
-                                 "loopback moves 4x payload through HBM (pack R+W, unpack R+W)"},
+                                 "loopback: HBM peak / (2 direct, 4 ring) bytes moved per payload byte"},
             "gpu_launches": steps}
     if rank == 0:
         print(json.dumps(line), flush=True)
@@ -437,10 +451,17 @@ def run_halo(args):
     comm = dt.Comm.from_process_group(device=local, **kw) if ws > 1 else \
         dt.Comm(0, 1, local, nccl_id=dt.Comm.nccl_unique_id() if mode == dt.XFER_NCCL else None, **kw)
     s = torch.cuda.current_stream()
+    if args.xfer_mode == "direct":  # one persistent direct plan: one kernel per exchange
+        xp = plan.direct_plan(comm, buf, single_rank=ws == 1)
+        exchange = lambda: xp.start(s)  # noqa: E731
+        check = xp.check
+    else:
+        exchange = lambda: plan.exchange(comm, buf, stream=s)  # noqa: E731
+        check = comm.check
     for _ in range(args.warmup):
-        plan.exchange(comm, buf, stream=s)
+        exchange()
     torch.cuda.synchronize()
-    comm.check()
+    check()
     ok = None
     if ws == 1:
         A = buf.view(torch.int32).view(L, L, L)
@@ -452,10 +473,10 @@ def run_halo(args):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(s)
     for _ in range(steps):
-        plan.exchange(comm, buf, stream=s)
+        exchange()
     e1.record(s)
     torch.cuda.synchronize()
-    comm.check()
+    check()
     ms = e0.elapsed_time(e1) / steps
     if ws > 1:
         x = torch.tensor([ms], dtype=torch.float64, device=dev)
@@ -618,7 +639,8 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--workload", default="c2", choices=["c2", "xfer", "halo", "sweep"])
     ap.add_argument("--sweep", default="all", help="--workload sweep: comma-separated config names or 'all'")
-    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl"])
+    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "direct"],
+                    help="p2p ring pipeline, NCCL double buffering, or a persistent direct plan (dt_xplan)")
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
     ap.add_argument("--xfer-depths", default="2,4")
     ap.add_argument("--xfer-ctas", type=int, default=0, help="CTAs per direction (0 = library default)")

@@ -156,6 +156,16 @@ dt_status dt_flatten(dt_t t, int64_t count, int64_t* disps, int64_t* lens, int64
 dt_status dt_plan(dt_t t, int64_t count, uint64_t origin_addr, uint64_t packed_addr, int64_t pos, int64_t len,
                   int* kernel, int64_t* granularity);
 
+/* Ship a layout to another rank: the flattened form (levels + block template +
+ * index tables, native byte order: homogeneous GPUs, reading A5) and the bounds.
+ * dt_type_serialize: out == NULL -> *nbytes = required size; else writes up to
+ * *nbytes (DT_ERR_ARG if too small).  dt_type_deserialize: a new uncommitted
+ * handle (one reference) whose typemap equals the serialized type's; it has no
+ * constructor tree but can be committed, packed and used as a component.
+ * Host only.  Errors: DT_ERR_ARG (NULL, malformed blob), DT_ERR_NOMEM. */
+dt_status dt_type_serialize(dt_t t, void* out, size_t* nbytes);
+dt_status dt_type_deserialize(const void* in, size_t nbytes, dt_t* out);
+
 /* ------------------------------------------------------------------ GPU <-> GPU transfer */
 enum { DT_XFER_P2P = 0, DT_XFER_NCCL = 1 };
 typedef struct {
@@ -202,6 +212,49 @@ dt_status dt_group_end(dt_comm_t c, void* stream);
 /* Poll/return the sticky device-side error flag (timeouts, truncation). */
 dt_status dt_comm_check(dt_comm_t c);
 dt_status dt_comm_free(dt_comm_t* c);
+
+/* ------------------------------------------------------------------ persistent direct exchange
+ * SURVEY §8(f) f1 across GPUs: the datatype -> datatype copy of dt_copy, with
+ * the destination in the PEER's memory.  A plan is a fixed set of sends and
+ * receives (an MPI persistent request set: the C4 halo's 6 + 6 faces); once
+ * connected, every dt_xplan_start is ONE kernel per rank that
+ *   1. posts this rank's receive buffers (release-stores "ready" = seq into each
+ *      source's flag page over NVLink),
+ *   2. copies every send straight from the local layout into the receiver's
+ *      layout in peer HBM (the receiver's flattened type was shipped at connect;
+ *      no ring, no packed intermediate, no receiver-side unpack: each byte is
+ *      read once and written once), after the receiver posted it,
+ *   3. publishes "done" = seq to each receiver (system-scope fence first) and
+ *      waits until all of this rank's receives are done,
+ * so the stream order after dt_xplan_start sees the received data.  The paper's
+ * pipeline exists to overlap pack / transfer / unpack ([L18:c4932 §4.1]); here
+ * all three are one pass over NVLink peer memory.
+ * Matching: send (dest d, tag t) of rank r <-> receive (source r, tag t) of d.
+ * Truncation (send bytes > receive capacity) is DT_ERR_TRUNCATE at connect,
+ * before any byte moves; an overlapping receive typemap is DT_ERR_OVERLAP.
+ * Every rank must start its plan the same number of times (collective);
+ * waits are bounded (DT_TIMEOUT_MS) and reported by dt_xplan_check. */
+typedef struct dt_xplan_s* dt_xplan_t;
+typedef struct {
+  void* buf;      /* D: origin of the layout (send: read; receive: written)          */
+  int64_t count;  /* instances of type                                              */
+  dt_t type;      /* committed type                                                 */
+  int32_t peer;   /* destination (send) / source (receive) rank; may be this rank   */
+  int32_t tag;    /* matching key of a (sender, receiver) pair                       */
+} dt_xop;
+/* Local part (allocates the flag page on the comm's device). nsend, nrecv <= 16. */
+dt_status dt_xplan_create(dt_comm_t c, int nsend, const dt_xop* sends, int nrecv, const dt_xop* recvs,
+                          dt_xplan_t* out);
+/* What this rank exports to its peers (IPC handles of the receive buffers and of
+ * the flag page, serialized receive types); out == NULL -> *nbytes = size. */
+dt_status dt_xplan_local_blob(dt_xplan_t p, void* out, size_t* nbytes);
+/* blobs: every rank's blob concatenated in rank order (H), sizes[r] bytes each.
+ * Maps peers' buffers once (cudaIpcOpenMemHandle, cached per comm), commits the
+ * receivers' types on this device and builds the launch. */
+dt_status dt_xplan_connect(dt_xplan_t p, const void* blobs, const size_t* sizes);
+dt_status dt_xplan_start(dt_xplan_t p, void* stream);
+dt_status dt_xplan_check(dt_xplan_t p);  /* sticky device-side error (timeout) */
+dt_status dt_xplan_free(dt_xplan_t* p);
 
 const char* dt_last_error(void);
 const char* dt_version(void);

@@ -16,7 +16,7 @@ LIBDIR = os.path.join(HERE, "lib")
 LIB = os.path.join(LIBDIR, "libdt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["dt_types.cpp", "dt_kernels.cu", "dt_xfer.cu"]
+SOURCES = ["dt_types.cpp", "dt_kernels.cu", "dt_xfer.cu", "dt_direct.cu"]
 
 
 def _sources():

@@ -909,6 +909,8 @@ struct RecGeo {
   int32_t invnch;      // ceil(2^16 / nch): idx / nch = (idx * invnch) >> 16 for idx < 4096
   int64_t e_lo, e_hi;  // elements touching [pos, pos+len)
   int64_t b0, nbatch;  // first batch element (multiple of 32) and number of batches
+  uint8_t woff[32];    // span word (G bytes) of packed word k of a record: in the kernel
+                       // parameters, so no table load precedes the first gather
 };
 constexpr int kRecMaxLPL = 8;
 
@@ -1020,5 +1022,51 @@ __device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, c
   }
   __syncwarp();
 }
+
+// ---------------------------------------------------------------- system-scope flags
+// (cross-GPU signalling over NVLink peer memory: transfer rings and direct plans)
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_sys_add(uint64_t* p, uint64_t v) {
+  asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+enum { XERR_TIMEOUT = 1, XERR_TRUNCATE = 2 };
+
+// spin until pred(*p) holds; false on timeout (sets *err)
+template <typename Pred>
+__device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeout_ns, int32_t* err, uint64_t* out,
+                                     bool sleep = true) {
+  uint64_t v = ld_acquire_sys(p);
+  if (pred(v)) { *out = v; return true; }
+  const uint64_t t0 = gtimer();
+  int ns = 32;
+  while (true) {
+    if (sleep) __nanosleep(ns);
+    if (ns < 256) ns <<= 1;
+    v = ld_acquire_sys(p);
+    if (pred(v)) { *out = v; return true; }
+    if ((int64_t)(gtimer() - t0) > timeout_ns) {
+      atomicCAS(err, 0, XERR_TIMEOUT);
+      return false;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- host helpers (dt_kernels.cu)
+dt_status dual_params(dt_type_s* st, int64_t scount, const void* src, dt_type_s* rt, int64_t rcount, void* dst,
+                      int64_t n, KP& S, KP& R, int* kind, int64_t* gran);
+int nonoverlap_cached(dt_type_s* rt, int64_t rcount);
 
 }  // namespace dt

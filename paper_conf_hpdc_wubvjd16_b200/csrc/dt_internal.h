@@ -103,7 +103,9 @@ struct DeviceDesc {
   size_t plan_next = 0;
 };
 
-enum Kind { K_BASIC, K_CONTIG, K_HVECTOR, K_HINDEXED, K_STRUCT, K_SUBARRAY, K_RESIZED };
+enum Kind { K_BASIC, K_CONTIG, K_HVECTOR, K_HINDEXED, K_STRUCT, K_SUBARRAY, K_RESIZED, K_FLAT };
+// K_FLAT: a type rebuilt from its serialized flattened form (dt_type_deserialize);
+// its Form is stored at creation and it has no constructor tree.
 
 }  // namespace dt
 
@@ -149,5 +151,7 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
 void build_levels(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count, KLevels& L);
 dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out);
 const Form& get_form(dt_type_s* t);
+// xfer.cu: identity of a communicator (direct exchange plans live beside it)
+void comm_info(dt_comm_t c, int* rank, int* nranks, int* device);
 dt_status ensure_wtab_pub(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out);
 }  // namespace dt

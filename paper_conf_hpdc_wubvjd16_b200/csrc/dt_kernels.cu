@@ -215,12 +215,12 @@ __global__ void __launch_bounds__(256, 3) k_rec(const KP P, const RecGeo R) {
     const int n = R.RB * R.nwr;
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
       const int r = i / R.nwr, k = i - r * R.nwr;
-      omap[i] = (uint16_t)(r * R.spanB + (int)(P.wtab[k] - R.a0));
+      omap[i] = (uint16_t)(r * R.spanB + G * (int)R.woff[k]);
     }
   } else {
     for (int i = threadIdx.x; i < R.spanB / G; i += blockDim.x) umap[i] = -1;
     __syncthreads();
-    for (int k = threadIdx.x; k < R.nwr; k += blockDim.x) umap[(int)(P.wtab[k] - R.a0) / G] = (int16_t)k;
+    for (int k = threadIdx.x; k < R.nwr; k += blockDim.x) umap[R.woff[k]] = (int16_t)k;
   }
   __syncthreads();
   const int64_t nwt = (int64_t)gridDim.x * nwc;
@@ -516,6 +516,10 @@ static bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint
   R->e_hi = (pos + len + ts - 1) / ts;
   R->b0 = R->e_lo & ~int64_t(31);
   R->nbatch = (R->e_hi - R->b0 + R->RB - 1) / R->RB;
+  if (R->nwr > 32) return false;
+  int k = 0;
+  for (size_t b = 0; b < f.bd.size(); b++)
+    for (int64_t o = 0; o < f.bl[b]; o += g) R->woff[k++] = (uint8_t)((f.bd[b] + o - a0) / g);
   return true;
 }
 
@@ -628,10 +632,6 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
       set_error("record-span geometry changed between plan and launch");
       return DT_ERR_ARG;
     }
-    const int32_t* wt = nullptr;
-    dt_status st = ensure_wtab(f, dd, g, &wt);
-    if (st != DT_OK) return st;
-    P.wtab = wt;
     P.nwords = R.nwr;
     const int nwc = 8;
     const size_t tabB = std::max<size_t>((size_t)R.RB * R.nwr * 2, (size_t)(R.spanB / g) * 2);
@@ -958,6 +958,66 @@ static dt_status make_kp(dt_type_s* t, int64_t count, const void* nc, int64_t n,
   return DT_OK;
 }
 
+}  // extern "C"
+
+// receive-side legality: the destination typemap must not overlap (cached per count)
+int dt::nonoverlap_cached(dt_type_s* rt, int64_t rcount) {
+  const Form& fr = get_form(rt);
+  std::lock_guard<std::mutex> g(rt->mu);
+  if (rt->ovl_count != rcount) {
+    rt->ovl_result = check_nonoverlap(rt, fr, rcount);
+    rt->ovl_count = rcount;
+  }
+  return rt->ovl_result;
+}
+
+// Parameters of a fused type -> type copy of n stream bytes from (st, scount, src)
+// to (rt, rcount, dst) and its kernel family, as dt_copy launches it: 1 dual block
+// walk (long runs), 2 dual word tables, 4 smem-staged (cp.async gather by the
+// source layout, scatter by the destination layout).  Word tables are attached.
+dt_status dt::dual_params(dt_type_s* st, int64_t scount, const void* src, dt_type_s* rt, int64_t rcount, void* dst,
+                      int64_t n, KP& S, KP& R, int* kind, int64_t* gran) {
+  const Form *fs, *fr;
+  DeviceDesc *ds, *dr;
+  dt_status s1 = make_kp(st, scount, src, n, S, &fs, &ds);
+  if (s1 != DT_OK) return s1;
+  s1 = make_kp(rt, rcount, dst, n, R, &fr, &dr);
+  if (s1 != DT_OK) return s1;
+  KLevels Ls, Lr;
+  build_levels(*fs, ds, st, scount, Ls);
+  build_levels(*fr, dr, rt, rcount, Lr);
+  int64_t gs = 1, gr = 1;
+  plan_kernel(*fs, Ls, (uint64_t)(uintptr_t)src, 0, 0, n, &gs);
+  plan_kernel(*fr, Lr, (uint64_t)(uintptr_t)dst, 0, 0, n, &gr);
+  const int64_t g = std::min(gs, gr);
+  const double ms = (double)S.tsize / (double)S.nblocks, mr = (double)R.tsize / (double)R.nblocks;
+  const bool words_ok = S.tsize % g == 0 && R.tsize % g == 0 && (S.tsize + R.tsize) / g <= kMaxWordTable &&
+                        template_fits_int32(*fs) && template_fits_int32(*fr);
+  const char* fk = getenv("DT_FORCE_KERNEL");
+  const int force = fk ? atoi(fk) : 0;
+  const double mm = std::min(ms, mr);
+  const bool use_words = words_ok && force != 1 && (force == 2 || mm < 256.0 || (g == 16 && mm < 1024.0));
+  *gran = g;
+  if (!use_words) {
+    *kind = 1;
+    return DT_OK;
+  }
+  const int32_t *wa = nullptr, *wb = nullptr;
+  s1 = ensure_wtab(*fs, *ds, g, &wa);
+  if (s1 != DT_OK) return s1;
+  s1 = ensure_wtab(*fr, *dr, g, &wb);
+  if (s1 != DT_OK) return s1;
+  S.wtab = wa;
+  S.nwords = (int32_t)(S.tsize / g);
+  R.wtab = wb;
+  R.nwords = (int32_t)(R.tsize / g);
+  // staged for >= 8-byte words (DT_FORCE_KERNEL=2 keeps the register word kernel)
+  *kind = (g >= 8 && force != 2) ? 4 : 2;
+  return DT_OK;
+}
+
+extern "C" {
+
 static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, int64_t rcount, void* dst,
                             void* stream) {
   if (!st || !rt || scount < 0 || rcount < 0) {
@@ -985,71 +1045,35 @@ static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, i
     s1 = check_dev_ptr((const uint8_t*)dst + rt->true_lb, "destination");
     if (s1 != DT_OK) return s1;
   }
-  KP S, R;
-  const Form *fs, *fr;
-  DeviceDesc *ds, *dr;
-  dt_status s1 = make_kp(st, scount, src, n, S, &fs, &ds);
-  if (s1 != DT_OK) return s1;
-  s1 = make_kp(rt, rcount, dst, n, R, &fr, &dr);
-  if (s1 != DT_OK) return s1;
-  {
-    std::lock_guard<std::mutex> g(rt->mu);
-    if (rt->ovl_count != rcount) {
-      rt->ovl_result = check_nonoverlap(rt, *fr, rcount);
-      rt->ovl_count = rcount;
-    }
-    if (rt->ovl_result != 1) {
-      set_error("dt_copy: destination typemap entries overlap");
-      return DT_ERR_OVERLAP;
-    }
+  if (nonoverlap_cached(rt, rcount) != 1) {
+    set_error("dt_copy: destination typemap entries overlap");
+    return DT_ERR_OVERLAP;
   }
+  KP S, R;
+  int kind = 1;
+  int64_t g = 1;
+  dt_status s1 = dual_params(st, scount, src, rt, rcount, dst, n, S, R, &kind, &g);
+  if (s1 != DT_OK) return s1;
   cudaStream_t s = (cudaStream_t)stream;
-  KLevels Ls, Lr;
-  build_levels(*fs, ds, st, scount, Ls);
-  build_levels(*fr, dr, rt, rcount, Lr);
-  int64_t gs = 1, gr = 1;
-  plan_kernel(*fs, Ls, (uint64_t)(uintptr_t)src, 0, 0, n, &gs);
-  plan_kernel(*fr, Lr, (uint64_t)(uintptr_t)dst, 0, 0, n, &gr);
-  const int64_t g = std::min(gs, gr);
-  const double ms = (double)S.tsize / (double)S.nblocks, mr = (double)R.tsize / (double)R.nblocks;
-  const bool words_ok = S.tsize % g == 0 && R.tsize % g == 0 && (S.tsize + R.tsize) / g <= kMaxWordTable &&
-                        template_fits_int32(*fs) && template_fits_int32(*fr);
-  const char* fk = getenv("DT_FORCE_KERNEL");
-  const int force = fk ? atoi(fk) : 0;
-  const double mm = std::min(ms, mr);
-  const bool use_words = words_ok && force != 1 && (force == 2 || mm < 256.0 || (g == 16 && mm < 1024.0));
   const int sms = num_sms();
-  if (use_words) {
-    const int32_t *wa = nullptr, *wb = nullptr;
-    s1 = ensure_wtab(*fs, *ds, g, &wa);
-    if (s1 != DT_OK) return s1;
-    s1 = ensure_wtab(*fr, *dr, g, &wb);
-    if (s1 != DT_OK) return s1;
-    S.wtab = wa;
-    S.nwords = (int32_t)(S.tsize / g);
-    R.wtab = wb;
-    R.nwords = (int32_t)(R.tsize / g);
+  if (kind == 4) {  // staged: cp.async gathers by S into smem tiles, scatter by R
+    const size_t smem2 = (size_t)kStageBufs * kStageTile + sizeof(int32_t) * (size_t)(S.nwords + R.nwords);
+    static bool attr = false;
+    if (!attr) {
+      cudaFuncSetAttribute(k_dual_stage<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
+      cudaFuncSetAttribute(k_dual_stage<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
+      attr = true;
+    }
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dual_stage<16>, 256, smem2) != cudaSuccess || occ < 1)
+      occ = 1;
+    const int64_t ntiles = (n + kStageTile - 1) / kStageTile;
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
+    if (g == 8) k_dual_stage<8><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
+    else k_dual_stage<16><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
+  } else if (kind == 2) {
     const size_t smem = sizeof(int32_t) * (size_t)(S.nwords + R.nwords);
     const int64_t nwords = n / g;
-    if (g >= 8 && force != 5) {  // staged: cp.async gathers by S into smem tiles, scatter by R
-      const size_t smem2 = (size_t)kStageBufs * kStageTile + smem;
-      static bool attr = false;
-      if (!attr) {
-        cudaFuncSetAttribute(k_dual_stage<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
-        cudaFuncSetAttribute(k_dual_stage<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
-        attr = true;
-      }
-      int occ = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_dual_stage<16>, 256, smem2) != cudaSuccess || occ < 1)
-        occ = 1;
-      const int64_t ntiles = (n + kStageTile - 1) / kStageTile;
-      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
-      if (g == 8) k_dual_stage<8><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
-      else k_dual_stage<16><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
-      cudaError_t e = cudaGetLastError();
-      if (e != cudaSuccess) return cuda_fail(e, "dt_copy launch");
-      return DT_OK;
-    }
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * 6, (nwords + 1023) / 1024));
     switch (g) {
       case 1: k_dual_word<1><<<grid, 256, smem, s>>>(S, R, n); break;

@@ -603,6 +603,9 @@ static Form build_form(const dt_type_s* t) {
     case K_RESIZED:
       f = build_form(t->old);
       break;
+    case K_FLAT:
+      f = *t->form;
+      break;
   }
   normalize(f);
   // keep the kernel's level budget: fold innermost levels into the template
@@ -687,6 +690,89 @@ dt_status dt_flatten(dt_t t, int64_t count, int64_t* disps, int64_t* lens, int64
     disps[i] = d[i];
     lens[i] = l[i];
   }
+  return DT_OK;
+}
+
+// ------------------------------------------------------------------ serialization
+// Wire format (int64 words, native byte order -- homogeneous GPUs, reading A5):
+//   magic, version, size, lb, ub, true_lb, true_ub, align, has_lb, has_ub,
+//   nlev, nblocks, [cnt, stride, table_len] x nlev, bd[nblocks], bl[nblocks],
+//   tables (concatenated, level order).
+// This ships a committed layout to a peer rank (direct exchange plans, f1): the
+// receiver's flattened form travels, not its constructor tree.
+static const int64_t kSerMagic = 0x4454464F524D0001LL;  // "DTFORM" v1
+
+dt_status dt_type_serialize(dt_t t, void* out, size_t* nbytes) {
+  CHECK_ARG(t && nbytes, "NULL argument");
+  const Form* f;
+  dt_status s = safe_form(t, &f);
+  if (s != DT_OK) return s;
+  std::vector<int64_t> w = {kSerMagic, 1, t->size, t->lb, t->ub, t->true_lb, t->true_ub, t->align,
+                            t->has_lb ? 1 : 0, t->has_ub ? 1 : 0, (int64_t)f->lv.size(), (int64_t)f->bd.size()};
+  for (auto& l : f->lv) {
+    w.push_back(l.cnt);
+    w.push_back(l.stride);
+    w.push_back(l.is_list() ? (int64_t)l.table->size() : -1);
+  }
+  w.insert(w.end(), f->bd.begin(), f->bd.end());
+  w.insert(w.end(), f->bl.begin(), f->bl.end());
+  for (auto& l : f->lv)
+    if (l.is_list()) w.insert(w.end(), l.table->begin(), l.table->end());
+  const size_t need = w.size() * sizeof(int64_t);
+  if (!out) {
+    *nbytes = need;
+    return DT_OK;
+  }
+  CHECK_ARG(*nbytes >= need, "buffer too small");
+  std::memcpy(out, w.data(), need);
+  *nbytes = need;
+  return DT_OK;
+}
+
+dt_status dt_type_deserialize(const void* in, size_t nbytes, dt_t* out) {
+  CHECK_ARG(in && out, "NULL argument");
+  CHECK_ARG(nbytes % 8 == 0 && nbytes >= 12 * 8, "truncated type blob");
+  const size_t nw = nbytes / 8;
+  std::vector<int64_t> w(nw);
+  std::memcpy(w.data(), in, nbytes);
+  CHECK_ARG(w[0] == kSerMagic && w[1] == 1, "not a serialized dt type");
+  const int64_t nlev = w[10], nb = w[11];
+  CHECK_ARG(nlev >= 0 && nlev < kMaxLevels && nb >= 0, "corrupt type blob");
+  size_t k = 12;
+  CHECK_ARG(k + 3 * (size_t)nlev + 2 * (size_t)nb <= nw, "truncated type blob");
+  std::unique_ptr<Form> f(new Form);
+  std::vector<int64_t> tl;
+  for (int64_t i = 0; i < nlev; i++) {
+    Level l;
+    l.cnt = w[k++];
+    l.stride = w[k++];
+    tl.push_back(w[k++]);
+    f->lv.push_back(l);
+  }
+  f->bd.assign(w.begin() + k, w.begin() + k + nb);
+  k += nb;
+  f->bl.assign(w.begin() + k, w.begin() + k + nb);
+  k += nb;
+  for (int64_t i = 0; i < nlev; i++) {
+    if (tl[i] < 0) continue;
+    CHECK_ARG(tl[i] == f->lv[i].cnt && k + (size_t)tl[i] <= nw, "truncated type blob");
+    f->lv[i].table = std::make_shared<std::vector<int64_t>>(w.begin() + k, w.begin() + k + tl[i]);
+    f->lv[i].stride = 0;
+    k += tl[i];
+  }
+  CHECK_ARG(k == nw, "trailing bytes in type blob");
+  auto* t = new dt_type_s;
+  t->kind = K_FLAT;
+  t->size = w[2];
+  t->lb = w[3];
+  t->ub = w[4];
+  t->true_lb = w[5];
+  t->true_ub = w[6];
+  t->align = w[7];
+  t->has_lb = w[8] != 0;
+  t->has_ub = w[9] != 0;
+  t->form = std::move(f);
+  *out = t;
   return DT_OK;
 }
 

@@ -71,45 +71,6 @@ struct XArgs {
   XOp ops[kMaxOps];
 };
 
-__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
-  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ void red_release_sys_add(uint64_t* p, uint64_t v) {
-  asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ uint64_t gtimer() {
-  uint64_t t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-
-enum { XERR_TIMEOUT = 1, XERR_TRUNCATE = 2 };
-
-// spin until pred(*p) holds; false on timeout (sets *err)
-template <typename Pred>
-__device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeout_ns, int32_t* err, uint64_t* out,
-                                     bool sleep = true) {
-  uint64_t v = ld_acquire_sys(p);
-  if (pred(v)) { *out = v; return true; }
-  const uint64_t t0 = gtimer();
-  int ns = 32;
-  while (true) {
-    if (sleep) __nanosleep(ns);
-    if (ns < 256) ns <<= 1;
-    v = ld_acquire_sys(p);
-    if (pred(v)) { *out = v; return true; }
-    if ((int64_t)(gtimer() - t0) > timeout_ns) {
-      atomicCAS(err, 0, XERR_TIMEOUT);
-      return false;
-    }
-  }
-}
-
 // pack or unpack stream bytes [lo, lo+len) of the current chunk with this CTA.
 // cb: the slot base such that stream byte x of the message lives at cb + x.  The
 // op's parameters stay in the grid-constant bank (no per-fragment struct copy).
@@ -393,6 +354,12 @@ struct dt_comm_s {
     return bases + ((((size_t)parity * 2 + dir) * nranks + peer) * nch + ch) * per();
   }
 };
+
+void dt::comm_info(dt_comm_t c, int* rank, int* nranks, int* device) {
+  *rank = c->rank;
+  *nranks = c->nranks;
+  *device = c->device;
+}
 
 static dt_status cufail(cudaError_t e, const char* what) {
   set_error("%s: %s", what, cudaGetErrorString(e));

@@ -36,6 +36,11 @@ class FormInfo(C.Structure):
                 ("level_stride", C.c_int64 * 8), ("granularity", C.c_int64)]
 
 
+class XOp(C.Structure):
+    _fields_ = [("buf", C.c_void_p), ("count", C.c_int64), ("type", C.c_void_p), ("peer", C.c_int32),
+                ("tag", C.c_int32)]
+
+
 class XferOpts(C.Structure):
     _fields_ = [("chunk_bytes", C.c_int64), ("depth", C.c_int32), ("mode", C.c_int32), ("ctas", C.c_int32),
                 ("flags", C.c_int32)]
@@ -78,6 +83,14 @@ _SIGS = {
     "dt_group_end": (C.c_int, [P, P]),
     "dt_comm_check": (C.c_int, [P]),
     "dt_comm_free": (C.c_int, [C.POINTER(P)]),
+    "dt_type_serialize": (C.c_int, [P, P, C.POINTER(C.c_size_t)]),
+    "dt_type_deserialize": (C.c_int, [P, C.c_size_t, C.POINTER(P)]),
+    "dt_xplan_create": (C.c_int, [P, C.c_int, P, C.c_int, P, C.POINTER(P)]),
+    "dt_xplan_local_blob": (C.c_int, [P, P, C.POINTER(C.c_size_t)]),
+    "dt_xplan_connect": (C.c_int, [P, P, C.POINTER(C.c_size_t)]),
+    "dt_xplan_start": (C.c_int, [P, P]),
+    "dt_xplan_check": (C.c_int, [P]),
+    "dt_xplan_free": (C.c_int, [C.POINTER(P)]),
     "dt_last_error": (C.c_char_p, []),
     "dt_version": (C.c_char_p, []),
 }
@@ -230,6 +243,22 @@ class Type:
         _check(lib().dt_flatten(self.h, count, d.ctypes.data_as(PI64), ln.ctypes.data_as(PI64), n.value,
                                 C.byref(n)))
         return d[: n.value], ln[: n.value]
+
+    def serialize(self) -> bytes:
+        """dt_type_serialize: the flattened form + bounds, to ship to another rank."""
+        n = C.c_size_t(0)
+        _check(lib().dt_type_serialize(self.h, None, C.byref(n)))
+        buf = C.create_string_buffer(n.value)
+        _check(lib().dt_type_serialize(self.h, buf, C.byref(n)))
+        return buf.raw[: n.value]
+
+    @staticmethod
+    def deserialize(blob: bytes) -> "Type":
+        """dt_type_deserialize: a new (uncommitted) handle with the serialized typemap."""
+        h = P()
+        buf = C.create_string_buffer(blob, len(blob))
+        _check(lib().dt_type_deserialize(buf, len(blob), C.byref(h)))
+        return Type(h)
 
     def plan(self, count, origin_addr, packed_addr, pos, nbytes):
         k = C.c_int()
@@ -413,3 +442,69 @@ def copy(stype: Type, scount: int, src, rtype: Type, rcount: int, dst, stream=No
     """dt_copy: fused datatype -> datatype copy on one GPU (no packed buffer)."""
     _check(lib().dt_copy(stype.h, scount, _ptr(src) + src_offset, rtype.h, rcount, _ptr(dst) + dst_offset,
                          _stream(stream)))
+
+
+# ------------------------------------------------------------------ persistent direct exchange (f1 across GPUs)
+class XPlan:
+    """dt_xplan_t: a fixed set of sends and receives executed as ONE kernel per rank
+    per start: each send is copied from its local layout straight into the
+    receiver's layout in peer memory (NVLink / CUDA IPC), no ring and no unpack.
+
+    sends / recvs: lists of (buf, count, type, peer, tag) (buf: tensor or device
+    address; tag pairs a send of rank r to rank d with d's receive from r).
+    Connect with `from_process_group` (blobs all-gathered through
+    torch.distributed) or, on a single rank, `local()`."""
+
+    def __init__(self, comm: Comm, sends, recvs):
+        self.comm = comm
+        self._keep = (sends, recvs)
+        mk = lambda ops: (XOp * max(1, len(ops)))(*[XOp(_ptr(b), c, t.h, p, g) for (b, c, t, p, g) in ops])  # noqa
+        so, ro = mk(sends), mk(recvs)
+        self.h = P()
+        _check(lib().dt_xplan_create(comm.h, len(sends), so, len(recvs), ro, C.byref(self.h)))
+
+    def local_blob(self) -> bytes:
+        n = C.c_size_t(0)
+        _check(lib().dt_xplan_local_blob(self.h, None, C.byref(n)))
+        buf = C.create_string_buffer(n.value)
+        _check(lib().dt_xplan_local_blob(self.h, buf, C.byref(n)))
+        return buf.raw[: n.value]
+
+    def connect(self, blobs):
+        sizes = (C.c_size_t * len(blobs))(*[len(b) for b in blobs])
+        allb = b"".join(blobs)
+        buf = C.create_string_buffer(allb, max(1, len(allb)))
+        _check(lib().dt_xplan_connect(self.h, buf, sizes))
+        return self
+
+    @classmethod
+    def from_process_group(cls, comm: Comm, sends, recvs, group=None) -> "XPlan":
+        import torch.distributed as tdist
+        x = cls(comm, sends, recvs)
+        out = [None] * tdist.get_world_size(group)
+        tdist.all_gather_object(out, x.local_blob(), group=group)
+        return x.connect(out)
+
+    @classmethod
+    def local(cls, comm: Comm, sends, recvs) -> "XPlan":
+        """Single-rank plan (every peer is this rank)."""
+        x = cls(comm, sends, recvs)
+        return x.connect([x.local_blob()])
+
+    def start(self, stream=None):
+        _check(lib().dt_xplan_start(self.h, _stream(stream)))
+
+    def check(self):
+        _check(lib().dt_xplan_check(self.h))
+
+    def free(self):
+        if self.h:
+            _check(lib().dt_xplan_free(C.byref(self.h)))
+            self.h = P()
+
+    def __del__(self):
+        try:
+            if self.h and _lib is not None:
+                _lib.dt_xplan_free(C.byref(self.h))
+        except Exception:
+            pass

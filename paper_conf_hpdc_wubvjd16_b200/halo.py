@@ -75,6 +75,19 @@ class HaloPlan:
                 comm.sendrecv(None, 0, None, -1, buf, 1, self.recv_types[face], peer, stream=stream)
         comm.group_end(stream)
 
+    def direct_plan(self, comm, buf, group=None, single_rank=False):
+        """The same exchange as a persistent direct plan (dt_xplan): one kernel per
+        exchange writes every boundary layer straight into the neighbour's ghost
+        layer in peer memory.  Tag = index of the SENDER's face in FACES, so the
+        pairing is unique even when both neighbours in a dimension are one rank."""
+        from .dt import XPlan
+        sends = [(buf, 1, self.send_types[f], neighbour(self.rank, f, self.dims), i) for i, f in enumerate(FACES)]
+        recvs = [(buf, 1, self.recv_types[OPPOSITE[f]], neighbour(self.rank, OPPOSITE[f], self.dims), i)
+                 for i, f in enumerate(FACES)]
+        if single_rank:
+            return XPlan.local(comm, sends, recvs)
+        return XPlan.from_process_group(comm, sends, recvs, group)
+
     def ops(self):
         """[(kind, face, peer)] in posting order: kind 'send' (my boundary layer `face`
         to `peer`) or 'recv' (ghost layer `face` from `peer`)."""

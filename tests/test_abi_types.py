@@ -148,3 +148,30 @@ def test_component_free_is_safe():
     gc.collect()
     d, ln = c.flatten(1)
     assert c.size == 96 and d.tolist() == [0, 40, 80, 136, 176] and ln.tolist() == [16, 16, 32, 16, 16]
+
+
+def test_type_serialize_roundtrip():
+    """dt_type_serialize / dt_type_deserialize (shipping a receive layout to the sender
+    of a direct plan): same bounds, same flattened typemap at several counts, usable
+    as a component, malformed blobs rejected."""
+    import numpy as np
+    from workloads import c1_submatrix, c3_block_cyclic, c4_face
+    recs = [c2_lower_triangle(300)[0], c3_block_cyclic(1024, 64)[0], c5_particles(56 * 100)[0], c4_face("x-", 40)[0],
+            c1_submatrix(64, 200, 1, 2)[0], c5b_irregular(1 << 12)[0],
+            ("resized", ("struct", [1, 1], [0, 16], [("basic", "DOUBLE")] * 2), -8, 40),
+            ("vector", 3, 1, -2, ("basic", "INT32"))]
+    for r in recs:
+        t = dt.from_recipe(r)
+        u = dt.Type.deserialize(t.serialize())
+        assert (u.size, u.extent, u.true_extent) == (t.size, t.extent, t.true_extent)
+        for count in (1, 3):
+            d1, l1 = t.flatten(count)
+            d2, l2 = u.flatten(count)
+            assert np.array_equal(d1, d2) and np.array_equal(l1, l2)
+        v = u.contiguous(2)
+        assert v.size == 2 * t.size
+    blob = bytearray(dt.from_recipe(recs[0]).serialize())
+    for bad in (bytes(blob[:40]), bytes(blob[:-8]), b"\0" * len(blob)):
+        with pytest.raises(dt.DTError) as e:
+            dt.Type.deserialize(bad)
+        assert e.value.name == "DT_ERR_ARG"

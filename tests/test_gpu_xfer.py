@@ -250,3 +250,164 @@ def test_fused_copy_direct(torch_cuda):
     with pytest.raises(dt.DTError) as e:
         dt.copy(dt.Type.basic("INT32").contiguous(12).commit(), 1, x, ov, 1, x)
     assert e.value.name == "DT_ERR_OVERLAP"
+
+
+# ------------------------------------------------------------------ persistent direct plans (dt_xplan, f1 across GPUs)
+def _direct_case(torch, srec, sorg, spar, rrec, rorg, rpar, seed):
+    """(send tensor, receive tensor, expected receive bytes) for one send -> receive."""
+    so, ro = oracle.from_recipe(srec), oracle.from_recipe(rrec)
+    sh = fill_bytes(spar, seed)
+    exp = np.full(rpar, 0xA5, dtype=np.uint8)
+    oracle.sendrecv(so, 1, sh, ro, 1, exp, sorg, rorg)
+    return torch.from_numpy(sh).cuda(), torch.full((rpar,), 0xA5, dtype=torch.uint8, device="cuda"), exp
+
+
+def test_direct_plan_single_rank(torch_cuda):
+    """A 1-rank plan of several sends-to-self with different send/receive types and
+    every copy family (long runs, word tables, staged): repeated starts reuse the
+    flags (sequence numbers), each start moves the CURRENT source bytes."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0)
+    pairs = [c3_block_cyclic(1024, 64)[:3] * 2,
+             c2_lower_triangle(257)[:3] + c5_particles(257 * 258 // 2 * 8)[:3],
+             c5_particles(56 * 3000)[:3] + (("contiguous", 3000 * 14, ("basic", "INT32")), 0, 3000 * 56),
+             c1_submatrix(128, 512, 3, 5)[:3] + (("contiguous", 128 * 128, ("basic", "DOUBLE")), 0, 128 * 128 * 8)]
+    for rnd in range(3):
+        sends, recvs, exps, bufs = [], [], [], []
+        for i, (sr, so_, sp, rr, ro_, rp) in enumerate(pairs):
+            sd, rd, exp = _direct_case(torch, sr, so_, sp, rr, ro_, rp, 40 + i + 10 * rnd)
+            st, rt = dt.from_recipe(sr).commit(), dt.from_recipe(rr).commit()
+            sends.append((sd.data_ptr() + so_, 1, st, 0, i))
+            recvs.append((rd.data_ptr() + ro_, 1, rt, 0, i))
+            exps.append(exp)
+            bufs.append((sd, rd, st, rt))
+        plan = dt.XPlan.local(comm, sends, recvs)
+        for _ in range(2):  # the second start re-sends the same bytes into the same layouts
+            plan.start()
+            torch.cuda.synchronize()
+            plan.check()
+        for (sd, rd, _, _), exp in zip(bufs, exps):
+            assert np.array_equal(rd.cpu().numpy(), exp), rnd
+        plan.free()
+    comm.free()
+
+
+def test_direct_plan_halo_single_rank(torch_cuda):
+    """1-rank periodic halo as one direct plan (12 ops, one kernel per exchange)."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import FACES, face_box, make_plan
+    n, h = 64, 1
+    L = n + 2 * h
+    comm = dt.Comm(0, 1, 0)
+    hp = make_plan(0, n, h, dims=(1, 1, 1))
+    A = np.full((L, L, L), 0xA5A5A5A5, dtype=np.uint32)
+    z, y, x = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
+    A[h:h + n, h:h + n, h:h + n] = (z * 1000000 + y * 1000 + x).astype(np.uint32)
+    buf = torch.from_numpy(A.view(np.uint8).reshape(-1).copy()).cuda()
+    xp = hp.direct_plan(comm, buf, single_rank=True)
+    for _ in range(3):
+        xp.start()
+    torch.cuda.synchronize()
+    xp.check()
+    B = buf.cpu().numpy().view(np.uint32).reshape(L, L, L)
+    for f in FACES:
+        sub, st = face_box(f, n, h, ghost=True)
+        zz, yy, xx = np.meshgrid(*[np.arange(s, s + k) for s, k in zip(st, sub)], indexing="ij")
+        exp = (((zz - h) % n) * 1000000 + ((yy - h) % n) * 1000 + ((xx - h) % n)).astype(np.uint32)
+        assert np.array_equal(B[zz, yy, xx], exp), f
+    # the interior is untouched
+    assert np.array_equal(B[h:h + n, h:h + n, h:h + n], A[h:h + n, h:h + n, h:h + n])
+    xp.free()
+    comm.free()
+
+
+def test_direct_plan_errors(torch_cuda):
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0)
+    x = torch.zeros(4096, dtype=torch.uint8, device="cuda")
+    a = dt.Type.basic("DOUBLE").contiguous(10).commit()
+    b = dt.Type.basic("DOUBLE").contiguous(9).commit()
+    with pytest.raises(dt.DTError) as e:   # 80 bytes into a 72-byte receive: at connect, before any byte moves
+        dt.XPlan.local(comm, [(x, 1, a, 0, 7)], [(x.data_ptr() + 1024, 1, b, 0, 7)])
+    assert e.value.name == "DT_ERR_TRUNCATE"
+    ov = dt.Type.basic("INT32").vector(4, 3, 2).commit()
+    with pytest.raises(dt.DTError) as e:
+        dt.XPlan.local(comm, [], [(x, 1, ov, 0, 1)])
+    assert e.value.name == "DT_ERR_OVERLAP"
+    with pytest.raises(dt.DTError) as e:   # no receive with this tag
+        dt.XPlan.local(comm, [(x, 1, a, 0, 1)], [(x.data_ptr() + 1024, 1, a, 0, 2)])
+    assert e.value.name == "DT_ERR_ARG"
+    comm.free()
+
+
+def _direct_worker(rank, port, q):
+    try:
+        import torch
+        import torch.distributed as tdist
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        os.environ.setdefault("DT_TIMEOUT_MS", "60000")
+        tdist.init_process_group("gloo", rank=rank, world_size=2)
+        torch.cuda.set_device(0)
+        from paper_conf_hpdc_wubvjd16_b200 import dt
+        comm = dt.Comm.from_process_group(device=0)
+        # rank 0 sends its lower triangle into rank 1's block-cyclic-shaped receive, rank 1
+        # sends its block-cyclic submatrix into rank 0's contiguous receive (types differ)
+        tri, torg, tpar = c2_lower_triangle(512)
+        bc, borg, bpar = c3_block_cyclic(1024, 64)
+        ot, ob = oracle.from_recipe(tri), oracle.from_recipe(bc)
+        ctg = ("contiguous", ob.size, ("basic", "BYTE"))
+        oc = oracle.from_recipe(ctg)
+        T, B, Cg = (dt.from_recipe(r).commit() for r in (tri, bc, ctg))
+        mine = torch.from_numpy(fill_bytes(max(tpar, bpar), 300 + rank)).cuda()
+        rbuf = torch.full((max(bpar, ob.size) + 64,), 0xA5, dtype=torch.uint8, device="cuda")
+        if rank == 0:
+            sends = [(mine.data_ptr() + torg, 1, T, 1, 5)]
+            recvs = [(rbuf, 1, Cg, 1, 9)]
+        else:
+            sends = [(mine.data_ptr() + borg, 1, B, 0, 9)]
+            # receive the 512^2 triangle's bytes into the first bytes of a block-cyclic layout
+            recvs = [(rbuf.data_ptr() + borg, 1, B, 0, 5)]
+        plan = dt.XPlan.from_process_group(comm, sends, recvs)
+        for _ in range(2):
+            plan.start()
+        torch.cuda.synchronize()
+        plan.check()
+        other = fill_bytes(max(tpar, bpar), 300 + (1 - rank))
+        exp = np.full(rbuf.numel(), 0xA5, dtype=np.uint8)
+        if rank == 0:
+            oracle.sendrecv(ob, 1, other, oc, 1, exp, borg, 0)
+        else:
+            oracle.sendrecv(ot, 1, other, ob, 1, exp, torg, borg)
+        ok = bool(np.array_equal(rbuf.cpu().numpy(), exp))
+        tdist.barrier()
+        plan.free()
+        comm.free()
+        q.put((rank, ok))
+        tdist.destroy_process_group()
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, traceback.format_exc() + repr(e)))
+
+
+def test_direct_plan_two_processes_ipc(torch_cuda):
+    """Two ranks (processes) with different send/receive types: each rank's kernel
+    writes straight into the other process's buffer through CUDA IPC."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_direct_worker, args=(r, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = [q.get(timeout=300) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+    for rank, ok in res:
+        assert ok is True, (rank, ok)
