@@ -310,17 +310,17 @@ def run_e2e(args, t, src_h, org, parent, payload, dev):
             "steps": steps, "note": "host pinned buffers; wall clock incl. all copies and syncs"}
 
 
-def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup):
+def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup, workload="c3"):
     """Pairwise C3 exchange through dt_sendrecv over a chunk x depth sweep (S7).
     Returns (results, payload, spot_parity); every timing is the max over ranks of
     the device time between a barrier-aligned pair of CUDA events."""
     import torch
 
     from paper_conf_hpdc_wubvjd16_b200 import dt
-    from workloads import c3_block_cyclic, fill_bytes, seed_for
+    from workloads import c3_block_cyclic, c5_particles, fill_bytes, seed_for
     dev = torch.device("cuda", local)
     peer = rank ^ 1 if (rank ^ 1) < ws else rank
-    rec, org, parent = c3_block_cyclic()
+    rec, org, parent = c3_block_cyclic() if workload == "c3" else c5_particles(128 << 20)
     t = dt.from_recipe(rec).commit()
     payload = t.size
     A = torch.from_numpy(fill_bytes(parent, seed_for(3) + rank)).to(dev)
@@ -370,9 +370,15 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup):
             if mode_name == "direct":
                 xp.free()
             comm.free()
-    # parity of the last exchange: my B must equal the peer's A (same layout on both sides)
+    # parity of the last exchange: the typemap bytes of my B must equal the peer's A's
+    # (same layout on both sides; gap bytes of B keep their poison)
     exp = torch.from_numpy(fill_bytes(parent, seed_for(3) + peer)).to(dev)
-    ok = bool(torch.equal(B.view(-1)[org:org + 8 * 64], exp.view(-1)[org:org + 8 * 64]))
+    pb = torch.empty(payload, dtype=torch.uint8, device=dev)
+    pe = torch.empty(payload, dtype=torch.uint8, device=dev)
+    dt.pack(t, 1, B, pb, origin_offset=org)
+    dt.pack(t, 1, exp, pe, origin_offset=org)
+    ok = bool(torch.equal(pb, pe))
+    del pb, pe
     return results, payload, ok, (t, A, B, org)
 
 
@@ -390,7 +396,8 @@ def run_xfer(args):
     steps = max(3, min(args.steps, 20))
     results, payload, ok, (t, A, B, org) = xfer_sweep(
         ws, rank, local, [int(x) << 10 for x in args.xfer_chunks_kib.split(",")],
-        [int(x) for x in args.xfer_depths.split(",")], args.xfer_mode, args.xfer_ctas, steps, args.warmup)
+        [int(x) for x in args.xfer_depths.split(",")], args.xfer_mode, args.xfer_ctas, steps, args.warmup,
+        args.xfer_workload)
     s = torch.cuda.current_stream()
     best = max(results, key=lambda r: r["gbs_per_rank"])
     value = ws * payload / (best["ms"] * 1e-3) / 1e9
@@ -411,8 +418,9 @@ def run_xfer(args):
     line = {"metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": ws, "steps": steps,
             "warmup": args.warmup, "ms_per_step": best["ms"], "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
-            "config": {"workload": "C3: ScaLAPACK 2D block-cyclic submatrix (N=8192 f64, nb=64, owner (0,1)), "
-                                   f"pairwise exchange, mode={args.xfer_mode}",
+            "config": {"workload": ("C3: ScaLAPACK 2D block-cyclic submatrix (N=8192 f64, nb=64, owner (0,1))"
+                                    if args.xfer_workload == "c3" else "C5: 128 MiB of LAMMPS-style particles")
+                                   + f", pairwise exchange, mode={args.xfer_mode}",
                        "payload_bytes": payload, "sweep": results, "spot_parity": ok,
                        "fused_loopback_gbs_per_rank": fused,
                        "pairs": "loopback (1 GPU)" if ws == 1 else "(r, r^1)"},
@@ -641,6 +649,7 @@ def main():
     ap.add_argument("--sweep", default="all", help="--workload sweep: comma-separated config names or 'all'")
     ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "direct"],
                     help="p2p ring pipeline, NCCL double buffering, or a persistent direct plan (dt_xplan)")
+    ap.add_argument("--xfer-workload", default="c3", choices=["c3", "c5"])
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
     ap.add_argument("--xfer-depths", default="2,4")
     ap.add_argument("--xfer-ctas", type=int, default=0, help="CTAs per direction (0 = library default)")

@@ -914,12 +914,13 @@ struct RecGeo {
 };
 constexpr int kRecMaxLPL = 8;
 
-template <int G>
+// [lo, hi): the stream bytes this call may write (the request, or one pipeline fragment)
+template <int G, int POL = LD_CS>
 __device__ __forceinline__ void rec_pack_batch(const KP& P, const RecGeo& R, uint8_t* cb, int64_t e0, uint8_t* buf,
-                                               const int64_t* sd, const uint16_t* omap, int lane) {
+                                               const int64_t* sd, const uint16_t* omap, int lane, int64_t lo,
+                                               int64_t end) {
   typedef typename WordT<G>::T W;
   constexpr int NW = 16 / G;
-  const int64_t end = P.pos + P.len;
   uint4 v[kRecMaxLPL];
 #pragma unroll
   for (int j = 0; j < kRecMaxLPL; j++) {
@@ -927,7 +928,7 @@ __device__ __forceinline__ void rec_pack_batch(const KP& P, const RecGeo& R, uin
       const int idx = lane + 32 * j;
       const int r = (idx * R.invnch) >> 16, ch = idx - r * R.nch;
       const int64_t e = e0 + r;
-      if (e >= R.e_lo && e < R.e_hi) v[j] = ldv<LD_CS>(reinterpret_cast<const uint4*>(P.nc + sd[r] + R.a0 + 16 * ch));
+      if (e >= R.e_lo && e < R.e_hi) v[j] = ldv<POL>(reinterpret_cast<const uint4*>(P.nc + sd[r] + R.a0 + 16 * ch));
     }
   }
 #pragma unroll
@@ -938,30 +939,30 @@ __device__ __forceinline__ void rec_pack_batch(const KP& P, const RecGeo& R, uin
   const int64_t sb = e0 * P.tsize;
   for (int vv = lane; vv < nvec; vv += 32) {
     const int64_t s = sb + 16 * (int64_t)vv;
-    if (s + 16 <= P.pos || s >= end) continue;
+    if (s + 16 <= lo || s >= end) continue;
     union {
       uint4 q;
       W w[NW];
     } o;
 #pragma unroll
     for (int k = 0; k < NW; k++) o.w[k] = *reinterpret_cast<const W*>(buf + omap[vv * NW + k]);
-    if (s >= P.pos && s + 16 <= end) {
+    if (s >= lo && s + 16 <= end) {
       stv(reinterpret_cast<uint4*>(cb + s), o.q);
     } else {
       const uint8_t* ob = reinterpret_cast<const uint8_t*>(&o.q);
       for (int k = 0; k < 16; k++)
-        if (s + k >= P.pos && s + k < end) cb[s + k] = ob[k];
+        if (s + k >= lo && s + k < end) cb[s + k] = ob[k];
     }
   }
   __syncwarp();
 }
 
-template <int G>
+template <int G, int POL = LD_CS>
 __device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, const uint8_t* cb, int64_t e0,
-                                                 uint8_t* buf, const int64_t* sd, const int16_t* umap, int lane) {
+                                                 uint8_t* buf, const int64_t* sd, const int16_t* umap, int lane,
+                                                 int64_t lo, int64_t end) {
   typedef typename WordT<G>::T W;
   constexpr int NW = 16 / G;
-  const int64_t end = P.pos + P.len;
   const int nvec = (int)((int64_t)R.RB * P.tsize / 16);
   const int64_t sb = e0 * P.tsize;
   uint4 v[kRecMaxLPL];
@@ -969,17 +970,17 @@ __device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, c
   for (int j = 0; j < kRecMaxLPL; j++) {  // nvec <= RB*spanB/16 = 32*LPL
     const int vv = lane + 32 * j;
     const int64_t s = sb + 16 * (int64_t)vv;
-    if (j < R.LPL && vv < nvec && s >= P.pos && s + 16 <= end) v[j] = ldv<LD_CS>(reinterpret_cast<const uint4*>(cb + s));
+    if (j < R.LPL && vv < nvec && s >= lo && s + 16 <= end) v[j] = ldv<POL>(reinterpret_cast<const uint4*>(cb + s));
   }
 #pragma unroll
   for (int j = 0; j < kRecMaxLPL; j++) {
     const int vv = lane + 32 * j;
     const int64_t s = sb + 16 * (int64_t)vv;
     if (j < R.LPL && vv < nvec) {
-      if (s >= P.pos && s + 16 <= end) reinterpret_cast<uint4*>(buf)[vv] = v[j];
-      else if (s + 16 > P.pos && s < end)  // ragged ends of the request: in-range words only
+      if (s >= lo && s + 16 <= end) reinterpret_cast<uint4*>(buf)[vv] = v[j];
+      else if (s + 16 > lo && s < end)  // ragged ends of the request: in-range words only
         for (int k = 0; k < 16; k += G)
-          if (s + k >= P.pos && s + k + G <= end)
+          if (s + k >= lo && s + k + G <= end)
             *reinterpret_cast<W*>(buf + 16 * vv + k) = *reinterpret_cast<const W*>(cb + s + k);
     }
   }
@@ -992,7 +993,7 @@ __device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, c
       const int64_t e = e0 + r;
       if (e >= R.e_lo && e < R.e_hi) {
         const int64_t rs = e * P.tsize;  // stream byte of the record's first word
-        const bool whole = rs >= P.pos && rs + P.tsize <= end;
+        const bool whole = rs >= lo && rs + P.tsize <= end;
         union {
           uint4 q;
           W w[NW];
@@ -1003,7 +1004,7 @@ __device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, c
           const int m = umap[ch * NW + k];
           if (m >= 0) {
             const int64_t x = rs + (int64_t)m * G;
-            if (whole || (x >= P.pos && x + G <= end)) {
+            if (whole || (x >= lo && x + G <= end)) {
               o.w[k] = *reinterpret_cast<const W*>(buf + (int64_t)r * P.tsize + (int64_t)m * G);
               mask |= 1u << k;
             }
@@ -1021,6 +1022,42 @@ __device__ __forceinline__ void rec_unpack_batch(const KP& P, const RecGeo& R, c
     }
   }
   __syncwarp();
+}
+
+// Per-CTA maps of the record-span kernels from the span words of the template:
+// pack -> omap[i] (tile word i -> shared byte), unpack -> umap[span word] (-1 = gap).
+template <bool UNPACK, int G>
+__device__ __forceinline__ void rec_maps(const RecGeo& R, uint16_t* omap) {
+  if (!UNPACK) {
+    const int n = R.RB * R.nwr;
+    for (int i = threadIdx.x; i < n; i += blockDim.x) {
+      const int r = i / R.nwr, k = i - r * R.nwr;
+      omap[i] = (uint16_t)(r * R.spanB + G * (int)R.woff[k]);
+    }
+  } else {
+    int16_t* umap = reinterpret_cast<int16_t*>(omap);
+    for (int i = threadIdx.x; i < R.spanB / G; i += blockDim.x) umap[i] = -1;
+    __syncthreads();
+    for (int k = threadIdx.x; k < R.nwr; k += blockDim.x) umap[R.woff[k]] = (int16_t)k;
+  }
+}
+
+// Records of stream bytes [lo, hi) by the warps (w, nwt) of a grid: batch b of RB records
+// starts at element R.b0 + b*RB (R.e_lo/e_hi/b0/nbatch describe [lo, hi)).
+template <bool UNPACK, int G, int POL>
+__device__ __forceinline__ void rec_range(const KP& P, const RecGeo& R, uint8_t* cb, int64_t lo, int64_t hi,
+                                          uint8_t* buf, int64_t* sd, uint16_t* omap, int64_t w, int64_t nwt,
+                                          int lane) {
+  for (int64_t b = w; b < R.nbatch; b += nwt) {
+    const int64_t e0 = R.b0 + b * R.RB;
+    for (int i = lane; i < R.RB; i += 32) {
+      const int64_t e = e0 + i;
+      sd[i] = (e >= R.e_lo && e < R.e_hi) ? elem_disp(P, (uint64_t)e) : 0;
+    }
+    __syncwarp();
+    if (UNPACK) rec_unpack_batch<G, POL>(P, R, cb, e0, buf, sd, reinterpret_cast<const int16_t*>(omap), lane, lo, hi);
+    else rec_pack_batch<G, POL>(P, R, cb, e0, buf, sd, omap, lane, lo, hi);
+  }
 }
 
 // ---------------------------------------------------------------- system-scope flags
@@ -1068,5 +1105,7 @@ __device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeo
 dt_status dual_params(dt_type_s* st, int64_t scount, const void* src, dt_type_s* rt, int64_t rcount, void* dst,
                       int64_t n, KP& S, KP& R, int* kind, int64_t* gran);
 int nonoverlap_cached(dt_type_s* rt, int64_t rcount);
+bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
+                  int64_t g, RecGeo* R);
 
 }  // namespace dt

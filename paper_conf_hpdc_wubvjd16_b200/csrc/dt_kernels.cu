@@ -209,31 +209,10 @@ __global__ void __launch_bounds__(256, 3) k_rec(const KP P, const RecGeo R) {
   uint8_t* buf = smem_rec + w * bufB;
   int64_t* sd = reinterpret_cast<int64_t*>(smem_rec + nwc * bufB) + w * R.RB;
   uint16_t* omap = reinterpret_cast<uint16_t*>(smem_rec + nwc * bufB + nwc * R.RB * 8);
-  int16_t* umap = reinterpret_cast<int16_t*>(omap);
-  // maps from the template's G-word table (source offset of packed word k)
-  if (!UNPACK) {
-    const int n = R.RB * R.nwr;
-    for (int i = threadIdx.x; i < n; i += blockDim.x) {
-      const int r = i / R.nwr, k = i - r * R.nwr;
-      omap[i] = (uint16_t)(r * R.spanB + G * (int)R.woff[k]);
-    }
-  } else {
-    for (int i = threadIdx.x; i < R.spanB / G; i += blockDim.x) umap[i] = -1;
-    __syncthreads();
-    for (int k = threadIdx.x; k < R.nwr; k += blockDim.x) umap[R.woff[k]] = (int16_t)k;
-  }
+  rec_maps<UNPACK, G>(R, omap);
   __syncthreads();
-  const int64_t nwt = (int64_t)gridDim.x * nwc;
-  for (int64_t b = (int64_t)blockIdx.x * nwc + w; b < R.nbatch; b += nwt) {
-    const int64_t e0 = R.b0 + b * R.RB;
-    for (int i = lane; i < R.RB; i += 32) {
-      const int64_t e = e0 + i;
-      sd[i] = (e >= R.e_lo && e < R.e_hi) ? elem_disp(P, (uint64_t)e) : 0;
-    }
-    __syncwarp();
-    if (UNPACK) rec_unpack_batch<G>(P, R, P.c - P.pos, e0, buf, sd, umap, lane);
-    else rec_pack_batch<G>(P, R, P.c - P.pos, e0, buf, sd, omap, lane);
-  }
+  rec_range<UNPACK, G, LD_CS>(P, R, P.c - P.pos, P.pos, P.pos + P.len, buf, sd, omap,
+                              (int64_t)blockIdx.x * nwc + w, (int64_t)gridDim.x * nwc, lane);
 }
 
 template <bool UNPACK, int G, int VW>
@@ -490,8 +469,8 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
 // Record-span geometry of a launch (k_rec), or false when it does not apply:
 // G >= 4, 16-byte-aligned element bases and packed side, the template inside a
 // 16-byte-aligned span of <= 128 B that is at least half payload.
-static bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos,
-                         int64_t len, int64_t g, RecGeo* R) {
+bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
+                  int64_t g, RecGeo* R) {
   if (g < 4 || f.bl.empty() || len <= 0) return false;
   if ((nc_addr & 15) || ((c_addr - (uint64_t)pos) & 15)) return false;
   int64_t lg = level_granularity(f);

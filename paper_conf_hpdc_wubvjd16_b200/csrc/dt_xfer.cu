@@ -45,7 +45,7 @@ constexpr uint64_t kAbort = 1ull << 63;
 struct XOp {
   KP P;            // pack (send role) or unpack (recv role) over the user's layout
   int32_t role;    // 0 send, 1 recv
-  int32_t kind;    // 1 segment walk, 2 word table
+  int32_t kind;    // 1 segment walk, 2 word table, 4 smem/TMA staging, 6 record spans
   int32_t single;  // segment walk over a single-block template
   int32_t g;       // word granularity
   int64_t n;       // send: bytes; recv: capacity in bytes
@@ -60,6 +60,7 @@ struct XOp {
   uint64_t* base_out;       // [depth] after it
   uint64_t seq;
   int32_t* err;
+  RecGeo rg;       // kind 6: record-span geometry (per-fragment element range set on the device)
 };
 
 struct XArgs {
@@ -80,6 +81,28 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, uint8_t* cb, int64_t lo,
   const KP& P = X.P;
   const int64_t hi = lo + len;
   constexpr int POL = UNPACK ? LD_CG : LD_CS;  // ring slots are rewritten by the peer: bypass L1
+  if (X.kind == 6) {  // record spans: the CTA's warps take RB-record batches of the fragment
+    const int64_t hb = hi - len % X.g;  // a ragged tail (< G bytes, last fragment) is walked below
+    RecGeo R = X.rg;
+    R.e_lo = lo / P.tsize;
+    R.e_hi = (hb + P.tsize - 1) / P.tsize;
+    R.b0 = R.e_lo & ~int64_t(31);
+    R.nbatch = (R.e_hi - R.b0 + R.RB - 1) / R.RB;
+    const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5;
+    uint8_t* buf = sbuf + w * (R.RB * R.spanB);
+    int64_t* sd = reinterpret_cast<int64_t*>(sbuf + nwc * (R.RB * R.spanB)) + w * R.RB;
+    uint16_t* omap = reinterpret_cast<uint16_t*>(sbuf + nwc * (R.RB * R.spanB) + nwc * R.RB * 8);
+    const int lane = threadIdx.x & 31;
+    if (lo < hb) {
+      switch (X.g) {
+        case 4: rec_range<UNPACK, 4, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane); break;
+        case 8: rec_range<UNPACK, 8, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane); break;
+        default: rec_range<UNPACK, 16, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane); break;
+      }
+    }
+    if (hb < hi && w == nwc - 1) seg_range<UNPACK, false, POL>(P, cb, hb, hi, lane);
+    return;
+  }
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
     const int64_t bh = hi - len % X.g;  // words; a ragged tail (< G bytes, last fragment) is walked below
     switch (X.g) {
@@ -138,6 +161,17 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
     for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
   if (X.kind == 4)
     for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
+  if (X.kind == 6) {  // record-span maps after the per-warp buffers (same layout as cta_chunk)
+    const RecGeo& R = X.rg;
+    uint16_t* omap = reinterpret_cast<uint16_t*>(xsm + (blockDim.x >> 5) * (R.RB * R.spanB + R.RB * 8));
+    if (X.role == 1) {
+      switch (X.g) { case 4: rec_maps<true, 4>(R, omap); break; case 8: rec_maps<true, 8>(R, omap); break;
+                     default: rec_maps<true, 16>(R, omap); break; }
+    } else {
+      switch (X.g) { case 4: rec_maps<false, 4>(R, omap); break; case 8: rec_maps<false, 8>(R, omap); break;
+                     default: rec_maps<false, 16>(R, omap); break; }
+    }
+  }
   const int64_t C = X.chunk;
   const int D = X.depth;
   if (threadIdx.x == 0) s_stop = 0;
@@ -611,10 +645,14 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   int64_t g = 1;
   // chunk starts are multiples of `chunk` (a multiple of 512) and ring slots are aligned
   int kind = plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
-  if (kind == 6) kind = g >= 8 ? 4 : 2;  // record-span kernel: standalone only (fragments use word gathers)
-  if ((kind == 2 || kind == 4) && lowp2u((uint64_t)chunk) < g) kind = 1;
+  if (kind == 6) {  // record spans: fragments start on 512-byte stream boundaries (16-byte aligned)
+    if (!rec_geometry(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, g, &X.rg) || getenv("DT_XFER_NOREC"))
+      kind = g >= 8 ? 4 : 2;
+  }
+  if ((kind == 2 || kind == 4 || kind == 6) && lowp2u((uint64_t)chunk) < g) kind = 1;
   if (kind == 4 && g < 8) kind = 2;
-  X.kind = (kind == 2 || kind == 4) ? kind : 1;  // the block-window kernel (3) is not used inside the pipeline
+  // the block-window kernel (3) is not used inside the pipeline
+  X.kind = (kind == 2 || kind == 4 || kind == 6) ? kind : 1;
   X.single = P.nblocks == 1;
   X.g = (int32_t)g;
   if (X.kind == 2 || X.kind == 4) {
@@ -625,6 +663,14 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
     P.nwords = (int32_t)(f.tsize() / g);
   }
   return DT_OK;
+}
+
+// shared memory of a record-span op in the transfer kernel: per-warp record buffers and
+// displacements, then the per-CTA map (layout as in cta_chunk / k_xfer)
+static size_t rec_smem_bytes(const RecGeo& R, int g) {
+  const size_t nwc = kXferThreads / 32;
+  const size_t tab = std::max<size_t>((size_t)R.RB * R.nwr * 2, (size_t)(R.spanB / g) * 2);
+  return nwc * ((size_t)R.RB * R.spanB + (size_t)R.RB * 8) + tab;
 }
 
 // CTAs per direction (capped by co-residency across the group's ops); 64 measured best for
@@ -638,7 +684,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   A.timeout_ns = (int64_t)(to ? atoll(to) : 30000) * 1000000ll;
   A.flags = getenv("DT_XFER_FLAGS") ? atoi(getenv("DT_XFER_FLAGS")) : 0;
   int nops = 0, cta = 0;
-  size_t smem = 0;
+  size_t smem = 0, rec_smem = 0;
   bool any_stage = false;
   std::vector<int> sch(c->nranks, 0), rch(c->nranks, 0);
   const int G = default_ctas(c);
@@ -669,6 +715,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
       if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
       any_stage = any_stage || X.kind == 4;
+      if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
     }
     if (p.source >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
@@ -696,11 +743,12 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
       if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
       any_stage = any_stage || X.kind == 4;
+      if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
     }
   }
   if (nops == 0) return DT_OK;
   A.nops = nops;
-  A.wt_off = any_stage ? kXferStageBufs * kStageTile : 0;
+  A.wt_off = (int32_t)std::max<size_t>(any_stage ? (size_t)kXferStageBufs * kStageTile : 0, (rec_smem + 127) & ~size_t(127));
   smem += (size_t)A.wt_off;
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA must be co-resident: fit the per-op CTA count to the occupancy

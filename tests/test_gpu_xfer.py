@@ -411,3 +411,22 @@ def test_direct_plan_two_processes_ipc(torch_cuda):
         p.join(timeout=60)
     for rank, ok in res:
         assert ok is True, (rank, ok)
+
+
+@pytest.mark.parametrize("chunk", [16 << 10, 256 << 10])
+def test_ring_record_spans(torch_cuda, chunk):
+    """Record-span fragments inside the ring pipeline (sender packs whole-record 16-byte
+    loads into the ring slot, receiver scatters covered chunks): particles and
+    other dense-record layouts against a contiguous peer, both directions, count 2."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from tests.test_gpu_parity import REC_TYPES
+    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=2, ring_loopback=True)
+    for name in sorted(REC_TYPES):
+        rec, org, parent = REC_TYPES[name]()
+        size = oracle.from_recipe(rec).size
+        ctg = ("contiguous", 2 * size, ("basic", "BYTE"))
+        ext = oracle.from_recipe(rec).extent
+        _loop_check(torch_cuda, comm, rec, org, parent + ext, ctg, 0, 2 * size, scount=2, rcount=1)
+        _loop_check(torch_cuda, comm, ctg, 0, 2 * size, rec, org, parent + ext, scount=1, rcount=2)
+        _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
+    comm.free()
