@@ -112,11 +112,14 @@ dt_status dt_free(dt_t* t);
 dt_status dt_pack(dt_t t, int64_t count, const void* origin, void* packed, int64_t pos, int64_t* len, void* stream);
 dt_status dt_unpack(dt_t t, int64_t count, const void* packed, void* origin, int64_t pos, int64_t* len, void* stream);
 
-/* Same operations on HOST buffers (pinned or pageable): the library stages
- * the bytes the layout spans through device memory on `stream` (H2D of the
- * layout span, GPU pack/unpack, D2H of the result) and synchronises the
- * stream before returning.  This is the end-to-end entry point a host user
- * calls; all byte movement still happens in the GPU kernels. */
+/* Same operations on HOST buffers: page-locked (pinned, device-mapped) buffers
+ * are read and written by the pack/unpack kernel itself over the host link
+ * (zero-copy: only the typemap's bytes and the packed stream cross it; unpack
+ * writes only typemap bytes, so host gap bytes stay untouched); pageable
+ * buffers are staged through device memory on `stream` (H2D of the layout
+ * span, GPU pack/unpack, D2H of the result; DT_HOST_STAGED=1 forces this).
+ * Synchronises the stream before returning.  This is the end-to-end entry
+ * point a host user calls; all byte movement happens in GPU kernels / copies. */
 dt_status dt_pack_host(dt_t t, int64_t count, const void* origin, void* packed, int64_t pos, int64_t* len,
                        void* stream);
 dt_status dt_unpack_host(dt_t t, int64_t count, const void* packed, void* origin, int64_t pos, int64_t* len,

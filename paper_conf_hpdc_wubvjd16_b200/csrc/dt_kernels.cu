@@ -828,8 +828,20 @@ static dt_status check_dev_ptr(const void* p, const char* what) {
 
 static bool g_check_ptrs = true;
 
+// pinned host memory the device can address directly (UVA: the same pointer)
+static bool host_mapped(const void* p, void** dptr) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  if (a.type != cudaMemoryTypeHost || !a.devicePointer) return false;
+  *dptr = a.devicePointer;
+  return true;
+}
+
 static dt_status pack_common(bool unpack, dt_t t, int64_t count, const void* nc, void* c, int64_t pos, int64_t* len,
-                             void* stream) {
+                             void* stream, bool check_ptrs = true) {
   if (!t || !len || count < 0 || pos < 0 || *len < 0) {
     set_error("dt_%s: bad argument", unpack ? "unpack" : "pack");
     return DT_ERR_ARG;
@@ -846,7 +858,7 @@ static dt_status pack_common(bool unpack, dt_t t, int64_t count, const void* nc,
     set_error("dt_%s: NULL buffer", unpack ? "unpack" : "pack");
     return DT_ERR_ARG;
   }
-  if (g_check_ptrs) {
+  if (g_check_ptrs && check_ptrs) {
     dt_status st = check_dev_ptr((const uint8_t*)nc + t->true_lb, "origin");
     if (st != DT_OK) return st;
     st = check_dev_ptr(c, "packed");
@@ -1141,6 +1153,24 @@ static dt_status host_common(bool unpack, dt_t t, int64_t count, const void* a, 
   const int64_t last = (count - 1) * t->extent();
   const int64_t lo = t->true_lb + std::min<int64_t>(0, last);
   const int64_t hi = t->true_ub + std::max<int64_t>(0, last);
+  // Pinned (page-locked, device-mapped) host buffers: the pack/unpack kernel itself reads
+  // and writes host memory over the host link (zero-copy) -- only the typemap's bytes and
+  // the packed stream cross it, no span staging and no extra pass.  Pageable buffers are
+  // staged through device scratch below.
+  {
+    const uint8_t* nc = unpack ? (const uint8_t*)b : (const uint8_t*)a;
+    const uint8_t* pk = unpack ? (const uint8_t*)a : (const uint8_t*)b;
+    void *d0 = nullptr, *d1 = nullptr, *d2 = nullptr;
+    if (!getenv("DT_HOST_STAGED") && host_mapped(nc + lo, &d0) && host_mapped(nc + hi - 1, &d1) &&
+        host_mapped(pk, &d2) && (uint8_t*)d1 - (uint8_t*)d0 == hi - lo - 1) {
+      uint8_t* dorig = (uint8_t*)d0 - lo;
+      int64_t m = n;
+      dt_status st = pack_common(unpack, t, count, dorig, d2, pos, &m, stream, /*check_ptrs=*/false);
+      if (st != DT_OK) return st;
+      CU(cudaStreamSynchronize((cudaStream_t)stream));
+      return DT_OK;
+    }
+  }
   std::lock_guard<std::mutex> g(g_scratch_mu);
   void *dspan, *dpack;
   dt_status st = scratch(0, (size_t)(hi - lo), &dspan);
@@ -1149,23 +1179,20 @@ static dt_status host_common(bool unpack, dt_t t, int64_t count, const void* a, 
   if (st != DT_OK) return st;
   cudaStream_t s = (cudaStream_t)stream;
   uint8_t* dorigin = (uint8_t*)dspan - lo;
-  bool saved = g_check_ptrs;
-  g_check_ptrs = false;
   int64_t m = n;
   if (!unpack) {
     const uint8_t* horigin = (const uint8_t*)a;
     CU(cudaMemcpyAsync(dspan, horigin + lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, s));
-    st = pack_common(false, t, count, dorigin, dpack, pos, &m, stream);
+    st = pack_common(false, t, count, dorigin, dpack, pos, &m, stream, false);
     if (st == DT_OK) CU(cudaMemcpyAsync(b, dpack, (size_t)n, cudaMemcpyDeviceToHost, s));
   } else {
     uint8_t* horigin = (uint8_t*)b;
     // gaps must stay untouched: bring the destination span in, scatter, send it back
     CU(cudaMemcpyAsync(dspan, horigin + lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, s));
     CU(cudaMemcpyAsync(dpack, a, (size_t)n, cudaMemcpyHostToDevice, s));
-    st = pack_common(true, t, count, dorigin, dpack, pos, &m, stream);
+    st = pack_common(true, t, count, dorigin, dpack, pos, &m, stream, false);
     if (st == DT_OK) CU(cudaMemcpyAsync(horigin + lo, dspan, (size_t)(hi - lo), cudaMemcpyDeviceToHost, s));
   }
-  g_check_ptrs = saved;
   if (st != DT_OK) return st;
   CU(cudaStreamSynchronize(s));
   return DT_OK;

@@ -228,6 +228,34 @@ def test_host_entry_points(torch_cuda):
     assert np.array_equal(dst, exp)
 
 
+@pytest.mark.parametrize("name", ["C2s", "C5", "C4x"])
+def test_host_entry_points_pinned(torch_cuda, name):
+    """Pinned host buffers: the kernels read/write host memory directly (zero-copy);
+    bit-exact vs the oracle, fragments, and host gap bytes untouched by unpack."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = {"C2s": lambda: c2_lower_triangle(700), "C5": lambda: c5_particles(56 * 5000),
+                        "C4x": lambda: c4_face("x+", 48)}[name]()
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    src_h = fill_bytes(parent, 15)
+    src = torch.from_numpy(src_h).pin_memory()
+    n = t.size
+    out = torch.full((n,), 0xA5, dtype=torch.uint8).pin_memory()
+    dt.pack_host(t, 1, src.data_ptr() + org, out.data_ptr(), stream=0)
+    exp = oracle.pack(ot, 1, src_h, org)
+    assert np.array_equal(out.numpy(), exp)
+    for a, b in ((0, n // 3), (n // 3, n - 5), (n - 5, n)):   # fragments at ragged positions
+        part = torch.full((b - a,), 0xA5, dtype=torch.uint8).pin_memory()
+        dt.pack_host(t, 1, src.data_ptr() + org, part.data_ptr(), a, b - a, stream=0)
+        assert np.array_equal(part.numpy(), exp[a:b])
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8).pin_memory()
+    dt.unpack_host(t, 1, out.data_ptr(), dst.data_ptr() + org, stream=0)
+    ref = np.full(parent, 0xA5, dtype=np.uint8)
+    oracle.unpack(ot, 1, exp, ref, org)
+    assert np.array_equal(dst.numpy(), ref)
+
+
 def test_full_size_sampled_c5_large(torch_cuda):
     """BASELINE sizes where the oracle cannot produce the whole stream quickly:
     compare sampled stream bytes against the oracle's per-position addresses."""
