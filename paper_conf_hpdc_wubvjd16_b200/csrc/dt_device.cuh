@@ -886,6 +886,304 @@ __device__ __forceinline__ void blk_range(const KP& P, uint8_t* cbase, int64_t p
   }
 }
 
+// ---------------------------------------------------------------- block spans
+// Short blocks of a large irregular block list (C5b: hindexed of 4..64-byte
+// blocks with 0..60-byte gaps; too many blocks for a word table).  A warp takes
+// the next 32 blocks of its slice as one window (lane i = block cb+i):
+//   * the window's descriptors (len, disp) arrive by cp.async into shared memory;
+//     its packed offsets are an inclusive warp-shuffle scan of the lengths (the
+//     paper's prefix-sum offsets, [L16:c5201 §3.2]) -- no boff[] traffic after
+//     the first block of the slice is found;
+//   * the window's layout span [lo, hi) is one warp-wide min/max reduction;
+//     when it fits kSpanBuf bytes the span moves as 16-byte chunks:
+//     pack:   cp.async (LDGSTS) of every span chunk into shared memory, a
+//             per-warp packed word map (span word of every packed word), then
+//             each lane assembles whole 16-byte packed chunks (coalesced
+//             stores; G-byte stores only at the window's two ends);
+//     unpack: cp.async of the packed window, a per-warp span word map (packed
+//             word of every covered span word), then each lane writes span
+//             chunks in address order -- one 16-byte store when the window
+//             covers the whole chunk, G-byte stores of the covered words
+//             otherwise (bytes outside the typemap are never written);
+//   * a wider span falls back to a warp-cooperative copy per block;
+//   * two-stage software pipeline: while window k is copied, the loads of window
+//     k+1 (its span or packed bytes) and the descriptors of window k+2 are in
+//     flight, so each window costs its copy work, not a DRAM round trip.
+// Every DRAM sector of the layout is requested once by a 16-byte access instead
+// of once per G-byte word (the per-word gathers of blk_range).
+constexpr int kSpanBuf = 4096;  // layout span bytes per window (multiple of 16)
+constexpr int kSpanOut = 2048;  // packed bytes per window (multiple of 16)
+constexpr int kSpanOutB = kSpanOut + 32;
+constexpr int kSpanDesc = 32 * 16;  // one window's (len, disp) pairs
+// per-warp shared memory: pack  = 2 spans + packed word map (G >= 4) + 2 descriptor sets;
+//                         unpack = 2 packed windows + span word map (G >= 4) + 2 descriptor sets
+constexpr int kSpanPackSmem = 2 * kSpanBuf + kSpanOutB / 2 + 2 * kSpanDesc;
+constexpr int kSpanUnpackSmem = 2 * kSpanOutB + (kSpanBuf / 4) * 2 + 2 * kSpanDesc;
+constexpr int kSpanWarpSmem = kSpanPackSmem > kSpanUnpackSmem ? kSpanPackSmem : kSpanUnpackSmem;
+
+// Move `n` bytes (a multiple of G) between the packed stream at global `g` and
+// shared memory at `s` with s == g (mod 16): G-byte head words up to 16-byte
+// alignment, 16-byte vectors, G-byte tail words.  TO_SMEM: g -> s by cp.async
+// (the caller commits and waits), else s -> g by stores.
+template <bool TO_SMEM, int G, int POL>
+__device__ __forceinline__ void span_window_io(uint8_t* g, uint8_t* s, int n, int lane) {
+  typedef typename WordT<G>::T W;
+  const int head = min(n, (int)((16 - ((uintptr_t)g & 15)) & 15));
+  const int hw = head / G;
+  if (lane < hw) {
+    if (TO_SMEM) cp_async<G>(s + lane * G, g + lane * G);
+    else reinterpret_cast<W*>(g)[lane] = reinterpret_cast<const W*>(s)[lane];
+  }
+  const int nv = (n - head) >> 4;
+  uint4* gv = reinterpret_cast<uint4*>(g + head);
+  uint4* sv = reinterpret_cast<uint4*>(s + head);
+  for (int i = lane; i < nv; i += 32) {
+    if (TO_SMEM) cp_async<16>(sv + i, gv + i);
+    else stv(gv + i, sv[i]);
+  }
+  const int tw = (n - head - nv * 16) / G;
+  if (lane < tw) {
+    W* gt = reinterpret_cast<W*>(g + head + nv * 16);
+    W* st = reinterpret_cast<W*>(s + head + nv * 16);
+    if (TO_SMEM) cp_async<G>(st + lane, gt + lane);
+    else gt[lane] = st[lane];
+  }
+}
+
+// Wide span (rare): warp-cooperative copy of each block of the window.  Not
+// inlined, so that the realigning copies' registers do not cap the fast path.
+template <bool UNPACK, int POL>
+__device__ __noinline__ void span_wide(int32_t n, int64_t a, int32_t off, uint8_t* cp, int lane) {
+  for (int j = 0; j < 32; j++) {
+    const int32_t nj = __shfl_sync(0xffffffffu, n, j);
+    if (nj == 0) break;
+    uint8_t* aj = reinterpret_cast<uint8_t*>(__shfl_sync(0xffffffffu, a, j));
+    uint8_t* pj = cp + __shfl_sync(0xffffffffu, off, j);
+    if (UNPACK) warp_copy<POL>(aj, pj, nj, lane);
+    else warp_copy<POL>(pj, aj, nj, lane);
+  }
+}
+
+// Block cursor of a warp: stream byte p is byte r of template block cb of element ce.
+struct SpanCur {
+  int64_t p, r, cb, ced;
+  uint64_t ce;
+};
+// Issue the descriptor loads of the window starting at the cursor into dsc
+// (lane i: block cb+i, wrapping into later elements); returns the lane's element.
+__device__ __forceinline__ uint64_t span_desc_issue(const KP& P, const SpanCur& c, int64_t* dsc, int lane) {
+  int64_t b = c.cb + lane;
+  uint64_t e = c.ce;
+  if (b >= P.nblocks) {
+    const uint64_t k = fdiv((uint64_t)b, P.fnb);
+    e += k;
+    b -= (int64_t)k * P.nblocks;
+  }
+  if (P.nblocks == 1) {
+    dsc[2 * lane] = P.bl0;
+    dsc[2 * lane + 1] = P.bd0;
+  } else {
+    cp_async<8>(dsc + 2 * lane, P.bl + b);
+    cp_async<8>(dsc + 2 * lane + 1, P.bd + b);
+  }
+  return e;
+}
+// One window's geometry (per lane: its block's share).
+struct SpanWin {
+  int64_t a;       // layout address of the lane's first byte (n > 0)
+  int64_t base16;  // layout span start, 16-byte aligned
+  uint8_t* cp;     // packed address of the window's first byte
+  int32_t off, n, L, nch;
+  bool fast;
+};
+// Window at cursor c from the landed descriptors; advances c past it.
+__device__ __forceinline__ SpanWin span_geom(const KP& P, SpanCur& c, uint64_t e, const int64_t* dsc,
+                                             uint8_t* cbase, int64_t p1, int lane) {
+  constexpr unsigned FULL = 0xffffffffu;
+  constexpr int32_t kClamp = 1 << 30;
+  SpanWin w;
+  const int64_t skip = lane == 0 ? c.r : 0;
+  // lengths clamped to 4 KiB for the 32-bit scan: a window never exceeds kSpanOut
+  const int32_t len = (int32_t)min(dsc[2 * lane] - skip, (int64_t)4096);
+  int32_t inc = len;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int32_t t = __shfl_up_sync(FULL, inc, d);
+    if (lane >= d) inc += t;
+  }
+  w.off = inc - len;
+  w.L = (int32_t)min((int64_t)min(kSpanOut, __shfl_sync(FULL, inc, 31)), p1 - c.p);
+  w.n = max(0, min(inc, w.L) - w.off);  // lanes with n > 0 are a prefix (lane 0 always)
+  w.a = 0;
+  if (w.n > 0) w.a = (int64_t)(uintptr_t)P.nc + (e == c.ce ? c.ced : elem_disp(P, e)) + dsc[2 * lane + 1] + skip;
+  const int64_t a0 = __shfl_sync(FULL, w.a, 0);
+  const int32_t rel = (int32_t)max((int64_t)-kClamp, min((int64_t)kClamp, w.a - a0));
+  int32_t rlo = w.n > 0 ? rel : INT32_MAX, rhi = w.n > 0 ? rel + w.n : INT32_MIN;
+#pragma unroll
+  for (int d = 16; d; d >>= 1) {
+    rlo = min(rlo, __shfl_xor_sync(FULL, rlo, d));
+    rhi = max(rhi, __shfl_xor_sync(FULL, rhi, d));
+  }
+  w.base16 = (a0 + rlo) & ~(int64_t)15;
+  const int64_t span = a0 + rhi - w.base16;
+  w.fast = span <= kSpanBuf;
+  w.nch = w.fast ? (int32_t)((span + 15) >> 4) : 0;
+  w.cp = cbase + c.p;
+  // advance the cursor past the window's L bytes
+  const int j = __popc(__ballot_sync(FULL, inc <= w.L));  // whole blocks consumed (a prefix of lanes)
+  const int32_t offj = __shfl_sync(FULL, w.off, j & 31);
+  c.p += w.L;
+  if (j == 32) {
+    c.cb += 32;
+    c.r = 0;
+  } else {
+    c.r = (j == 0 ? c.r : 0) + (w.L - offj);
+    c.cb += j;
+  }
+  if (c.cb >= P.nblocks) {
+    const uint64_t k = fdiv((uint64_t)c.cb, P.fnb);
+    c.ce += k;
+    c.cb -= (int64_t)k * P.nblocks;
+    c.ced = elem_disp(P, c.ce);
+  }
+  return w;
+}
+
+// One warp moves stream bytes [p, p1) (multiples of G); sm = kSpanWarpSmem bytes
+// of 16-byte-aligned shared memory owned by the warp.
+template <bool UNPACK, int G, int POL>
+__device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, int64_t p, const int64_t p1, int lane,
+                                           uint8_t* sm) {
+  typedef typename WordT<G>::T W;
+  constexpr int NWL = 16 / G;
+  if (p >= p1) return;
+  // shared-memory carve-up (see kSpanPackSmem / kSpanUnpackSmem)
+  uint8_t* buf0 = sm;  // pack: span 0 | unpack: packed window 0
+  uint8_t* buf1 = sm + (UNPACK ? kSpanOutB : kSpanBuf);
+  uint16_t* omap = reinterpret_cast<uint16_t*>(sm + 2 * kSpanBuf);  // pack: packed word map
+  uint16_t* wmap = reinterpret_cast<uint16_t*>(sm + 2 * kSpanOutB);  // unpack: span word map
+  int64_t* dsc0 =
+      reinterpret_cast<int64_t*>(sm + (UNPACK ? 2 * kSpanOutB + (kSpanBuf / 4) * 2 : 2 * kSpanBuf + kSpanOutB / 2));
+  int64_t* dsc1 = dsc0 + 64;
+  SpanCur c;
+  c.p = p;
+  c.ce = fdiv((uint64_t)p, P.ftsize);
+  c.r = p - (int64_t)c.ce * P.tsize;
+  c.cb = 0;
+  if (P.nblocks != 1) {
+    c.cb = warp_find_block(P.boff, P.nblocks, c.r, lane);
+    c.r -= __ldg(P.boff + c.cb);
+  }
+  c.ced = elem_disp(P, c.ce);
+  // prologue: window 0's descriptors, geometry, loads; window 1's descriptors
+  uint64_t e = span_desc_issue(P, c, dsc0, lane);
+  cp_async_commit();
+  cp_async_wait<0>();
+  __syncwarp();
+  SpanWin w = span_geom(P, c, e, dsc0, cbase, p1, lane);
+  auto issue = [&](const SpanWin& x, uint8_t* b) {
+    if (!x.fast) return;
+    if (UNPACK) {
+      span_window_io<true, G, POL>(x.cp, b + ((uintptr_t)x.cp & 15), x.L, lane);
+    } else {
+      for (int i = lane; i < x.nch; i += 32) cp_async<16>(b + 16 * i, reinterpret_cast<const void*>(x.base16 + 16 * i));
+    }
+  };
+  issue(w, buf0);
+  if (c.p < p1) e = span_desc_issue(P, c, dsc1, lane);
+  cp_async_commit();
+  int k = 0;
+  while (true) {
+    cp_async_wait<0>();  // window k's bytes and window k+1's descriptors have landed
+    __syncwarp();
+    uint8_t* bk = (k & 1) ? buf1 : buf0;
+    const bool more = c.p < p1;
+    SpanWin nx;
+    if (more) {
+      int64_t* dn = (k & 1) ? dsc0 : dsc1;  // window k+1's descriptors
+      nx = span_geom(P, c, e, dn, cbase, p1, lane);
+      issue(nx, (k & 1) ? buf0 : buf1);
+      if (c.p < p1) e = span_desc_issue(P, c, (k & 1) ? dsc1 : dsc0, lane);  // window k+2's
+      cp_async_commit();
+    }
+    // ---- copy window k
+    if (!w.fast) {
+      span_wide<UNPACK, POL>(w.n, w.a, w.off, w.cp, lane);
+    } else if (!UNPACK) {
+      // packed-word map: omap[word of the window's 16-byte-aligned packed range] =
+      // span word; then each lane assembles whole 16-byte packed chunks
+      const int ob = (int)((uintptr_t)w.cp & 15);
+      const int sw = (int)((w.a - w.base16) / G), ow = (ob + w.off) / G, nw = w.n / G;
+#pragma unroll 4
+      for (int i = 0; i < nw; i++) omap[ow + i] = (uint16_t)(sw + i);
+      __syncwarp();
+      const W* sp = reinterpret_cast<const W*>(bk);
+      const int w0 = ob / G, w1 = (ob + w.L) / G, nco = (ob + w.L + 15) >> 4;
+      uint8_t* c16 = reinterpret_cast<uint8_t*>((uintptr_t)w.cp & ~(uintptr_t)15);
+      for (int ch = lane; ch < nco; ch += 32) {
+        union {
+          uint16_t e[NWL];
+          typename WordT<2 * NWL>::T all;
+        } m;
+        m.all = reinterpret_cast<const typename WordT<2 * NWL>::T*>(omap)[ch];
+        union {
+          uint4 v;
+          W w[NWL];
+        } u;
+        const int wi = ch * NWL;
+        if (wi >= w0 && wi + NWL <= w1) {
+#pragma unroll
+          for (int i = 0; i < NWL; i++) u.w[i] = sp[m.e[i]];
+          stv(reinterpret_cast<uint4*>(c16 + 16 * ch), u.v);
+        } else {
+#pragma unroll
+          for (int i = 0; i < NWL; i++)
+            if (wi + i >= w0 && wi + i < w1) reinterpret_cast<W*>(c16 + 16 * ch)[i] = sp[m.e[i]];
+        }
+      }
+      __syncwarp();
+    } else {
+      const int ob = (int)((uintptr_t)w.cp & 15);
+      uint4* m4 = reinterpret_cast<uint4*>(wmap);  // 8 entries per 16-byte store
+      for (int i = lane; i < (w.nch * NWL + 7) / 8; i += 32) m4[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
+      __syncwarp();
+      const int sw = (int)((w.a - w.base16) / G), ow = (ob + w.off) / G, nw = w.n / G;
+#pragma unroll 4
+      for (int i = 0; i < nw; i++) wmap[sw + i] = (uint16_t)(ow + i);
+      __syncwarp();
+      const W* owp = reinterpret_cast<const W*>(bk);
+      for (int ch = lane; ch < w.nch; ch += 32) {
+        union {
+          uint16_t e[NWL];
+          typename WordT<2 * NWL>::T all;
+        } m;
+        m.all = reinterpret_cast<const typename WordT<2 * NWL>::T*>(wmap)[ch];
+        bool full = true;
+#pragma unroll
+        for (int i = 0; i < NWL; i++) full = full && m.e[i] != 0xFFFFu;
+        uint8_t* d = reinterpret_cast<uint8_t*>(w.base16 + 16 * ch);
+        if (full) {
+          union {
+            uint4 v;
+            W w[NWL];
+          } u;
+#pragma unroll
+          for (int i = 0; i < NWL; i++) u.w[i] = owp[m.e[i]];
+          stv(reinterpret_cast<uint4*>(d), u.v);
+        } else {
+#pragma unroll
+          for (int i = 0; i < NWL; i++)
+            if (m.e[i] != 0xFFFFu) reinterpret_cast<W*>(d)[i] = owp[m.e[i]];
+        }
+      }
+      __syncwarp();
+    }
+    if (!more) break;
+    w = nx;
+    k++;
+  }
+}
+
 // ---------------------------------------------------------------- record spans
 // Short blocks inside small dense records (C5's 56-of-64-byte particles; any
 // template whose blocks lie in a 16-byte-aligned span of <= 128 B that is at least

@@ -147,6 +147,19 @@ __global__ void __launch_bounds__(256) k_blk(const KP P) {
   blk_range<UNPACK, G, LD_CS>(P, P.c - P.pos, p, p1, lane, sa);
 }
 
+// block-span pack/unpack (short blocks of a large irregular list): warp w owns
+// stream bytes [pos + w*per_warp, ...) and walks them 32 blocks at a time
+template <bool UNPACK, int G>
+__global__ void __launch_bounds__(256, 2) k_span(const KP P) {
+  extern __shared__ __align__(16) uint8_t smem_span[];
+  const int lane = threadIdx.x & 31;
+  uint8_t* sm = smem_span + (threadIdx.x >> 5) * kSpanWarpSmem;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t p = P.pos + gw * P.per_warp;
+  const int64_t p1 = min(p + P.per_warp, P.pos + P.len);
+  span_range<UNPACK, G, LD_CS>(P, P.c - P.pos, p, p1, lane, sm);
+}
+
 // shared-memory staged pack/unpack (cp.async gathers / TMA bulk), CTA c owns a
 // contiguous run of 16 KiB tiles of the stream
 template <bool UNPACK, int G>
@@ -526,6 +539,7 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   if (force == 6 && rec_ok) return 6;
   if (force == 2 && word_ok) return 2;
   if (force == 3 && blk_ok) return 3;
+  if (force == 7 && g >= 4) return 7;
   if (force == 4 && stage_ok) return 4;
   if (force == 1) return 1;
   // short blocks / co-aligned runs up to 1 KiB: with >= 8-byte words the smem/TMA
@@ -534,6 +548,8 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   // short blocks in small dense records (C5 particles): whole-record 16-byte loads
   if (mean < 256.0 && rec_ok && !force) return 6;
   if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return stage_ok && g >= 8 ? 4 : 2;
+  // many short blocks (no word table): block spans with >= 4-byte words, else block windows
+  if (mean < 128.0 && g >= 4 && !force) return 7;
   if (mean < 128.0 && blk_ok) return 3;
   return 1;
 }
@@ -688,6 +704,34 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
       switch (g) { case 4: LS(false, 4); break; case 8: LS(false, 8); break; default: LS(false, 16); break; }
     }
 #undef LS
+  } else if (kind == 7) {
+    P.fnb = make_fd((uint64_t)P.nblocks);
+    const size_t smem = 8 * (size_t)kSpanWarpSmem;
+    static bool attr = false;
+    if (!attr) {
+      const void* fs[] = {(const void*)k_span<false, 4>, (const void*)k_span<false, 8>, (const void*)k_span<false, 16>,
+                          (const void*)k_span<true, 4>,  (const void*)k_span<true, 8>,  (const void*)k_span<true, 16>};
+      for (const void* fp : fs) cudaFuncSetAttribute(fp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      attr = true;
+    }
+    static int occ = 0;
+    if (!occ && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_span<false, 4>, 256, smem) != cudaSuccess ||
+                 occ < 1))
+      occ = 1;
+    const int64_t max_warps = (int64_t)sms * occ * 8;
+    int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
+    int64_t per = (len + nw - 1) / nw;
+    per = (per + 15) & ~int64_t(15);
+    nw = (len + per - 1) / per;
+    P.per_warp = per;
+    const unsigned grid = (unsigned)((nw + 7) / 8);
+#define LP(U, G) k_span<U, G><<<grid, 256, smem, s>>>(P)
+    if (unpack) {
+      switch (g) { case 4: LP(true, 4); break; case 8: LP(true, 8); break; default: LP(true, 16); break; }
+    } else {
+      switch (g) { case 4: LP(false, 4); break; case 8: LP(false, 8); break; default: LP(false, 16); break; }
+    }
+#undef LP
   } else if (kind == 3) {
     P.fnb = make_fd((uint64_t)P.nblocks);
     const int64_t max_warps = (int64_t)sms * 4 * 8;

@@ -170,7 +170,7 @@ def test_random_tiny_types(torch_cuda):
                 raise
 
 
-@pytest.mark.parametrize("kind", ["1", "2", "3", "4", "6"])
+@pytest.mark.parametrize("kind", ["1", "2", "3", "4", "6", "7"])
 @pytest.mark.parametrize("name", ["C1b", "C2s", "C3s", "C4x", "C4y", "C5", "C5b", "ctg"])
 def test_every_kernel_family(torch_cuda, kind, name, monkeypatch):
     """Every kernel family (1 warp segments, 2 word table, 3 block windows, 4 smem/TMA
@@ -321,5 +321,68 @@ def test_record_span_kernel(torch_cuda, name):
         total = count * size
         for _ in range(3):
             a = int(rng.integers(0, total // 16)) * 16
+            b = int(rng.integers(a // 4, total // 4 + 1)) * 4
+            check_pack_unpack(torch_cuda, rec, org, parent, count=count, pos=a, nbytes=b - a, seed=a)
+
+
+def _hindexed(lens, disp):
+    return ("hindexed", np.asarray(lens, dtype=np.int64), np.asarray(disp, dtype=np.int64), ("basic", "BYTE"))
+
+
+def _span_types():
+    rng = np.random.default_rng(77)
+    out = {}
+    # C5b-like blocks, typemap order != address order (shuffled within groups of 48 blocks)
+    n = 20000
+    lens = rng.integers(1, 17, n) * 4
+    gaps = rng.integers(0, 16, n) * 4
+    disp = np.concatenate([[0], np.cumsum(lens[:-1] + gaps[:-1])])
+    perm = np.concatenate([rng.permutation(48) + i for i in range(0, n - n % 48, 48)] + [np.arange(n - n % 48, n)])
+    out["shuffled4"] = (_hindexed(lens[perm], disp[perm]), 0, int(disp[-1] + lens[-1]))
+    # occasional 8 KiB jumps: windows alternate between the span path and the wide fallback
+    gaps2 = gaps.copy()
+    gaps2[::37] = 8192
+    disp2 = np.concatenate([[0], np.cumsum(lens[:-1] + gaps2[:-1])])
+    out["jumps4"] = (_hindexed(lens, disp2), 0, int(disp2[-1] + lens[-1]))
+    # 8- and 16-byte granular blocks (G = 8, 16)
+    for g in (8, 16):
+        l8 = rng.integers(1, 9, n) * g
+        g8 = rng.integers(0, 5, n) * g
+        d8 = np.concatenate([[0], np.cumsum(l8[:-1] + g8[:-1])])
+        out[f"gran{g}"] = (_hindexed(l8, d8), 0, int(d8[-1] + l8[-1]))
+    # negative and descending displacements (origin inside the buffer)
+    dd = -disp[:5000][::-1] - lens[:5000][::-1]
+    span = int(disp[4999] + lens[4999])
+    out["descending"] = (_hindexed(lens[:5000][::-1], dd), span, span + 64)
+    # small irregular template repeated (count > 1): windows wrap across elements
+    l3 = rng.integers(1, 9, 45) * 4
+    d3 = np.concatenate([[0], np.cumsum(l3[:-1] + 12)])
+    ext = int(d3[-1] + l3[-1] + 4)
+    out["repeat"] = (("resized", _hindexed(l3, d3), 0, ext), 0, ext)
+    return out
+
+
+SPAN_TYPES = _span_types()
+
+
+@pytest.mark.parametrize("name", sorted(SPAN_TYPES))
+def test_block_span_kernel(torch_cuda, name, monkeypatch):
+    """k_span (short blocks of a large irregular list): the planner's choice for C5b-like
+    lists; bit-exact on unsorted, descending and jumping displacements, G = 4/8/16,
+    element wrap-around inside a window (forced), and ragged pos/len."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = SPAN_TYPES[name]
+    t = dt.from_recipe(rec).commit()
+    if name == "repeat":
+        monkeypatch.setenv("DT_FORCE_KERNEL", "7")
+    else:
+        assert t.plan(1, 4096, 8192, 0, t.size)[0] == 7
+    size = t.size
+    check_pack_unpack(torch_cuda, rec, org, parent, seed=5)
+    rng = np.random.default_rng(11)
+    for count in (1, 3):
+        total = count * size
+        for _ in range(3):
+            a = int(rng.integers(0, total // 4)) * 4
             b = int(rng.integers(a // 4, total // 4 + 1)) * 4
             check_pack_unpack(torch_cuda, rec, org, parent, count=count, pos=a, nbytes=b - a, seed=a)

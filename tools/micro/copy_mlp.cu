@@ -20,6 +20,48 @@ __global__ void __launch_bounds__(256) vcopy(const uint4* __restrict__ a, uint4*
   for (; i < n; i += st) b[i] = a[i];
 }
 
+// read-only stream (sum of words; result stored only to defeat dead-code elimination)
+template <int U>
+__global__ void __launch_bounds__(256) vread(const uint4* __restrict__ a, uint4* __restrict__ b, int64_t n) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t st = (int64_t)gridDim.x * blockDim.x;
+  unsigned acc = 0;
+  for (; i + (U - 1) * st < n; i += U * st) {
+    uint4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) v[u] = __ldcs(a + i + u * st);
+#pragma unroll
+    for (int u = 0; u < U; u++) acc ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
+  }
+  if (acc == 0x12345678u) b[0] = make_uint4(acc, 0, 0, 0);
+}
+// software-pipelined copy: the loads of iteration k+1 are issued before the stores of k
+template <int U>
+__global__ void __launch_bounds__(256) vcopy_pipe(const uint4* __restrict__ a, uint4* __restrict__ b, int64_t n) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t st = (int64_t)gridDim.x * blockDim.x;
+  uint4 v[U], w[U];
+  if (i + (U - 1) * st >= n) { for (; i < n; i += st) b[i] = a[i]; return; }
+#pragma unroll
+  for (int u = 0; u < U; u++) v[u] = __ldcs(a + i + u * st);
+  for (;;) {
+    const int64_t j = i + U * st;
+    const bool more = j + (U - 1) * st < n;
+    if (more) {
+#pragma unroll
+      for (int u = 0; u < U; u++) w[u] = __ldcs(a + j + u * st);
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++) __stcs(b + i + u * st, v[u]);
+    i = j;
+    if (!more) break;
+#pragma unroll
+    for (int u = 0; u < U; u++) v[u] = w[u];
+  }
+  for (; i < n; i += st) b[i] = a[i];
+}
+__global__ void empty_k() {}
+
 __device__ __forceinline__ uint32_t sa(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 // each CTA: NB stages of CH bytes; thread 0 issues bulk loads, waits, issues bulk stores
 template <int NB>
@@ -95,6 +137,17 @@ int main() {
            er == cudaSuccess ? "" : cudaGetErrorString(er));
   };
   const int64_t nv = n / 16;
+  run("empty kernel", [&] { empty_k<<<sms, 256>>>(); });
+  run("cudaMemcpyAsync D2D 64 MiB", [&] { cudaMemcpyAsync(b, a, n, cudaMemcpyDeviceToDevice); });
+  for (int occ : {4, 8}) {
+    char nm[64];
+    snprintf(nm, 64, "vread U=8 grid=%d/SM (GB/s = 2x read)", occ);
+    run(nm, [&] { vread<8><<<sms * occ, 256>>>((const uint4*)a, (uint4*)b, nv); });
+    snprintf(nm, 64, "vcopy_pipe U=4 grid=%d/SM", occ);
+    run(nm, [&] { vcopy_pipe<4><<<sms * occ, 256>>>((const uint4*)a, (uint4*)b, nv); });
+    snprintf(nm, 64, "vcopy_pipe U=8 grid=%d/SM", occ);
+    run(nm, [&] { vcopy_pipe<8><<<sms * occ, 256>>>((const uint4*)a, (uint4*)b, nv); });
+  }
   for (int occ : {4, 8}) {
     char nm[64];
     snprintf(nm, 64, "vcopy U=4 grid=%d/SM", occ);
