@@ -324,10 +324,11 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup, 
     import torch
 
     from paper_conf_hpdc_wubvjd16_b200 import dt
-    from workloads import c3_block_cyclic, c5_particles, fill_bytes, seed_for
+    from workloads import c3_block_cyclic, c5_particles, c5b_irregular, fill_bytes, seed_for
     dev = torch.device("cuda", local)
     peer = rank ^ 1 if (rank ^ 1) < ws else rank
-    rec, org, parent = c3_block_cyclic() if workload == "c3" else c5_particles(128 << 20)
+    rec, org, parent = {"c3": c3_block_cyclic, "c5": lambda: c5_particles(128 << 20),
+                        "c5b": lambda: c5b_irregular(128 << 20)}[workload]()
     t = dt.from_recipe(rec).commit()
     payload = t.size
     A = torch.from_numpy(fill_bytes(parent, seed_for(3) + rank)).to(dev)
@@ -426,7 +427,9 @@ def run_xfer(args):
             "warmup": args.warmup, "ms_per_step": best["ms"], "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
             "config": {"workload": ("C3: ScaLAPACK 2D block-cyclic submatrix (N=8192 f64, nb=64, owner (0,1))"
-                                    if args.xfer_workload == "c3" else "C5: 128 MiB of LAMMPS-style particles")
+                                    if args.xfer_workload == "c3" else "C5: 128 MiB of LAMMPS-style particles"
+                                    if args.xfer_workload == "c5" else
+                                    "C5b: 128 MiB irregular hindexed (4..64-byte blocks, 0..60-byte gaps)")
                                    + f", pairwise exchange, mode={args.xfer_mode}",
                        "payload_bytes": payload, "sweep": results, "spot_parity": ok,
                        "fused_loopback_gbs_per_rank": fused,
@@ -656,7 +659,7 @@ def main():
     ap.add_argument("--sweep", default="all", help="--workload sweep: comma-separated config names or 'all'")
     ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "direct"],
                     help="p2p ring pipeline, NCCL double buffering, or a persistent direct plan (dt_xplan)")
-    ap.add_argument("--xfer-workload", default="c3", choices=["c3", "c5"])
+    ap.add_argument("--xfer-workload", default="c3", choices=["c3", "c5", "c5b"])
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
     ap.add_argument("--xfer-depths", default="2,4")
     ap.add_argument("--xfer-ctas", type=int, default=0, help="CTAs per direction (0 = library default)")

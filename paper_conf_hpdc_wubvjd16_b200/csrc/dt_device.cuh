@@ -931,7 +931,8 @@ __device__ __forceinline__ void span_window_io(uint8_t* g, uint8_t* s, int n, in
   const int head = min(n, (int)((16 - ((uintptr_t)g & 15)) & 15));
   const int hw = head / G;
   if (lane < hw) {
-    if (TO_SMEM) cp_async<G>(s + lane * G, g + lane * G);
+    if (TO_SMEM && POL == LD_CG) reinterpret_cast<W*>(s)[lane] = __ldcg(reinterpret_cast<const W*>(g) + lane);
+    else if (TO_SMEM) cp_async<G>(s + lane * G, g + lane * G);
     else reinterpret_cast<W*>(g)[lane] = reinterpret_cast<const W*>(s)[lane];
   }
   const int nv = (n - head) >> 4;
@@ -945,7 +946,8 @@ __device__ __forceinline__ void span_window_io(uint8_t* g, uint8_t* s, int n, in
   if (lane < tw) {
     W* gt = reinterpret_cast<W*>(g + head + nv * 16);
     W* st = reinterpret_cast<W*>(s + head + nv * 16);
-    if (TO_SMEM) cp_async<G>(st + lane, gt + lane);
+    if (TO_SMEM && POL == LD_CG) st[lane] = __ldcg(gt + lane);
+    else if (TO_SMEM) cp_async<G>(st + lane, gt + lane);
     else gt[lane] = st[lane];
   }
 }
@@ -962,6 +964,19 @@ __device__ __noinline__ void span_wide(int32_t n, int64_t a, int32_t off, uint8_
     if (UNPACK) warp_copy<POL>(aj, pj, nj, lane);
     else warp_copy<POL>(pj, aj, nj, lane);
   }
+}
+
+// m[at + i] = val + i for i < n, two entries per 4-byte store
+__device__ __forceinline__ void map_fill(uint16_t* m, int at, int val, int n) {
+  int i = 0;
+  if ((at & 1) && n > 0) {
+    m[at] = (uint16_t)val;
+    i = 1;
+  }
+#pragma unroll 4
+  for (; i + 1 < n; i += 2)
+    *reinterpret_cast<uint32_t*>(m + at + i) = (uint32_t)(val + i) | ((uint32_t)(val + i + 1) << 16);
+  if (i < n) m[at + i] = (uint16_t)(val + i);
 }
 
 // Block cursor of a warp: stream byte p is byte r of template block cb of element ce.
@@ -1049,14 +1064,31 @@ __device__ __forceinline__ SpanWin span_geom(const KP& P, SpanCur& c, uint64_t e
   return w;
 }
 
-// One warp moves stream bytes [p, p1) (multiples of G); sm = kSpanWarpSmem bytes
-// of 16-byte-aligned shared memory owned by the warp.
+// start of a warp's slice at stream byte p (a 32-ary block search; the standalone
+// kernel takes it from a cached plan instead)
+__device__ __forceinline__ PlanEnt span_start(const KP& P, int64_t p, int lane) {
+  PlanEnt s;
+  s.p = p;
+  s.e = (int64_t)fdiv((uint64_t)p, P.ftsize);
+  s.r = p - s.e * P.tsize;
+  s.b = 0;
+  if (P.nblocks != 1) {
+    s.b = warp_find_block(P.boff, P.nblocks, s.r, lane);
+    s.r -= __ldg(P.boff + s.b);
+  }
+  s.ed = elem_disp(P, (uint64_t)s.e);
+  return s;
+}
+
+// One warp moves stream bytes [start.p, p1) (multiples of G; start = block b, byte
+// r, element e of the plan); sm = kSpanWarpSmem bytes of 16-byte-aligned shared
+// memory owned by the warp.
 template <bool UNPACK, int G, int POL>
-__device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, int64_t p, const int64_t p1, int lane,
-                                           uint8_t* sm) {
+__device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, const PlanEnt& start, const int64_t p1,
+                                           int lane, uint8_t* sm) {
   typedef typename WordT<G>::T W;
   constexpr int NWL = 16 / G;
-  if (p >= p1) return;
+  if (start.p >= p1) return;
   // shared-memory carve-up (see kSpanPackSmem / kSpanUnpackSmem)
   uint8_t* buf0 = sm;  // pack: span 0 | unpack: packed window 0
   uint8_t* buf1 = sm + (UNPACK ? kSpanOutB : kSpanBuf);
@@ -1065,16 +1097,12 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, int64_t 
   int64_t* dsc0 =
       reinterpret_cast<int64_t*>(sm + (UNPACK ? 2 * kSpanOutB + (kSpanBuf / 4) * 2 : 2 * kSpanBuf + kSpanOutB / 2));
   int64_t* dsc1 = dsc0 + 64;
-  SpanCur c;
-  c.p = p;
-  c.ce = fdiv((uint64_t)p, P.ftsize);
-  c.r = p - (int64_t)c.ce * P.tsize;
-  c.cb = 0;
-  if (P.nblocks != 1) {
-    c.cb = warp_find_block(P.boff, P.nblocks, c.r, lane);
-    c.r -= __ldg(P.boff + c.cb);
-  }
-  c.ced = elem_disp(P, c.ce);
+  SpanCur c;  // the warp's start, resolved by k_plan
+  c.p = start.p;
+  c.ce = (uint64_t)start.e;
+  c.r = start.r;
+  c.cb = start.b;
+  c.ced = start.ed;
   // prologue: window 0's descriptors, geometry, loads; window 1's descriptors
   uint64_t e = span_desc_issue(P, c, dsc0, lane);
   cp_async_commit();
@@ -1114,8 +1142,7 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, int64_t 
       // span word; then each lane assembles whole 16-byte packed chunks
       const int ob = (int)((uintptr_t)w.cp & 15);
       const int sw = (int)((w.a - w.base16) / G), ow = (ob + w.off) / G, nw = w.n / G;
-#pragma unroll 4
-      for (int i = 0; i < nw; i++) omap[ow + i] = (uint16_t)(sw + i);
+      map_fill(omap, ow, sw, nw);
       __syncwarp();
       const W* sp = reinterpret_cast<const W*>(bk);
       const int w0 = ob / G, w1 = (ob + w.L) / G, nco = (ob + w.L + 15) >> 4;
@@ -1148,8 +1175,7 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, int64_t 
       for (int i = lane; i < (w.nch * NWL + 7) / 8; i += 32) m4[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
       __syncwarp();
       const int sw = (int)((w.a - w.base16) / G), ow = (ob + w.off) / G, nw = w.n / G;
-#pragma unroll 4
-      for (int i = 0; i < nw; i++) wmap[sw + i] = (uint16_t)(ow + i);
+      map_fill(wmap, sw, ow, nw);
       __syncwarp();
       const W* owp = reinterpret_cast<const W*>(bk);
       for (int ch = lane; ch < w.nch; ch += 32) {

@@ -96,7 +96,7 @@ struct DeviceDesc {
   int32_t* wtab[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
   // cached cost-balanced warp plans of the long-run kernel, keyed by the launch shape
   struct PlanSlot {
-    int64_t count = -1, pos = 0, len = 0, nw = 0, alpha = 0, tsize = 0;
+    int64_t count = -1, pos = 0, len = 0, nw = 0, alpha = 0, tsize = 0, gran = 1;
     void* d = nullptr;
   };
   std::vector<PlanSlot> plans;

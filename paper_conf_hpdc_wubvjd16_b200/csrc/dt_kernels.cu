@@ -123,12 +123,19 @@ __global__ void __launch_bounds__(256, 3) k_seg_eq(const KP P, int64_t per) {
 }
 
 // one thread per warp boundary: cost-balanced cut positions (see PlanEnt)
+// (gran > 1: cuts rounded down to multiples of gran bytes -- the block-span kernel
+// moves whole G-byte words)
 __global__ void k_plan(const KP P, int64_t alpha, FastDiv fce, int64_t ce, int64_t C0, int64_t C1, int64_t nw,
-                       PlanEnt* plan) {
+                       int64_t gran, PlanEnt* plan) {
   const int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (w > nw) return;
   const int64_t C = w == nw ? C1 : C0 + (int64_t)((__int128)(C1 - C0) * w / nw);
   PlanEnt r = pos_of_cost(P, alpha, fce, ce, C);
+  if (gran > 1) {
+    const int64_t d = r.r % gran;
+    r.r -= d;
+    r.p -= d;
+  }
   const int64_t end = P.pos + P.len;
   if (w == nw || r.p > end) r.p = end;
   if (r.p < P.pos) r.p = P.pos;
@@ -150,14 +157,14 @@ __global__ void __launch_bounds__(256) k_blk(const KP P) {
 // block-span pack/unpack (short blocks of a large irregular list): warp w owns
 // stream bytes [pos + w*per_warp, ...) and walks them 32 blocks at a time
 template <bool UNPACK, int G>
-__global__ void __launch_bounds__(256, 2) k_span(const KP P) {
+__global__ void __launch_bounds__(256, 2) k_span(const KP P, const PlanEnt* __restrict__ plan, int64_t nw) {
   extern __shared__ __align__(16) uint8_t smem_span[];
   const int lane = threadIdx.x & 31;
   uint8_t* sm = smem_span + (threadIdx.x >> 5) * kSpanWarpSmem;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t p = P.pos + gw * P.per_warp;
-  const int64_t p1 = min(p + P.per_warp, P.pos + P.len);
-  span_range<UNPACK, G, LD_CS>(P, P.c - P.pos, p, p1, lane, sm);
+  if (gw >= nw) return;
+  const PlanEnt a = plan[gw];
+  span_range<UNPACK, G, LD_CS>(P, P.c - P.pos, a, plan[gw + 1].p, lane, sm);
 }
 
 // shared-memory staged pack/unpack (cp.async gathers / TMA bulk), CTA c owns a
@@ -440,12 +447,12 @@ static int64_t host_cost(const KP& P, const Form& f, int64_t alpha, int64_t p) {
 
 // cached (or freshly computed) cost-balanced plan for this launch shape
 static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& dd, int64_t count, int64_t nw,
-                          cudaStream_t s, const PlanEnt** out) {
-  const int64_t alpha = seg_alpha();
+                          cudaStream_t s, const PlanEnt** out, int64_t alpha = -1, int64_t gran = 1) {
+  if (alpha < 0) alpha = seg_alpha();
   std::lock_guard<std::mutex> g(t->mu);
   for (auto& sl : dd.plans) {
     if (sl.d && sl.count == count && sl.pos == P.pos && sl.len == P.len && sl.nw == nw && sl.alpha == alpha &&
-        sl.tsize == P.tsize) {
+        sl.tsize == P.tsize && sl.gran == gran) {
       *out = (const PlanEnt*)sl.d;
       return DT_OK;
     }
@@ -467,13 +474,14 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
   const int64_t ce = P.tsize + alpha * P.nblocks;
   const int64_t C0 = host_cost(P, f, alpha, P.pos), C1 = host_cost(P, f, alpha, P.pos + P.len);
   k_plan<<<(unsigned)((nw + 1 + 255) / 256), 256, 0, s>>>(P, alpha, make_fd((uint64_t)ce), ce, C0, C1, nw,
-                                                          (PlanEnt*)sl.d);
+                                                          gran, (PlanEnt*)sl.d);
   CU(cudaGetLastError());
   sl.count = count;
   sl.pos = P.pos;
   sl.len = P.len;
   sl.nw = nw;
   sl.alpha = alpha;
+  sl.gran = gran;
   sl.tsize = P.tsize;
   *out = (const PlanEnt*)sl.d;
   return DT_OK;
@@ -718,14 +726,15 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     if (!occ && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_span<false, 4>, 256, smem) != cudaSuccess ||
                  occ < 1))
       occ = 1;
+    // equal byte slices (alpha 0) cut at word boundaries, resolved once per launch
+    // shape by k_plan and cached on the type (no per-warp block search)
     const int64_t max_warps = (int64_t)sms * occ * 8;
-    int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
-    int64_t per = (len + nw - 1) / nw;
-    per = (per + 15) & ~int64_t(15);
-    nw = (len + per - 1) / per;
-    P.per_warp = per;
+    const int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (len + 4095) / 4096));
+    const PlanEnt* plan = nullptr;
+    dt_status pst = get_plan(t, P, f, dd, count, nw, s, &plan, 0, g);
+    if (pst != DT_OK) return pst;
     const unsigned grid = (unsigned)((nw + 7) / 8);
-#define LP(U, G) k_span<U, G><<<grid, 256, smem, s>>>(P)
+#define LP(U, G) k_span<U, G><<<grid, 256, smem, s>>>(P, plan, nw)
     if (unpack) {
       switch (g) { case 4: LP(true, 4); break; case 8: LP(true, 8); break; default: LP(true, 16); break; }
     } else {

@@ -45,7 +45,7 @@ constexpr uint64_t kAbort = 1ull << 63;
 struct XOp {
   KP P;            // pack (send role) or unpack (recv role) over the user's layout
   int32_t role;    // 0 send, 1 recv
-  int32_t kind;    // 1 segment walk, 2 word table, 4 smem/TMA staging, 6 record spans
+  int32_t kind;    // 1 segment walk, 2 word table, 4 smem/TMA staging, 6 record spans, 7 block spans
   int32_t single;  // segment walk over a single-block template
   int32_t g;       // word granularity
   int64_t n;       // send: bytes; recv: capacity in bytes
@@ -101,6 +101,24 @@ __device__ __forceinline__ void cta_chunk(const XOp& X, uint8_t* cb, int64_t lo,
       }
     }
     if (hb < hi && w == nwc - 1) seg_range<UNPACK, false, POL>(P, cb, hb, hi, lane);
+    return;
+  }
+  if (X.kind == 7) {  // block spans: the CTA's warps take equal 16-byte-multiple slices of the fragment
+    const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t body = len - len % X.g;  // a ragged tail (< G bytes, last fragment) is walked below
+    int64_t per = (body + nwc - 1) / nwc;
+    per = (per + 15) & ~int64_t(15);
+    const int64_t a = lo + (int64_t)w * per, b = min(a + per, lo + body);
+    if (a < b) {
+      const PlanEnt st = span_start(P, a, lane);
+      uint8_t* sm = sbuf + (size_t)w * kSpanWarpSmem;
+      switch (X.g) {
+        case 4: span_range<UNPACK, 4, POL>(P, cb, st, b, lane, sm); break;
+        case 8: span_range<UNPACK, 8, POL>(P, cb, st, b, lane, sm); break;
+        default: span_range<UNPACK, 16, POL>(P, cb, st, b, lane, sm); break;
+      }
+    }
+    if (body < len && w == nwc - 1) seg_range<UNPACK, false, POL>(P, cb, lo + body, hi, lane);
     return;
   }
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
@@ -649,10 +667,12 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
     if (!rec_geometry(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, g, &X.rg) || getenv("DT_XFER_NOREC"))
       kind = g >= 8 ? 4 : 2;
   }
-  if ((kind == 2 || kind == 4 || kind == 6) && lowp2u((uint64_t)chunk) < g) kind = 1;
+  if ((kind == 2 || kind == 4 || kind == 6 || kind == 7) && lowp2u((uint64_t)chunk) < g) kind = 1;
   if (kind == 4 && g < 8) kind = 2;
+  if (kind == 7 && getenv("DT_XFER_NOSPAN")) kind = 1;
   // the block-window kernel (3) is not used inside the pipeline
-  X.kind = (kind == 2 || kind == 4 || kind == 6) ? kind : 1;
+  X.kind = (kind == 2 || kind == 4 || kind == 6 || kind == 7) ? kind : 1;
+  if (X.kind == 7) P.fnb = make_fd((uint64_t)P.nblocks);
   X.single = P.nblocks == 1;
   X.g = (int32_t)g;
   if (X.kind == 2 || X.kind == 4) {
@@ -716,6 +736,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
       any_stage = any_stage || X.kind == 4;
       if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
+      if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)(kXferThreads / 32) * kSpanWarpSmem);
     }
     if (p.source >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
@@ -744,6 +765,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
       any_stage = any_stage || X.kind == 4;
       if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
+      if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)(kXferThreads / 32) * kSpanWarpSmem);
     }
   }
   if (nops == 0) return DT_OK;

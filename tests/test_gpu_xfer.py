@@ -430,3 +430,25 @@ def test_ring_record_spans(torch_cuda, chunk):
         _loop_check(torch_cuda, comm, ctg, 0, 2 * size, rec, org, parent + ext, scount=1, rcount=2)
         _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
     comm.free()
+
+
+@pytest.mark.parametrize("chunk", [16 << 10, 1 << 20])
+def test_ring_block_spans(torch_cuda, chunk):
+    """Block-span fragments inside the ring pipeline (C5b-like irregular lists of short
+    blocks: 32-block windows per warp, span loads, packed/span word maps) against a
+    contiguous peer in both directions and type to itself, count 2 (element wrap)."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from tests.test_gpu_parity import SPAN_TYPES
+    from workloads import c5b_irregular
+    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=2, ring_loopback=True)
+    cases = dict(SPAN_TYPES)
+    cases["c5b"] = c5b_irregular(3 << 20)
+    for name in sorted(cases):
+        rec, org, parent = cases[name]
+        size = oracle.from_recipe(rec).size
+        ext = oracle.from_recipe(rec).extent
+        ctg = ("contiguous", 2 * size, ("basic", "BYTE"))
+        _loop_check(torch_cuda, comm, rec, org, parent + ext, ctg, 0, 2 * size, scount=2, rcount=1)
+        _loop_check(torch_cuda, comm, ctg, 0, 2 * size, rec, org, parent + ext, scount=1, rcount=2)
+        _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
+    comm.free()
