@@ -896,19 +896,20 @@ __device__ __forceinline__ void blk_range(const KP& P, uint8_t* cbase, int64_t p
 //     the first block of the slice is found;
 //   * the window's layout span [lo, hi) is one warp-wide min/max reduction;
 //     when it fits kSpanBuf bytes the span moves as 16-byte chunks:
-//     pack:   cp.async (LDGSTS) of every span chunk into shared memory, a
+//     pack:   the span's 16-byte chunks land in shared memory, a
 //             per-warp packed word map (span word of every packed word), then
 //             each lane assembles whole 16-byte packed chunks (coalesced
 //             stores; G-byte stores only at the window's two ends);
-//     unpack: cp.async of the packed window, a per-warp span word map (packed
+//     unpack: the packed window lands in shared memory, a per-warp span word map (packed
 //             word of every covered span word), then each lane writes span
 //             chunks in address order -- one 16-byte store when the window
 //             covers the whole chunk, G-byte stores of the covered words
 //             otherwise (bytes outside the typemap are never written);
 //   * a wider span falls back to a warp-cooperative copy per block;
 //   * two-stage software pipeline: while window k is copied, the loads of window
-//     k+1 (its span or packed bytes) and the descriptors of window k+2 are in
-//     flight, so each window costs its copy work, not a DRAM round trip.
+//     k+1 (its span or packed bytes: ONE TMA bulk copy, completion on an mbarrier)
+//     and the descriptors of window k+2 are in flight, so each window costs its
+//     copy work, not a DRAM round trip.
 // Every DRAM sector of the layout is requested once by a 16-byte access instead
 // of once per G-byte word (the per-word gathers of blk_range).
 constexpr int kSpanBuf = 4096;  // layout span bytes per window (multiple of 16)
@@ -917,8 +918,9 @@ constexpr int kSpanOutB = kSpanOut + 32;
 constexpr int kSpanDesc = 32 * 16;  // one window's (len, disp) pairs
 // per-warp shared memory: pack  = 2 spans + packed word map (G >= 4) + 2 descriptor sets;
 //                         unpack = 2 packed windows + span word map (G >= 4) + 2 descriptor sets
-constexpr int kSpanPackSmem = 2 * kSpanBuf + kSpanOutB / 2 + 2 * kSpanDesc;
-constexpr int kSpanUnpackSmem = 2 * kSpanOutB + (kSpanBuf / 4) * 2 + 2 * kSpanDesc;
+// (+ 2 mbarriers, at the end)
+constexpr int kSpanPackSmem = 2 * kSpanBuf + kSpanOutB / 2 + 2 * kSpanDesc + 16;
+constexpr int kSpanUnpackSmem = 2 * kSpanOutB + (kSpanBuf / 4) * 2 + 2 * kSpanDesc + 16;
 constexpr int kSpanWarpSmem = kSpanPackSmem > kSpanUnpackSmem ? kSpanPackSmem : kSpanUnpackSmem;
 
 // Move `n` bytes (a multiple of G) between the packed stream at global `g` and
@@ -1097,6 +1099,14 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, const Pl
   int64_t* dsc0 =
       reinterpret_cast<int64_t*>(sm + (UNPACK ? 2 * kSpanOutB + (kSpanBuf / 4) * 2 : 2 * kSpanBuf + kSpanOutB / 2));
   int64_t* dsc1 = dsc0 + 64;
+  uint64_t* mb = reinterpret_cast<uint64_t*>(sm + kSpanWarpSmem - 16);  // one per span/window buffer
+  if (lane == 0) {
+    mbar_init(mb, 1);
+    mbar_init(mb + 1, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  uint32_t phase = 0;  // bit s: parity of the next completion of buffer s
   SpanCur c;  // the warp's start, resolved by k_plan
   c.p = start.p;
   c.ce = (uint64_t)start.e;
@@ -1109,20 +1119,32 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, const Pl
   cp_async_wait<0>();
   __syncwarp();
   SpanWin w = span_geom(P, c, e, dsc0, cbase, p1, lane);
-  auto issue = [&](const SpanWin& x, uint8_t* b) {
-    if (!x.fast) return;
+  // one TMA bulk copy (UBLKCP) per window: the layout span (pack) or the 16-byte-aligned
+  // hull of the packed window (unpack; buffer + (cp & 15) == cp mod 16), completion on mb[st]
+  auto issue = [&](const SpanWin& x, uint8_t* b, int st) {
+    if (!x.fast || lane != 0) return;
+    const uint8_t* src;
+    uint32_t bytes;
     if (UNPACK) {
-      span_window_io<true, G, POL>(x.cp, b + ((uintptr_t)x.cp & 15), x.L, lane);
+      src = reinterpret_cast<const uint8_t*>((uintptr_t)x.cp & ~(uintptr_t)15);
+      bytes = (uint32_t)((((uintptr_t)x.cp & 15) + x.L + 15) & ~15);
     } else {
-      for (int i = lane; i < x.nch; i += 32) cp_async<16>(b + 16 * i, reinterpret_cast<const void*>(x.base16 + 16 * i));
+      src = reinterpret_cast<const uint8_t*>(x.base16);
+      bytes = (uint32_t)x.nch * 16u;
     }
+    mbar_expect_tx(mb + st, bytes);
+    bulk_load(b, src, bytes, mb + st);
   };
-  issue(w, buf0);
+  issue(w, buf0, 0);
   if (c.p < p1) e = span_desc_issue(P, c, dsc1, lane);
   cp_async_commit();
   int k = 0;
   while (true) {
-    cp_async_wait<0>();  // window k's bytes and window k+1's descriptors have landed
+    cp_async_wait<0>();  // window k+1's descriptors have landed
+    if (w.fast) {        // window k's bytes
+      mbar_wait(mb + (k & 1), (phase >> (k & 1)) & 1u);
+      phase ^= 1u << (k & 1);
+    }
     __syncwarp();
     uint8_t* bk = (k & 1) ? buf1 : buf0;
     const bool more = c.p < p1;
@@ -1130,7 +1152,7 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, const Pl
     if (more) {
       int64_t* dn = (k & 1) ? dsc0 : dsc1;  // window k+1's descriptors
       nx = span_geom(P, c, e, dn, cbase, p1, lane);
-      issue(nx, (k & 1) ? buf0 : buf1);
+      issue(nx, (k & 1) ? buf0 : buf1, (k + 1) & 1);
       if (c.p < p1) e = span_desc_issue(P, c, (k & 1) ? dsc1 : dsc0, lane);  // window k+2's
       cp_async_commit();
     }
@@ -1208,6 +1230,14 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, const Pl
     w = nx;
     k++;
   }
+  // the warp's smem may be re-carved by its next call (next ring fragment): retire the
+  // mbarriers (an mbarrier must be invalidated before its memory is re-initialised)
+  __syncwarp();
+  if (lane == 0) {
+    asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(mb)) : "memory");
+    asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(mb + 1)) : "memory");
+  }
+  __syncwarp();
 }
 
 // ---------------------------------------------------------------- record spans
