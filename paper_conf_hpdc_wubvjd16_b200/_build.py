@@ -50,6 +50,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
             cmd[1:1] = ["-x", "cu"]
         if os.environ.get("DT_PTXAS_V"):
             cmd += ["-Xptxas", "-v"]
+        if os.environ.get("DT_NVCC_FLAGS"):  # tuning experiments, e.g. -DDT_STORE_WB=1
+            cmd += os.environ["DT_NVCC_FLAGS"].split()
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
         cmds.append(cmd)

@@ -82,9 +82,13 @@ __device__ __forceinline__ V ldv(const V* p) {
   if (POL == LD_CG) return __ldcg(p);
   return __ldcs(p);
 }
+#ifndef DT_STORE_WB
+#define DT_STORE_WB 0
+#endif
 template <typename V>
 __device__ __forceinline__ void stv(V* p, const V& v) {
-  __stcs(p, v);
+  if (DT_STORE_WB) *p = v;  // write-back (L2-allocating) stores
+  else __stcs(p, v);        // streaming (evict-first) stores
 }
 
 // Copy n bytes with the whole warp, vector width V chosen from the relative
