@@ -458,7 +458,7 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
     }
   }
   size_t idx;
-  if (dd.plans.size() < 16) {
+  if (dd.plans.size() < 64) {  // (a host-link pipeline uses one plan per chunk)
     dd.plans.emplace_back();
     idx = dd.plans.size() - 1;
   } else {
@@ -1188,6 +1188,80 @@ static dt_status scratch(int i, size_t n, void** out) {
   return DT_OK;
 }
 
+// Host-link pipeline for pinned buffers: the SMs move the layout side over the host link
+// (zero-copy gather from / scatter to the pinned origin, into / out of a device ring of
+// chunks) while the copy engine moves the packed side chunk by chunk in the other
+// direction -- the paper's pipelining of pack with the transfer ([L18:c4394 §4.1]) applied
+// to the host link.  Measured on B200 (tools/micro/zerocopy.cu): a kernel that reads and
+// writes host memory at once tops out at ~74-79 GB/s, a zero-copy read (51 GB/s) or write
+// (52 GB/s) next to a copy-engine copy the other way is not capped that way (two memcpys:
+// 99 GB/s).  Chunk C = DT_HOST_CHUNK (default 4 MiB), 3 ring slots; DT_HOST_PIPE=0 keeps the
+// single zero-copy kernel for both directions.  Ordered after the caller's stream; synchronous like the rest of
+// the host entry points.
+struct HostPipe {
+  int dev = -1;
+  cudaStream_t ks = nullptr, cs = nullptr;
+  cudaEvent_t ev_start = nullptr, ev_k[3] = {}, ev_c[3] = {}, ev_end[2] = {};
+};
+static HostPipe g_hp;
+
+static dt_status host_pipe(bool unpack, dt_t t, int64_t count, uint8_t* dorig, uint8_t* hpk, int64_t pos, int64_t n,
+                           cudaStream_t us) {
+  constexpr int D = 3;
+  const int64_t C = getenv("DT_HOST_CHUNK") ? std::max<int64_t>(4096, atoll(getenv("DT_HOST_CHUNK")) & ~int64_t(4095))
+                                                   : (int64_t)4 << 20;
+  int dev = 0;
+  CU(cudaGetDevice(&dev));
+  if (g_hp.dev != dev) {
+    CU(cudaStreamCreateWithFlags(&g_hp.ks, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&g_hp.cs, cudaStreamNonBlocking));
+    CU(cudaEventCreateWithFlags(&g_hp.ev_start, cudaEventDisableTiming));
+    for (int i = 0; i < D; i++) {
+      CU(cudaEventCreateWithFlags(&g_hp.ev_k[i], cudaEventDisableTiming));
+      CU(cudaEventCreateWithFlags(&g_hp.ev_c[i], cudaEventDisableTiming));
+    }
+    for (int i = 0; i < 2; i++) CU(cudaEventCreateWithFlags(&g_hp.ev_end[i], cudaEventDisableTiming));
+    g_hp.dev = dev;
+  }
+  void* ring = nullptr;
+  dt_status st = scratch(1, (size_t)(D * C), &ring);
+  if (st != DT_OK) return st;
+  uint8_t* rb = (uint8_t*)ring;
+  const cudaStream_t ks = g_hp.ks, cs = g_hp.cs;
+  CU(cudaEventRecord(g_hp.ev_start, us));
+  CU(cudaStreamWaitEvent(ks, g_hp.ev_start, 0));
+  CU(cudaStreamWaitEvent(cs, g_hp.ev_start, 0));
+  const int64_t nk = (n + C - 1) / C;
+  for (int64_t k = 0; k < nk; k++) {
+    const int slot = (int)(k % D);
+    int64_t m = std::min(C, n - k * C);
+    uint8_t* sl = rb + (size_t)slot * C;
+    if (!unpack) {
+      if (k >= D) CU(cudaStreamWaitEvent(ks, g_hp.ev_c[slot], 0));  // slot's previous D2H done
+      st = pack_common(false, t, count, dorig, sl, pos + k * C, &m, ks, /*check_ptrs=*/false);
+      if (st != DT_OK) return st;
+      CU(cudaEventRecord(g_hp.ev_k[slot], ks));
+      CU(cudaStreamWaitEvent(cs, g_hp.ev_k[slot], 0));
+      CU(cudaMemcpyAsync(hpk + k * C, sl, (size_t)m, cudaMemcpyDeviceToHost, cs));
+      CU(cudaEventRecord(g_hp.ev_c[slot], cs));
+    } else {
+      if (k >= D) CU(cudaStreamWaitEvent(cs, g_hp.ev_k[slot], 0));  // slot's previous unpack done
+      CU(cudaMemcpyAsync(sl, hpk + k * C, (size_t)m, cudaMemcpyHostToDevice, cs));
+      CU(cudaEventRecord(g_hp.ev_c[slot], cs));
+      CU(cudaStreamWaitEvent(ks, g_hp.ev_c[slot], 0));
+      st = pack_common(true, t, count, dorig, sl, pos + k * C, &m, ks, /*check_ptrs=*/false);
+      if (st != DT_OK) return st;
+      CU(cudaEventRecord(g_hp.ev_k[slot], ks));
+    }
+  }
+  CU(cudaEventRecord(g_hp.ev_end[0], ks));
+  CU(cudaEventRecord(g_hp.ev_end[1], cs));
+  CU(cudaStreamWaitEvent(us, g_hp.ev_end[0], 0));
+  CU(cudaStreamWaitEvent(us, g_hp.ev_end[1], 0));
+  CU(cudaStreamSynchronize(us));
+  return DT_OK;
+}
+
 static dt_status host_common(bool unpack, dt_t t, int64_t count, const void* a, void* b, int64_t pos, int64_t* len,
                              void* stream) {
   if (!t || !len || count < 0 || pos < 0 || *len < 0 || !a || !b) {
@@ -1217,6 +1291,15 @@ static dt_status host_common(bool unpack, dt_t t, int64_t count, const void* a, 
     if (!getenv("DT_HOST_STAGED") && host_mapped(nc + lo, &d0) && host_mapped(nc + hi - 1, &d1) &&
         host_mapped(pk, &d2) && (uint8_t*)d1 - (uint8_t*)d0 == hi - lo - 1) {
       uint8_t* dorig = (uint8_t*)d0 - lo;
+      // pipeline: unpack only by default (CE H2D of packed chunks + zero-copy scatter: C2
+      // 1.88 -> 1.71 ms); for pack the SM's zero-copy reads slow down next to the CE's D2H
+      // (1.87 -> 2.21 ms), so pack keeps the single kernel (DT_HOST_PIPE=2 pipelines both)
+      const char* hp = getenv("DT_HOST_PIPE");
+      const int mode = hp ? atoi(hp) : 1;
+      if (n > ((int64_t)8 << 20) && (mode == 2 || (mode == 1 && unpack))) {
+        std::lock_guard<std::mutex> g(g_scratch_mu);
+        return host_pipe(unpack, t, count, dorig, (uint8_t*)pk, pos, n, (cudaStream_t)stream);
+      }
       int64_t m = n;
       dt_status st = pack_common(unpack, t, count, dorig, d2, pos, &m, stream, /*check_ptrs=*/false);
       if (st != DT_OK) return st;

@@ -256,6 +256,40 @@ def test_host_entry_points_pinned(torch_cuda, name):
     assert np.array_equal(dst.numpy(), ref)
 
 
+@pytest.mark.parametrize("chunk", [None, str(1 << 20), str(3 << 20)])
+@pytest.mark.parametrize("pipe", ["1", "2"])
+@pytest.mark.parametrize("name", ["C2", "C5b"])
+def test_host_pipeline_pinned(torch_cuda, name, chunk, pipe, monkeypatch):
+    """Pinned host buffers above 8 MiB: the host-link pipeline (zero-copy gather/scatter on
+    the SMs into a device chunk ring, copy engine for the packed side, two internal streams)
+    is bit-exact vs the oracle for whole streams and a ragged fragment, at chunk sizes that
+    do and do not divide the stream; unpack leaves the host gap bytes untouched."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    if chunk:
+        monkeypatch.setenv("DT_HOST_CHUNK", chunk)
+    monkeypatch.setenv("DT_HOST_PIPE", pipe)  # 1: unpack pipelined, 2: pack too
+    rec, org, parent = {"C2": lambda: c2_lower_triangle(), "C5b": lambda: c5b_irregular(24 << 20)}[name]()
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    src_h = fill_bytes(parent, 17)
+    src = torch.from_numpy(src_h).pin_memory()
+    n = t.size
+    exp = oracle.pack(ot, 1, src_h, org)
+    out = torch.full((n,), 0xA5, dtype=torch.uint8).pin_memory()
+    dt.pack_host(t, 1, src.data_ptr() + org, out.data_ptr(), stream=0)
+    assert np.array_equal(out.numpy(), exp)
+    a, b = 4100, n - 9000  # fragment: ragged both ends
+    part = torch.full((b - a,), 0xA5, dtype=torch.uint8).pin_memory()
+    dt.pack_host(t, 1, src.data_ptr() + org, part.data_ptr(), a, b - a, stream=0)
+    assert np.array_equal(part.numpy(), exp[a:b])
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8).pin_memory()
+    dt.unpack_host(t, 1, out.data_ptr(), dst.data_ptr() + org, stream=0)
+    ref = np.full(parent, 0xA5, dtype=np.uint8)
+    oracle.unpack(ot, 1, exp, ref, org)
+    assert np.array_equal(dst.numpy(), ref)
+
+
 def test_full_size_sampled_c5_large(torch_cuda):
     """BASELINE sizes where the oracle cannot produce the whole stream quickly:
     compare sampled stream bytes against the oracle's per-position addresses."""
