@@ -243,7 +243,7 @@ def run_ours(args):
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(f"c2_{dom}")
-    e2e = run_e2e(args, t, src_h, org, parent, payload, dev) if rank == 0 else None
+    e2e = run_e2e(args, t, src_h, org, parent, payload, dev) if rank == 0 and not args.no_e2e else None
     transfer = None
     if ws > 1:
         # the north_star's multi-GPU metric: pipelined non-contiguous exchange between
@@ -690,6 +690,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-e2e", action="store_true",
+                    help="skip the host-buffer e2e leg (ncu launch lists of the timed device step)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     args = ap.parse_args()
     if args.warmup < 3:

@@ -114,10 +114,11 @@ def test_plan_selects_kernels():
     assert t.plan(1, 0x10000, 0x20000, 0, 800)[0] == 2
     # byte-granular start position lowers the word size
     assert t.plan(1, 0x10000, 0x20000, 3, 100) == (2, 1)
-    # irregular short blocks under a template too large for a word table: window kernel
+    # irregular short blocks under a template too large for a word table: block spans
     t = dt.from_recipe(c5b_irregular(1 << 20)[0])
-    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 20) == (3, 4)
-    assert t.plan(1, 0x10000, 0x20008, 0, 1 << 20)[0] == 1     # packed side not 16-B aligned
+    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 20) == (7, 4)
+    assert t.plan(1, 0x10000, 0x20008, 0, 1 << 20) == (7, 4)   # packed side only word-aligned
+    assert t.plan(1, 0x10000, 0x20000, 1, 1 << 19) == (3, 1)   # byte words: block windows
     # contiguous type, many instances: one long run
     t = dt.Type.basic("DOUBLE").contiguous(10)
     assert t.plan(1000, 0x10000, 0x20000, 0, 80000)[0] == 1
