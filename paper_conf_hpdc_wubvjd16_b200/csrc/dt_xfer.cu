@@ -50,7 +50,7 @@ struct XOp {
   int32_t g;       // word granularity
   int64_t n;       // send: bytes; recv: capacity in bytes
   int64_t chunk;
-  int32_t depth, cta0, ncta, pad;
+  int32_t depth, cta0, ncta, rep;  // rep (send role): CTAs per sub-ring, alternating fragments
   uint8_t* ring;   // slot 0 of the (pair, channel) ring (send: peer memory; recv: local)
   uint64_t* ready; // [depth]  send: peer; recv: local
   uint64_t* ack;   // [depth]  send: local; recv: peer
@@ -200,14 +200,21 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   // D slots and flags, so every CTA pipelines on its own (no cross-CTA wait per
   // fragment).  The sender runs one CTA per sub-ring; receiver CTA j serves
   // sub-rings j, j+ncta, ...
+  // Replicas: with an even depth, sub-ring js is served by `rep` CTAs that take alternate
+  // fragments (fragment k -> replica k % rep; slot k % D belongs to one replica), so two
+  // fragments of a sub-ring are in flight at once and each fragment's fixed cost (credit
+  // poll, store completion, publication) overlaps the other's copy.
   int64_t n = X.n;
-  int gs;
+  int gs, rep;
+  __shared__ int s_rep;
   if (X.role == 0) {
-    gs = X.ncta;
-    // ---- send role: header {seq, nbytes, gs}, wait for "go" (receiver-driven, [L20:c3973])
+    rep = X.rep > 1 ? X.rep : 1;
+    gs = X.ncta / rep;
+    // ---- send role: header {seq, nbytes, gs, rep}, wait for "go" (receiver-driven, [L20:c3973])
     if (j == 0 && threadIdx.x == 0) {
       st_release_sys(X.hdr + 1, (uint64_t)n);
       st_release_sys(X.hdr + 2, (uint64_t)gs);
+      st_release_sys(X.hdr + 3, (uint64_t)rep);
       st_release_sys(X.hdr, X.seq);
     }
     if (threadIdx.x == 0) {
@@ -228,12 +235,14 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       bool ok = spin(X.hdr, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v);
       s_val = ok ? ld_acquire_sys(X.hdr + 1) : 0;
       s_gs = ok ? (int)ld_acquire_sys(X.hdr + 2) : 1;
+      s_rep = ok ? (int)ld_acquire_sys(X.hdr + 3) : 1;
       s_stop = ok ? 0 : 2;
     }
     __syncthreads();
     if (s_stop == 2) return;
     n = (int64_t)s_val;
     gs = s_gs;
+    rep = s_rep > 1 ? s_rep : 1;
     if (n > X.n) {
       if (j == 0 && threadIdx.x == 0) {
         atomicCAS(X.err, 0, XERR_TRUNCATE);
@@ -247,10 +256,29 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
 
   const int64_t Cs = C / gs;
   const int64_t K = (n + C - 1) / C;
+  // this CTA's replica and sub-rings: sender CTA j = replica j / gs of sub-ring j % gs;
+  // receiver CTAs split into rep groups of nsub (a receiver with fewer CTAs than
+  // replicas serves every fragment)
+  int myrep = 0, js0 = j, jstep = X.ncta;
+  bool all_k = rep == 1;
+  if (X.role == 0) {
+    myrep = j / gs;
+    js0 = j % gs;
+    jstep = gs;
+  } else if (X.ncta >= rep && rep > 1) {
+    const int nsub = X.ncta / rep;
+    myrep = j / nsub;
+    js0 = j % nsub;
+    jstep = nsub;
+    if (myrep >= rep) js0 = gs;  // surplus CTA: no sub-ring
+  } else {
+    all_k = true;
+  }
   for (int64_t k = 0; k < K; k++) {
+    if (!all_k && (int)(k % rep) != myrep) continue;
     const int slot = (int)(k % D);
     const int64_t round = k / D;
-    for (int js = j; js < gs; js += X.ncta) {
+    for (int js = js0; js < gs; js += jstep) {
       const int64_t off = k * C + (int64_t)js * Cs;
       if (off >= n) continue;
       const int64_t len = min(Cs, n - off);
@@ -399,7 +427,7 @@ struct dt_comm_s {
   int64_t* szbuf = nullptr;  // device size handshake buffers [2][kMaxOps]
   int64_t* szhost = nullptr; // pinned
   // layout helpers (uint64 flag words): per (peer, channel) kMaxSub*depth ready
-  // counters, a 4-word header {seq, nbytes, sub-rings, -}, kMaxSub*depth ack
+  // counters, a 4-word header {seq, nbytes, sub-rings, replicas}, kMaxSub*depth ack
   // counters and a go word; then one error word.  The ring of a (source,
   // channel) pair is depth*chunk bytes, split among the sender's sub-rings.
   size_t per() const { return (size_t)kMaxSub * o.depth; }
@@ -790,11 +818,19 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   const int per_op = std::max(1, std::min(G, occ * sms / nops));
   for (int i = 0; i < nops; i++) {
     int n_i = per_op;
-    if (A.ops[i].role == 0) {  // one CTA per sub-ring; a sub-ring slot is C/gs bytes, a multiple of 512
+    if (A.ops[i].role == 0) {  // rep CTAs per sub-ring; a sub-ring slot is C/gs bytes, a multiple of 512
       const int64_t C = A.ops[i].chunk;
+      // replicas: each slot must belong to one replica, and each replica keeps >= 2 slots
+      // (with one slot a replica waits a full round trip per fragment: C3 4 MiB, depth 2:
+      // 441 -> 306 GB/s; depth 4 with 2 replicas: 436 -> 487, 1 MiB: 192 -> 296)
+      const char* rp = getenv("DT_XFER_REP");
+      int rep = rp ? std::max(1, atoi(rp)) : 2;
+      const int dep = A.ops[i].depth;
+      if (dep % rep != 0 || dep / rep < 2 || per_op < rep) rep = 1;
       int g = 1;
-      while (g * 2 <= per_op && g * 2 <= kMaxSub && C % ((int64_t)g * 2 * 512) == 0) g *= 2;
-      n_i = g;
+      while (g * 2 * rep <= per_op && g * 2 <= kMaxSub && C % ((int64_t)g * 2 * 512) == 0) g *= 2;
+      n_i = g * rep;
+      A.ops[i].rep = rep;
     }
     A.ops[i].cta0 = cta;
     A.ops[i].ncta = n_i;

@@ -452,3 +452,20 @@ def test_ring_block_spans(torch_cuda, chunk):
         _loop_check(torch_cuda, comm, ctg, 0, 2 * size, rec, org, parent + ext, scount=1, rcount=2)
         _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
     comm.free()
+
+
+@pytest.mark.parametrize("rep,depth", [("1", 4), ("2", 4), ("2", 8), ("4", 8), ("2", 2)])
+def test_ring_replicas(torch_cuda, rep, depth, monkeypatch):
+    """Replicated sub-rings (rep CTAs per sub-ring taking alternate fragments, announced in
+    the header; the receiver maps its CTAs onto the replicas): bit-exact for every
+    replica/depth combination, including the fallback to one replica when a replica
+    would own a single slot, with repeated messages on the same channel."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    monkeypatch.setenv("DT_XFER_REP", rep)
+    comm = dt.Comm(0, 1, 0, chunk_bytes=256 << 10, depth=depth, ring_loopback=True)
+    rec, org, parent = c3_block_cyclic(2048, 64)
+    for s in range(2):
+        _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent, seed=20 + s)
+    rec5, org5, parent5 = c5_particles(3 << 20)
+    _loop_check(torch_cuda, comm, rec5, org5, parent5, rec5, org5, parent5, seed=7)
+    comm.free()
