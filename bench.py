@@ -252,7 +252,7 @@ def run_ours(args):
         del src, dst, packed, flush, flush_rd
         torch.cuda.empty_cache()
         try:
-            res, xpay, xok, _ = xfer_sweep(ws, rank, local, [1 << 20, 4 << 20], [4], "p2p", 0, 10, 3)
+            res, xpay, xok, _ = xfer_sweep(ws, rank, local, [1 << 20, 4 << 20], [8], "p2p", 0, 10, 3)
             xb = max(res, key=lambda r: r["gbs_per_rank"])
             transfer = {"workload": "C3 block-cyclic 128 MiB per direction, pairs (r, r^1), dt_sendrecv P2P",
                         "value": round(ws * xpay / (xb["ms"] * 1e-3) / 1e9, 1), "unit": UNIT,
@@ -683,7 +683,7 @@ def main():
                     help="p2p ring pipeline, NCCL double buffering, or a persistent direct plan (dt_xplan)")
     ap.add_argument("--xfer-workload", default="c3", choices=["c3", "c5", "c5b"])
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
-    ap.add_argument("--xfer-depths", default="2,4")
+    ap.add_argument("--xfer-depths", default="2,4,8")
     ap.add_argument("--xfer-ctas", type=int, default=0, help="CTAs per direction (0 = library default)")
     ap.add_argument("--ring-loopback", action="store_true", help="halo at N=1: loopback through the ring pipeline")
     ap.add_argument("--steps", type=int, default=200)

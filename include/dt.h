@@ -173,7 +173,7 @@ dt_status dt_type_deserialize(const void* in, size_t nbytes, dt_t* out);
 enum { DT_XFER_P2P = 0, DT_XFER_NCCL = 1 };
 typedef struct {
   int64_t chunk_bytes; /* pipeline fragment size C (reading A15); 0 = default 1 MiB        */
-  int32_t depth;       /* ring slots D per peer; 0 = default 4                             */
+  int32_t depth;       /* ring slots D per peer; 0 = default 8                             */
   int32_t mode;        /* DT_XFER_P2P (pack straight into the peer's ring over NVLink) or
                           DT_XFER_NCCL (double-buffered ncclSend/ncclRecv of packed chunks) */
   int32_t ctas;        /* CTAs per direction for the P2P pipeline kernel; 0 = default      */

@@ -311,7 +311,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
         // the generic release.  A full SC fence (bit 2 of DT_XFER_FLAGS) cost 20-25 % of
         // the loopback exchange rate at 1-4 MiB fragments and is not needed for this pattern.
         if (A.flags & 4) __threadfence_system();
-        asm volatile("fence.proxy.async.global;" ::: "memory");
+        if (X.kind == 4 && X.role == 0) asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA stores
         red_release_sys_add(X.role == 0 ? X.ready + fi : X.ack + fi, (uint64_t)len);
       }
     }
@@ -470,7 +470,7 @@ static dt_status cufail(cudaError_t e, const char* what) {
 
 static void fill_opts(dt_xfer_opts& o, const dt_xfer_opts* in) {
   o.chunk_bytes = 1 << 20;
-  o.depth = 4;
+  o.depth = 8;
   o.mode = DT_XFER_P2P;
   o.ctas = 0;
   o.flags = in ? in->flags : 0;
@@ -823,9 +823,15 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       // replicas: each slot must belong to one replica, and each replica keeps >= 2 slots
       // (with one slot a replica waits a full round trip per fragment: C3 4 MiB, depth 2:
       // 441 -> 306 GB/s; depth 4 with 2 replicas: 436 -> 487, 1 MiB: 192 -> 296)
+      // default: the most replicas (<= 4) that still leave each >= 2 slots (depth 8: 4
+      // replicas, C3 1 MiB 415 GB/s; depth 4: 2 replicas, 300 GB/s)
       const char* rp = getenv("DT_XFER_REP");
-      int rep = rp ? std::max(1, atoi(rp)) : 2;
       const int dep = A.ops[i].depth;
+      int rep = rp ? std::max(1, atoi(rp)) : 4;
+      if (!rp) {
+        const int64_t K = (A.ops[i].n + C - 1) / C;  // fragments: replicas beyond K would idle
+        while (rep > 1 && (dep % rep != 0 || dep / rep < 2 || rep > K)) rep /= 2;
+      }
       if (dep % rep != 0 || dep / rep < 2 || per_op < rep) rep = 1;
       int g = 1;
       while (g * 2 * rep <= per_op && g * 2 <= kMaxSub && C % ((int64_t)g * 2 * 512) == 0) g *= 2;
