@@ -420,3 +420,53 @@ def test_block_span_kernel(torch_cuda, name, monkeypatch):
             a = int(rng.integers(0, total // 4)) * 4
             b = int(rng.integers(a // 4, total // 4 + 1)) * 4
             check_pack_unpack(torch_cuda, rec, org, parent, count=count, pos=a, nbytes=b - a, seed=a)
+
+
+def test_random_types_forced_block_spans(torch_cuda, monkeypatch):
+    """Tiny random types (the oracle pins' enumeration, another third of it) forced through
+    the block-span kernel where it applies (G >= 4; the planner falls back otherwise), with
+    counts 1-3, ragged pos/len and misaligned origins."""
+    from tests.test_oracle_pins import _tiny_types
+    monkeypatch.setenv("DT_FORCE_KERNEL", "7")
+    rng = np.random.default_rng(12)
+    for i, r in enumerate(_tiny_types()[1::3]):
+        info = oracle.from_recipe(r).info()
+        if info["size"] == 0:
+            continue
+        lo = min(0, info["true_lb"], info["true_lb"] + 2 * info["extent"])
+        hi = max(info["true_ub"], info["true_ub"] + 2 * info["extent"], 1)
+        count = int(rng.integers(1, 4))
+        total = count * info["size"]
+        a, b = sorted(rng.integers(0, total + 1, size=2))
+        try:
+            check_pack_unpack(torch_cuda, r, -lo + 16, hi - lo + 32, count=count, pos=int(a), nbytes=int(b - a),
+                              seed=i, origin_pad=int(rng.integers(0, 16)))
+        except Exception as e:  # noqa: BLE001
+            if "DT_ERR_OVERLAP" not in str(e):
+                raise
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_random_irregular_struct_lists(torch_cuda, seed):
+    """Seeded random index lists of small structs (int32 + double pairs, resized records,
+    random signed displacements, random block counts per entry) -- the nested
+    struct/hindexed family of config C5 with irregular blocks -- through the planner's
+    choice, whole streams and random 4-byte-aligned fragments, counts 1 and 2."""
+    rng = np.random.default_rng(100 + seed)
+    rec_sz = int(rng.choice([16, 24, 32]))
+    rec = ("resized", ("struct", [1, 1], [0, 8], [("basic", "INT32"), ("basic", "DOUBLE")]), 0, rec_sz)
+    n = int(rng.integers(3000, 9000))
+    slots = rng.permutation(4 * n)[:n] - n  # signed, unsorted record slots
+    bl = rng.integers(1, 4, size=n)
+    rec_t = ("hindexed", bl, slots.astype(np.int64) * rec_sz * 4, rec)
+    lo_slot, hi_slot = int(slots.min()), int(slots.max())
+    org = -lo_slot * rec_sz * 4 + 64
+    parent = (hi_slot - lo_slot) * rec_sz * 4 + 4 * rec_sz * 4 + 128
+    size = oracle.from_recipe(rec_t).size
+    ext = oracle.from_recipe(rec_t).extent
+    check_pack_unpack(torch_cuda, rec_t, org, parent + ext, seed=seed)
+    for count in (1, 2):
+        total = count * size
+        a = int(rng.integers(0, total // 4)) * 4
+        b = int(rng.integers(a // 4, total // 4 + 1)) * 4
+        check_pack_unpack(torch_cuda, rec_t, org, parent + ext, count=count, pos=a, nbytes=b - a, seed=a)
