@@ -958,13 +958,28 @@ __device__ __forceinline__ void span_window_io(uint8_t* g, uint8_t* s, int n, in
   }
 }
 
-// Wide span (rare): warp-cooperative copy of each block of the window.  Not
-// inlined, so that the realigning copies' registers do not cap the fast path.
-template <bool UNPACK, int POL>
+// Wide span (scattered or unsorted blocks): blocks shorter than 256 bytes are
+// copied by their own lane with G-byte words (the window's 32 blocks in flight at
+// once), longer ones by the whole warp.  Not inlined, so that the realigning
+// copies' registers do not cap the fast path.
+template <bool UNPACK, int G, int POL>
 __device__ __noinline__ void span_wide(int32_t n, int64_t a, int32_t off, uint8_t* cp, int lane) {
-  for (int j = 0; j < 32; j++) {
+  typedef typename WordT<G>::T W;
+  if (n > 0 && n < 256) {
+    W* lw = reinterpret_cast<W*>(a);
+    W* pw = reinterpret_cast<W*>(cp + off);
+    const int nw = n / G;
+#pragma unroll 4
+    for (int i = 0; i < nw; i++) {
+      if (UNPACK) lw[i] = POL == LD_CG ? __ldcg(pw + i) : pw[i];  // (ring slots: L2 only)
+      else pw[i] = lw[i];
+    }
+  }
+  unsigned big = __ballot_sync(0xffffffffu, n >= 256);
+  while (big) {
+    const int j = __ffs(big) - 1;
+    big &= big - 1;
     const int32_t nj = __shfl_sync(0xffffffffu, n, j);
-    if (nj == 0) break;
     uint8_t* aj = reinterpret_cast<uint8_t*>(__shfl_sync(0xffffffffu, a, j));
     uint8_t* pj = cp + __shfl_sync(0xffffffffu, off, j);
     if (UNPACK) warp_copy<POL>(aj, pj, nj, lane);
@@ -1065,7 +1080,8 @@ __device__ __forceinline__ SpanWin span_geom(const KP& P, SpanCur& c, uint64_t e
     const uint64_t k = fdiv((uint64_t)c.cb, P.fnb);
     c.ce += k;
     c.cb -= (int64_t)k * P.nblocks;
-    c.ced = elem_disp(P, c.ce);
+    // (past the slice's end the element may not exist: a list level has no entry for it)
+    if (c.p < p1) c.ced = elem_disp(P, c.ce);
   }
   return w;
 }
@@ -1162,7 +1178,7 @@ __device__ __forceinline__ void span_range(const KP& P, uint8_t* cbase, const Pl
     }
     // ---- copy window k
     if (!w.fast) {
-      span_wide<UNPACK, POL>(w.n, w.a, w.off, w.cp, lane);
+      span_wide<UNPACK, G, POL>(w.n, w.a, w.off, w.cp, lane);
     } else if (!UNPACK) {
       // packed-word map: omap[word of the window's 16-byte-aligned packed range] =
       // span word; then each lane assembles whole 16-byte packed chunks

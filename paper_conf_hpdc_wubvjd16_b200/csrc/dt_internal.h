@@ -40,6 +40,7 @@ struct Form {
   // per-call planning must stay O(levels): O(n) facts are computed once and cached
   mutable int64_t gran_cache = -1, tsize_cache = -1, lvl_gran_cache = -1;
   mutable int fits32_cache = -1;
+  mutable int span_local_cache = -1;  // block-span kernel: are 32-block windows locally dense?
   mutable int64_t span_lo = 0, span_hi = -1;  // cached min bd / max bd+bl (span_hi < span_lo: not computed)
   void span(int64_t* lo, int64_t* hi) const {
     if (span_hi < span_lo) {
@@ -62,6 +63,7 @@ struct Form {
   void invalidate() const {
     gran_cache = tsize_cache = lvl_gran_cache = -1;
     fits32_cache = -1;
+    span_local_cache = -1;
     span_lo = 0;
     span_hi = -1;
     hoff_cache.clear();

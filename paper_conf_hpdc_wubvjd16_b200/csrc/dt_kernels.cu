@@ -21,6 +21,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "dt_device.cuh"
@@ -523,6 +524,60 @@ bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_
   return true;
 }
 
+// Block-span kernel precondition (cached per form, O(1) per call): the 32-block
+// windows of the stream must be local -- at most a few span buffers wide -- else
+// they all take the kernel's wide-span fallback and the block-window kernel is
+// faster (tools/kind_probe.py, 64 MiB pack: C5b fully shuffled 110 vs 180 us and an
+// unsorted record list 49 vs 82 us favour block windows; C5b 104 vs 58, 16-byte
+// blocks with spans around 4 KiB 82 vs 40, C5b shuffled within 48 blocks 102 vs 115
+// favour / tie with block spans).  Rule: half of the sampled windows within 16 KiB.
+// Sampled: 64 windows of the template, or, for templates of < 32 blocks, 64 windows
+// of the innermost level (its stride, or consecutive entries of its table).
+static bool span_local(const Form& f) {
+  if (f.span_local_cache >= 0) return f.span_local_cache != 0;
+  const int64_t nb = (int64_t)f.bl.size();
+  constexpr int64_t kBuf = 4 * 4096;
+  int good = 0, tot = 0;
+  if (nb >= 32) {
+    for (int s = 0; s < 64; s++) {
+      const int64_t i0 = (nb - 32) * s / 63;
+      int64_t lo = INT64_MAX, hi = INT64_MIN;
+      for (int64_t i = i0; i < i0 + 32; i++) {
+        lo = std::min(lo, f.bd[(size_t)i]);
+        hi = std::max(hi, f.bd[(size_t)i] + f.bl[(size_t)i]);
+      }
+      tot++;
+      good += hi - lo <= kBuf;
+    }
+  } else if (!f.lv.empty()) {
+    int64_t tlo, thi;
+    f.span(&tlo, &thi);
+    const int64_t tspan = thi - tlo, epw = (32 + nb - 1) / nb;  // elements per window
+    const Level& in = f.lv.back();
+    if (!in.is_list()) {
+      tot = 1;
+      good = (int)(std::llabs(in.stride) * (epw - 1) + tspan <= kBuf);
+    } else {
+      const std::vector<int64_t>& tb = *in.table;
+      const int64_t n = (int64_t)tb.size();
+      for (int s = 0; s < 64; s++) {
+        const int64_t i0 = std::max<int64_t>(0, n - epw) * s / 63;
+        int64_t lo = INT64_MAX, hi = INT64_MIN;
+        for (int64_t i = i0; i < std::min(n, i0 + epw); i++) {
+          lo = std::min(lo, tb[(size_t)i]);
+          hi = std::max(hi, tb[(size_t)i]);
+        }
+        tot++;
+        good += hi - lo + tspan <= kBuf;
+      }
+    }
+  } else {
+    tot = good = 1;  // one small template: instances at the extent (dense for these lists)
+  }
+  f.span_local_cache = good * 2 >= tot ? 1 : 0;
+  return f.span_local_cache != 0;
+}
+
 int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
                 int64_t* gran) {
   if (len <= 0 || f.bl.empty()) return 0;
@@ -557,7 +612,7 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   if (mean < 256.0 && rec_ok && !force) return 6;
   if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return stage_ok && g >= 8 ? 4 : 2;
   // many short blocks (no word table): block spans with >= 4-byte words, else block windows
-  if (mean < 128.0 && g >= 4 && !force) return 7;
+  if (mean < 128.0 && g >= 4 && !force && span_local(f)) return 7;
   if (mean < 128.0 && blk_ok) return 3;
   return 1;
 }

@@ -119,6 +119,16 @@ def test_plan_selects_kernels():
     assert t.plan(1, 0x10000, 0x20000, 0, 1 << 20) == (7, 4)
     assert t.plan(1, 0x10000, 0x20008, 0, 1 << 20) == (7, 4)   # packed side only word-aligned
     assert t.plan(1, 0x10000, 0x20000, 1, 1 << 19) == (3, 1)   # byte words: block windows
+    # ... unless the list is not locally dense (shuffled blocks / unsorted records): windows
+    rec, _, _ = c5b_irregular(1 << 20)
+    perm = np.random.default_rng(9).permutation(len(rec[1]))
+    t = dt.from_recipe(("hindexed", rec[1][perm], rec[2][perm], rec[3]))
+    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 20) == (3, 4)
+    rs = ("resized", ("struct", [1, 1], [0, 8], [("basic", "INT32"), ("basic", "DOUBLE")]), 0, 16)
+    slots = np.random.default_rng(5).permutation(1 << 16)[: 1 << 15].astype(np.int64)
+    t = dt.from_recipe(("hindexed", np.ones(1 << 15, dtype=np.int64), slots * 16, rs))
+    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 16)[0] == 6    # whole-record loads, any order
+    assert t.plan(1, 0x10008, 0x20000, 0, 1 << 16)[0] == 2    # records not 16-B aligned: word table
     # contiguous type, many instances: one long run
     t = dt.Type.basic("DOUBLE").contiguous(10)
     assert t.plan(1000, 0x10000, 0x20000, 0, 80000)[0] == 1
