@@ -495,6 +495,9 @@ def run_halo(args):
         xp = plan.direct_plan(comm, buf, single_rank=ws == 1)
         exchange = lambda: xp.start(s)  # noqa: E731
         check = xp.check
+    elif args.xfer_mode == "hybrid":  # y/z faces direct, x faces through the ring on a side stream
+        exchange = plan.hybrid(comm, buf, s, single_rank=ws == 1)
+        check = exchange.check
     else:
         exchange = lambda: plan.exchange(comm, buf, stream=s)  # noqa: E731
         check = comm.check
@@ -679,8 +682,9 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--workload", default="c2", choices=["c2", "xfer", "halo", "sweep"])
     ap.add_argument("--sweep", default="all", help="--workload sweep: comma-separated config names or 'all'")
-    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "direct"],
-                    help="p2p ring pipeline, NCCL double buffering, or a persistent direct plan (dt_xplan)")
+    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "direct", "hybrid"],
+                    help="p2p ring pipeline, NCCL double buffering, a persistent direct plan (dt_xplan), "
+                         "or (halo only) hybrid: y/z faces direct, x faces through the ring")
     ap.add_argument("--xfer-workload", default="c3", choices=["c3", "c5", "c5b"])
     ap.add_argument("--xfer-chunks-kib", default="64,256,1024,4096", help="pipeline fragment sizes (reading A15)")
     ap.add_argument("--xfer-depths", default="2,4,8")
@@ -699,6 +703,8 @@ def main():
     if args.impl == "reference":
         run_reference(args)
     elif args.workload == "xfer":
+        if args.xfer_mode == "hybrid":
+            ap.error("--xfer-mode hybrid applies to --workload halo only")
         run_xfer(args)
     elif args.workload == "halo":
         run_halo(args)

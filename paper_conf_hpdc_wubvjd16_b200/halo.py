@@ -58,7 +58,7 @@ class HaloPlan:
     send_types: dict
     recv_types: dict
 
-    def exchange(self, comm, buf, stream=None):
+    def exchange(self, comm, buf, stream=None, faces=FACES):
         """Post all 12 transfers of one exchange as one group.  The message sent
         through face f is received by the neighbour through its face OPPOSITE[f];
         messages between the same pair are matched in posting order, so both sides
@@ -75,25 +75,54 @@ class HaloPlan:
                 comm.sendrecv(None, 0, None, -1, buf, 1, self.recv_types[face], peer, stream=stream)
         comm.group_end(stream)
 
-    def direct_plan(self, comm, buf, group=None, single_rank=False):
+    def direct_plan(self, comm, buf, group=None, single_rank=False, faces=FACES):
         """The same exchange as a persistent direct plan (dt_xplan): one kernel per
         exchange writes every boundary layer straight into the neighbour's ghost
         layer in peer memory.  Tag = index of the SENDER's face in FACES, so the
         pairing is unique even when both neighbours in a dimension are one rank."""
         from .dt import XPlan
-        sends = [(buf, 1, self.send_types[f], neighbour(self.rank, f, self.dims), i) for i, f in enumerate(FACES)]
+        sends = [(buf, 1, self.send_types[f], neighbour(self.rank, f, self.dims), i)
+                 for i, f in enumerate(FACES) if f in faces]
         recvs = [(buf, 1, self.recv_types[OPPOSITE[f]], neighbour(self.rank, OPPOSITE[f], self.dims), i)
-                 for i, f in enumerate(FACES)]
+                 for i, f in enumerate(FACES) if f in faces]
         if single_rank:
             return XPlan.local(comm, sends, recvs)
         return XPlan.from_process_group(comm, sends, recvs, group)
 
-    def ops(self):
+    def ops(self, faces=FACES):
         """[(kind, face, peer)] in posting order: kind 'send' (my boundary layer `face`
-        to `peer`) or 'recv' (ghost layer `face` from `peer`)."""
-        out = [("send", f, neighbour(self.rank, f, self.dims)) for f in FACES]
-        out += [("recv", OPPOSITE[f], neighbour(self.rank, OPPOSITE[f], self.dims)) for f in FACES]
+        to `peer`) or 'recv' (ghost layer `face` from `peer`), for the transfers
+        sent through `faces`."""
+        fs = [f for f in FACES if f in faces]
+        out = [("send", f, neighbour(self.rank, f, self.dims)) for f in fs]
+        out += [("recv", OPPOSITE[f], neighbour(self.rank, OPPOSITE[f], self.dims)) for f in fs]
         return out
+
+    def hybrid(self, comm, buf, stream, group=None, single_rank=False):
+        """Hybrid exchange: the y/z faces (long contiguous runs of n*h elements)
+        go through a persistent direct plan on `stream`, the x faces (one element
+        per run, 4-B blocks) through the packed ring group on a second stream, so
+        the short-block faces move as dense packed fragments while the long-run
+        faces skip the ring.  Returns a callable that posts one exchange, ordered
+        on `stream` (the second stream joins back through an event)."""
+        import torch
+        yz = tuple(f for f in FACES if f[0] != "x")
+        xs = tuple(f for f in FACES if f[0] == "x")
+        xp = self.direct_plan(comm, buf, group=group, single_rank=single_rank, faces=yz)
+        side = torch.cuda.Stream(device=stream.device)
+        fork, join = torch.cuda.Event(), torch.cuda.Event()
+
+        def run():
+            fork.record(stream)
+            side.wait_event(fork)
+            self.exchange(comm, buf, stream=side, faces=xs)
+            join.record(side)
+            xp.start(stream)
+            stream.wait_event(join)
+
+        run.plan = xp
+        run.check = lambda: (xp.check(), comm.check())
+        return run
 
 
 def make_plan(rank: int, n: int = 512, h: int = 1, dims=(2, 2, 2), basic: str = "FLOAT") -> HaloPlan:

@@ -325,6 +325,42 @@ def test_direct_plan_halo_single_rank(torch_cuda):
     comm.free()
 
 
+@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+def test_hybrid_halo_single_rank(torch_cuda, ring):
+    """1-rank periodic halo, hybrid: y/z faces through a direct plan on the main
+    stream, x faces through the ring group on a side stream joined by an event."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import FACES, face_box, make_plan
+    n, h = 48, 1
+    L = n + 2 * h
+    comm = dt.Comm(0, 1, 0, chunk_bytes=8 << 10, depth=2, ring_loopback=ring)
+    hp = make_plan(0, n, h, dims=(1, 1, 1))
+    assert [f for _, f, _ in hp.ops(("x-", "x+"))] == ["x-", "x+", "x+", "x-"]
+    A = np.full((L, L, L), 0xA5A5A5A5, dtype=np.uint32)
+    z, y, x = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
+    A[h:h + n, h:h + n, h:h + n] = (z * 1000000 + y * 1000 + x).astype(np.uint32)
+    buf = torch.from_numpy(A.view(np.uint8).reshape(-1).copy()).cuda()
+    s = torch.cuda.current_stream()
+    run = hp.hybrid(comm, buf, s, single_rank=True)
+    for _ in range(3):
+        run()
+    torch.cuda.synchronize()
+    run.check()
+    B = buf.cpu().numpy().view(np.uint32).reshape(L, L, L)
+    for f in FACES:
+        sub, st = face_box(f, n, h, ghost=True)
+        zz, yy, xx = np.meshgrid(*[np.arange(s_, s_ + k) for s_, k in zip(st, sub)], indexing="ij")
+        exp = (((zz - h) % n) * 1000000 + ((yy - h) % n) * 1000 + ((xx - h) % n)).astype(np.uint32)
+        assert np.array_equal(B[zz, yy, xx], exp), f
+    assert np.array_equal(B[h:h + n, h:h + n, h:h + n], A[h:h + n, h:h + n, h:h + n])
+    # edges and corners (outside every face box) are untouched
+    assert np.all(B[0, 0, :] == 0xA5A5A5A5) and np.all(B[:, 0, 0] == 0xA5A5A5A5)
+    run.plan.free()
+    comm.free()
+
+
 def test_direct_plan_errors(torch_cuda):
     import torch
 
