@@ -533,7 +533,7 @@ def run_halo(args):
             "config": {"workload": f"C4: 3D halo 512^3 f32 per rank, 6 faces x {face} B, grid {dims}, "
                                    f"mode={args.xfer_mode}", "us_per_exchange": round(ms * 1e3, 2),
                        "periodic_self_check": ok, "np": np.__version__},
-            "gpu_launches": steps}
+            "gpu_launches": steps * (2 if args.xfer_mode == "hybrid" else 1)}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if ws > 1:
