@@ -1,7 +1,9 @@
 """Diagnostic: C4 halo (512^3 f32, 1 GPU, periodic on itself) through the ring
-pipeline (loopback) with the exchange split by face set, event-timed."""
+pipeline (loopback) with the exchange split by face set, event-timed; also the host time spent
+posting each exchange (a GPU time equal to it means the loop is host-bound)."""
 import os
 import sys
+import time
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
@@ -26,13 +28,17 @@ def main():
         for _ in range(3):
             plan.exchange(comm, buf, stream=s, faces=faces)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
         e0.record(s)
+        t0 = time.perf_counter()
         for _ in range(20):
             plan.exchange(comm, buf, stream=s, faces=faces)
+        t1 = time.perf_counter()
         e1.record(s)
         torch.cuda.synchronize()
         comm.check()
-        res[name] = round(e0.elapsed_time(e1) / 20 * 1e3, 1)
+        # GPU us per exchange, and host us per exchange spent posting it (enqueue only)
+        res[name] = (round(e0.elapsed_time(e1) / 20 * 1e3, 1), round((t1 - t0) / 20 * 1e6, 1))
     print(os.environ.get("PROBE_TAG", ""), f"chunk={chunk} depth={depth}", res, flush=True)
 
 
