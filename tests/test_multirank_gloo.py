@@ -152,3 +152,24 @@ def test_halo_plan_geometry():
             assert neighbour(neighbour(r, f, dims), OPPOSITE[f], dims) == r
     # 2x2x2 periodic: both x neighbours are the same rank (3 distinct peers, reading A17)
     assert len({neighbour(0, f, dims) for f in FACES}) == 3
+
+
+def test_halo_ops_face_subsets():
+    """The hybrid exchange splits one exchange into face subsets closed under
+    OPPOSITE; the subsets' ops partition the full exchange's ops, and each subset
+    keeps the global posting order (sender's face in FACES order)."""
+    from paper_conf_hpdc_wubvjd16_b200.halo import FACES, OPPOSITE, HaloPlan
+    for dims in [(2, 2, 2), (1, 2, 2), (1, 1, 2)]:
+        for r in range(dims[0] * dims[1] * dims[2]):
+            hp = HaloPlan(8, 1, dims, r, {}, {})
+            full = hp.ops()
+            xs, yz = hp.ops(("x-", "x+")), hp.ops(("y-", "y+", "z-", "z+"))
+            assert sorted(xs + yz) == sorted(full)
+            for sub in (xs, yz):
+                sends = [f for k, f, _ in sub if k == "send"]
+                recvs = [f for k, f, _ in sub if k == "recv"]
+                assert sends == [f for f in FACES if f in sends]
+                assert recvs == [OPPOSITE[f] for f in sends]
+                # order within the subset is the order in the full exchange
+                assert [full.index(o) for o in sub if o[0] == "send"] == sorted(
+                    full.index(o) for o in sub if o[0] == "send")
