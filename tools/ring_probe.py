@@ -17,7 +17,8 @@ def main():
     dst = torch.zeros_like(src)
     s = torch.cuda.current_stream()
     for chunk, depth in [(1 << 20, 2), (1 << 20, 8), (4 << 20, 2), (256 << 10, 4)]:
-        comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth, ring_loopback=True)
+        comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth, ring_loopback=True,
+                       ctas=int(os.environ.get("PROBE_CTAS", 0)))
         row = {}
         for n in [64 << 10, 256 << 10, 1 << 20, 4 << 20, 16 << 20, 64 << 20]:
             for _ in range(3):
@@ -31,7 +32,7 @@ def main():
             comm.check()
             assert torch.equal(dst[:n], src[:n])
             row[f"{n >> 10}K"] = round(e0.elapsed_time(e1) / 10 * 1e3, 1)
-        print(f"unit={unit} chunk={chunk >> 10}K depth={depth}", row, flush=True)
+        print(f"unit={unit} ctas={os.environ.get('PROBE_CTAS', 0)} chunk={chunk >> 10}K depth={depth}", row, flush=True)
         comm.free()
 
 
