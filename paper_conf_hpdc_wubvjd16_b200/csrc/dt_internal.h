@@ -100,6 +100,8 @@ struct DeviceDesc {
   struct PlanSlot {
     int64_t count = -1, pos = 0, len = 0, nw = 0, alpha = 0, tsize = 0, gran = 1;
     void* d = nullptr;
+    void* made_on = nullptr;  // stream the k_plan that filled `d` was enqueued on
+    void* ready = nullptr;    // cudaEvent_t recorded after that k_plan (cross-stream reuse waits on it)
   };
   std::vector<PlanSlot> plans;
   size_t plan_next = 0;

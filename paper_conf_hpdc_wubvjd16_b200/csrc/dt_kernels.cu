@@ -251,15 +251,29 @@ __global__ void __launch_bounds__(256) k_word(const KP P) {
                                                      (int64_t)gridDim.x * blockDim.x);
 }
 // --------------------------------------------------------------- host side
-static int g_num_sms = 0;
+// Per-device launch state: kernel attributes (max dynamic smem) are per device, so
+// a process driving several devices (dt_comm_connect supports it) sets them on each.
+struct DevLaunch {
+  int sms = 0;
+  bool rec_attr = false, stage_attr = false, span_attr = false, dual_attr = false;
+  int span_occ = 0, word_occ = 0;
+  int seg_occ[2][2] = {{0, 0}, {0, 0}};
+};
+static DevLaunch g_devl[64];
+static DevLaunch& devl() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return g_devl[dev & 63];
+}
 static int num_sms() {
-  if (!g_num_sms) {
+  DevLaunch& d = devl();
+  if (!d.sms) {
     int dev = 0;
     cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-    if (g_num_sms <= 0) g_num_sms = 148;
+    cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev);
+    if (d.sms <= 0) d.sms = 148;
   }
-  return g_num_sms;
+  return d.sms;
 }
 
 static dt_status cuda_fail(cudaError_t e, const char* what) {
@@ -283,7 +297,10 @@ void free_desc(DeviceDesc& dd) {
   for (auto*& w : dd.wtab) { cudaFree(w); w = nullptr; }
   dd.bd = dd.bl = dd.boff = nullptr;
   dd.tables.clear();
-  for (auto& sl : dd.plans) cudaFree(sl.d);
+  for (auto& sl : dd.plans) {
+    cudaFree(sl.d);
+    if (sl.ready) cudaEventDestroy((cudaEvent_t)sl.ready);
+  }
   dd.plans.clear();
   if (cur >= 0 && dd.device >= 0 && dd.device != cur) cudaSetDevice(cur);
 }
@@ -454,6 +471,8 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
   for (auto& sl : dd.plans) {
     if (sl.d && sl.count == count && sl.pos == P.pos && sl.len == P.len && sl.nw == nw && sl.alpha == alpha &&
         sl.tsize == P.tsize && sl.gran == gran) {
+      // the plan was filled by a kernel on sl.made_on: another stream must wait for it
+      if ((void*)s != sl.made_on) CU(cudaStreamWaitEvent(s, (cudaEvent_t)sl.ready, 0));
       *out = (const PlanEnt*)sl.d;
       return DT_OK;
     }
@@ -477,6 +496,9 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
   k_plan<<<(unsigned)((nw + 1 + 255) / 256), 256, 0, s>>>(P, alpha, make_fd((uint64_t)ce), ce, C0, C1, nw,
                                                           gran, (PlanEnt*)sl.d);
   CU(cudaGetLastError());
+  if (!sl.ready) CU(cudaEventCreateWithFlags((cudaEvent_t*)&sl.ready, cudaEventDisableTiming));
+  CU(cudaEventRecord((cudaEvent_t)sl.ready, s));
+  sl.made_on = (void*)s;
   sl.count = count;
   sl.pos = P.pos;
   sl.len = P.len;
@@ -618,8 +640,7 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
 }
 
 static int seg_occupancy(bool unpack, bool single) {
-  static int occ[2][2] = {{0, 0}, {0, 0}};
-  int& o = occ[unpack][single];
+  int& o = devl().seg_occ[unpack][single];
   if (!o) {
     const void* f = unpack ? (single ? (const void*)k_seg<true, true> : (const void*)k_seg<true, false>)
                            : (single ? (const void*)k_seg<false, true> : (const void*)k_seg<false, false>);
@@ -694,7 +715,7 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     const int nwc = 8;
     const size_t tabB = std::max<size_t>((size_t)R.RB * R.nwr * 2, (size_t)(R.spanB / g) * 2);
     const size_t smem = (size_t)nwc * R.RB * R.spanB + (size_t)nwc * R.RB * 8 + ((tabB + 15) & ~size_t(15));
-    static bool attr = false;
+    bool& attr = devl().rec_attr;
     if (!attr) {
       const void* fs[] = {(const void*)k_rec<false, 4>, (const void*)k_rec<false, 8>, (const void*)k_rec<false, 16>,
                           (const void*)k_rec<true, 4>,  (const void*)k_rec<true, 8>,  (const void*)k_rec<true, 16>};
@@ -748,7 +769,7 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     P.nwords = (int32_t)(f.tsize() / g);
     const size_t smem = (size_t)kStageBufs * kStageTile + sizeof(int32_t) * (size_t)P.nwords;
     const int64_t ntiles = (len + kStageTile - 1) / kStageTile;
-    static bool attr_set = false;
+    bool& attr_set = devl().stage_attr;
     if (!attr_set) {
       const void* fs[] = {(const void*)k_stage<false, 4>, (const void*)k_stage<false, 8>,
                           (const void*)k_stage<false, 16>, (const void*)k_stage<true, 4>,
@@ -770,14 +791,14 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
   } else if (kind == 7) {
     P.fnb = make_fd((uint64_t)P.nblocks);
     const size_t smem = 8 * (size_t)kSpanWarpSmem;
-    static bool attr = false;
+    bool& attr = devl().span_attr;
     if (!attr) {
       const void* fs[] = {(const void*)k_span<false, 4>, (const void*)k_span<false, 8>, (const void*)k_span<false, 16>,
                           (const void*)k_span<true, 4>,  (const void*)k_span<true, 8>,  (const void*)k_span<true, 16>};
       for (const void* fp : fs) cudaFuncSetAttribute(fp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       attr = true;
     }
-    static int occ = 0;
+    int& occ = devl().span_occ;
     if (!occ && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_span<false, 4>, 256, smem) != cudaSuccess ||
                  occ < 1))
       occ = 1;
@@ -826,7 +847,7 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     const int64_t nvec = (len + vw - 1) / vw;
     size_t smem = sizeof(int32_t) * (size_t)P.nwords;
     // one wave of resident CTAs (grid-stride loop inside)
-    static int occ_w = 0;
+    int& occ_w = devl().word_occ;
     if (!occ_w && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_w, k_word<false, 4, 16>, 256, 4096) !=
                        cudaSuccess || occ_w < 1))
       occ_w = 4;
@@ -1157,7 +1178,7 @@ static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, i
   const int sms = num_sms();
   if (kind == 4) {  // staged: cp.async gathers by S into smem tiles, scatter by R
     const size_t smem2 = (size_t)kStageBufs * kStageTile + sizeof(int32_t) * (size_t)(S.nwords + R.nwords);
-    static bool attr = false;
+    bool& attr = devl().dual_attr;
     if (!attr) {
       cudaFuncSetAttribute(k_dual_stage<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
       cudaFuncSetAttribute(k_dual_stage<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);

@@ -59,7 +59,8 @@ class HaloPlan:
     recv_types: dict
 
     def exchange(self, comm, buf, stream=None, faces=FACES):
-        """Post all 12 transfers of one exchange as one group.  The message sent
+        """Post the transfers sent through `faces` (all 12 of an exchange by
+        default) as one group.  The message sent
         through face f is received by the neighbour through its face OPPOSITE[f];
         messages between the same pair are matched in posting order, so both sides
         post in one global order keyed by the SENDER's face f: sends go out in
@@ -68,7 +69,7 @@ class HaloPlan:
         same FACES order.  With 2 ranks per dimension both x neighbours are the
         same rank, and this ordering still pairs x- sends with x+ ghosts."""
         comm.group_start()
-        for kind, face, peer in self.ops():
+        for kind, face, peer in self.ops(faces):
             if kind == "send":
                 comm.sendrecv(buf, 1, self.send_types[face], peer, None, 0, None, -1, stream=stream)
             else:

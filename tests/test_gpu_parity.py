@@ -69,6 +69,41 @@ def check_pack_unpack(torch, recipe, origin, parent, count=1, pos=0, nbytes=None
     assert np.array_equal(d[GUARD:GUARD + len(dst_h)], dst_h), "unpack mismatch"
 
 
+def _oracle_overlaps(ot, count):
+    """True iff the typemap of `count` instances has two entries sharing a byte
+    (reading A9: such a map may be packed but not unpacked)."""
+    kk, dd = ot.typemap()
+    ext = ot.extent
+    iv = sorted((k * ext + int(d), k * ext + int(d) + oracle.BASIC_SIZE[int(kind)])
+                for k in range(count) for kind, d in zip(kk, dd))
+    return any(b[0] < a[1] for a, b in zip(iv, iv[1:]))
+
+
+def check_or_overlap(torch, r, origin, parent, count, **kw):
+    """check_pack_unpack; a DT_ERR_OVERLAP is accepted only when the oracle's own
+    typemap of `count` instances really overlaps (no silent false rejection)."""
+    try:
+        check_pack_unpack(torch, r, origin, parent, count=count, **kw)
+    except Exception as e:  # noqa: BLE001
+        if "DT_ERR_OVERLAP" not in str(e):
+            raise
+        assert _oracle_overlaps(oracle.from_recipe(r), count), ("false DT_ERR_OVERLAP", r, count)
+
+
+def check_empty(torch, recipe, count, pos=0, nbytes=64):
+    """Count 0 or size 0 (SURVEY §8(b) errors): DT_OK, 0 bytes, nothing written."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    t = dt.from_recipe(recipe).commit()
+    src = torch.full((4096,), 0x5A, dtype=torch.uint8, device="cuda")
+    out = _poisoned(torch, 64)
+    assert dt.pack(t, count, src.data_ptr() + 2048, out.data_ptr() + GUARD, pos, nbytes) == 0
+    dst = _poisoned(torch, 4096)
+    pk = torch.full((64,), 0x3C, dtype=torch.uint8, device="cuda")
+    assert dt.unpack(t, count, pk, dst.data_ptr() + GUARD + 2048, pos, nbytes) == 0
+    torch.cuda.synchronize()
+    assert bool((out == 0xA5).all()) and bool((dst == 0xA5).all()), "empty request wrote bytes"
+
+
 # ------------------------------------------------------------------ the paper's workloads at full size
 @pytest.mark.parametrize("r0c0", [(0, 0), (1, 1), (3, 7)])
 def test_c1_submatrix(torch_cuda, r0c0):
@@ -154,7 +189,8 @@ def test_random_tiny_types(torch_cuda):
     for i, r in enumerate(tys[::3]):
         ot = oracle.from_recipe(r)
         info = ot.info()
-        if info["size"] == 0:
+        if info["size"] == 0:   # size 0: DT_OK, no bytes, nothing written
+            check_empty(torch_cuda, r, int(rng.integers(0, 4)))
             continue
         lo = min(0, info["true_lb"], info["true_lb"] + 2 * info["extent"])
         hi = max(info["true_ub"], info["true_ub"] + 2 * info["extent"], 1)
@@ -162,12 +198,8 @@ def test_random_tiny_types(torch_cuda):
         total = count * info["size"]
         a, b = sorted(rng.integers(0, total + 1, size=2))
         # overlapping typemaps are only packed (unpack is rejected, reading A9)
-        try:
-            check_pack_unpack(torch_cuda, r, -lo + 16, hi - lo + 32, count=count, pos=int(a), nbytes=int(b - a),
-                              seed=i, origin_pad=int(rng.integers(0, 16)))
-        except Exception as e:  # noqa: BLE001
-            if "DT_ERR_OVERLAP" not in str(e):
-                raise
+        check_or_overlap(torch_cuda, r, -lo + 16, hi - lo + 32, count, pos=int(a), nbytes=int(b - a),
+                         seed=i, origin_pad=int(rng.integers(0, 16)))
 
 
 @pytest.mark.parametrize("kind", ["1", "2", "3", "4", "6", "7"])
@@ -432,18 +464,15 @@ def test_random_types_forced_block_spans(torch_cuda, monkeypatch):
     for i, r in enumerate(_tiny_types()[1::3]):
         info = oracle.from_recipe(r).info()
         if info["size"] == 0:
+            check_empty(torch_cuda, r, int(rng.integers(0, 4)))
             continue
         lo = min(0, info["true_lb"], info["true_lb"] + 2 * info["extent"])
         hi = max(info["true_ub"], info["true_ub"] + 2 * info["extent"], 1)
         count = int(rng.integers(1, 4))
         total = count * info["size"]
         a, b = sorted(rng.integers(0, total + 1, size=2))
-        try:
-            check_pack_unpack(torch_cuda, r, -lo + 16, hi - lo + 32, count=count, pos=int(a), nbytes=int(b - a),
-                              seed=i, origin_pad=int(rng.integers(0, 16)))
-        except Exception as e:  # noqa: BLE001
-            if "DT_ERR_OVERLAP" not in str(e):
-                raise
+        check_or_overlap(torch_cuda, r, -lo + 16, hi - lo + 32, count, pos=int(a), nbytes=int(b - a),
+                         seed=i, origin_pad=int(rng.integers(0, 16)))
 
 
 @pytest.mark.parametrize("seed", [1, 2, 3])
@@ -470,3 +499,72 @@ def test_random_irregular_struct_lists(torch_cuda, seed):
         a = int(rng.integers(0, total // 4)) * 4
         b = int(rng.integers(a // 4, total // 4 + 1)) * 4
         check_pack_unpack(torch_cuda, rec_t, org, parent + ext, count=count, pos=a, nbytes=b - a, seed=a)
+
+
+# ------------------------------------------------------------------ derived old types (VERDICT r01 pin gap)
+_R8 = ("resized", ("basic", "INT32"), 0, 8)
+_SDI = ("struct", [1, 1], [0, 8], [("basic", "DOUBLE"), ("basic", "INT32")])
+_SHB = ("struct", [1, 1], [0, 2], [("basic", "INT16"), ("basic", "BYTE")])
+
+
+def _transpose(n):
+    """MPI transpose idiom: contiguous(N, resized(vector(N,1,N,DOUBLE),0,8)) reads an
+    N x N column-major f64 matrix row by row (extent 8 per column type)."""
+    return ("contiguous", n, ("resized", ("vector", n, 1, n, ("basic", "DOUBLE")), 0, 8)), 0, n * n * 8
+
+
+@pytest.mark.parametrize("name", ["vec_resized", "idx_struct", "iblk_resized", "vec_struct16", "hidx_struct",
+                                  "transpose64", "transpose300"])
+def test_derived_old_types(torch_cuda, name):
+    """vector / indexed / indexed_block / hindexed over old types whose extent differs
+    from their size (resized, padded structs; MPI-3.1 §4.1.2, the constructors the paper
+    relies on [L14:c1262 §3]), and the transpose idiom -- whole streams, counts 1-3,
+    ragged fragments, every kernel family the planner picks."""
+    rng = np.random.default_rng(hash(name) % 1000)
+    mk = {
+        "vec_resized": lambda: (("vector", 3000, 1, 3, _R8), 0, 3000 * 24 + 64),
+        "idx_struct": lambda: (("indexed", [1, 2, 1] * 700, list(range(0, 2800 * 3, 4)), _SDI), 0, 2800 * 3 * 16 + 64),
+        "iblk_resized": lambda: (("indexed_block", 2, list(range(0, 4000 * 5, 5)), _R8), 0, 4000 * 5 * 8 + 64),
+        "vec_struct16": lambda: (("vector", 2000, 3, 5, _SHB), 0, 2000 * 5 * 4 + 64),
+        "hidx_struct": lambda: (("hindexed", [2, 1] * 600, list(range(0, 1200 * 100, 100)), _SDI), 0, 1200 * 100 + 64),
+        "transpose64": lambda: _transpose(64),
+        "transpose300": lambda: _transpose(300),
+    }
+    rec, org, parent = mk[name]()
+    ot = oracle.from_recipe(rec)
+    size, ext = ot.size, ot.extent
+    check_pack_unpack(torch_cuda, rec, org, parent)
+    for count in (2, 3):
+        total = count * size
+        a, b = sorted(int(x) for x in rng.integers(0, total + 1, size=2))
+        check_or_overlap(torch_cuda, rec, org, parent + (count - 1) * abs(ext) + 64, count, pos=a, nbytes=b - a,
+                         origin_pad=int(rng.integers(0, 16)))
+
+
+def test_transpose_idiom_equals_numpy(torch_cuda):
+    """Transpose idiom on the GPU against numpy's transpose of the same bytes (an
+    independent library routine): pack(contiguous(N, resized(vector(N,1,N)))) of a
+    column-major A == A.T raveled column-major."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    n = 257
+    rec, org, parent = _transpose(n)
+    src_h = fill_bytes(parent, 0x7A)
+    A = src_h.view(np.float64).reshape(n, n).T      # A[r, c], column-major storage
+    exp = np.ascontiguousarray(A.T).ravel(order="F").view(np.uint8)
+    t = dt.from_recipe(rec).commit()
+    out = torch.empty(len(exp), dtype=torch.uint8, device="cuda")
+    dt.pack(t, 1, _dev(torch, src_h), out)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), exp)
+
+
+@pytest.mark.parametrize("recipe", [("vector", 5, 2, 3, ("basic", "INT32")), _SDI,
+                                    ("indexed", [0, 0], [1, 2], ("basic", "DOUBLE")),
+                                    ("contiguous", 0, ("basic", "BYTE"))],
+                         ids=["vector", "struct", "size0_indexed", "size0_contig"])
+def test_count_or_size_zero(torch_cuda, recipe):
+    """count 0, size 0 and pos beyond the stream: DT_OK, 0 bytes, destination untouched."""
+    check_empty(torch_cuda, recipe, 0)
+    check_empty(torch_cuda, recipe, 0, nbytes=0)
+    check_empty(torch_cuda, recipe, 2, pos=1 << 20)

@@ -361,6 +361,37 @@ def test_hybrid_halo_single_rank(torch_cuda, ring):
     comm.free()
 
 
+@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+def test_halo_exchange_face_subset(torch_cuda, ring):
+    """exchange(faces=xs) posts only the x transfers: the x ghost layers are filled,
+    the y/z ghost layers keep their poison (the subset was ignored)."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import FACES, face_box, make_plan
+    n, h = 40, 1
+    L = n + 2 * h
+    comm = dt.Comm(0, 1, 0, chunk_bytes=8 << 10, depth=2, ring_loopback=ring)
+    hp = make_plan(0, n, h, dims=(1, 1, 1))
+    A = np.full((L, L, L), 0xA5A5A5A5, dtype=np.uint32)
+    z, y, x = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
+    A[h:h + n, h:h + n, h:h + n] = (z * 1000000 + y * 1000 + x).astype(np.uint32)
+    buf = torch.from_numpy(A.view(np.uint8).reshape(-1).copy()).cuda()
+    hp.exchange(comm, buf, faces=("x-", "x+"))
+    torch.cuda.synchronize()
+    comm.check()
+    B = buf.cpu().numpy().view(np.uint32).reshape(L, L, L)
+    for f in FACES:
+        sub, st = face_box(f, n, h, ghost=True)
+        zz, yy, xx = np.meshgrid(*[np.arange(s_, s_ + k) for s_, k in zip(st, sub)], indexing="ij")
+        if f[0] == "x":
+            exp = (((zz - h) % n) * 1000000 + ((yy - h) % n) * 1000 + ((xx - h) % n)).astype(np.uint32)
+            assert np.array_equal(B[zz, yy, xx], exp), f
+        else:
+            assert np.all(B[zz, yy, xx] == 0xA5A5A5A5), f
+    comm.free()
+
+
 def test_direct_plan_errors(torch_cuda):
     import torch
 

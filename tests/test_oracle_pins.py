@@ -200,6 +200,24 @@ def _tiny_types():
     for d0, d1 in itertools.product(range(0, 17, 3), range(0, 17, 4)):
         out.append(("struct", [1, 2], [d0, d1], [I, Dd]))
         out.append(("struct", [2, 1], [d0, d1], [("resized", I, -2, 8), Bt]))
+    # derived old types whose extent != size (MPI-3.1 §4.1.2: strides and element
+    # displacements count in extent(old) units) and structs whose largest basic
+    # alignment is < 8 (the ε rule rounds to that alignment, reading A8)
+    S16 = ("basic", "INT16")
+    R8 = ("resized", I, 0, 8)
+    SDI = ("struct", [1, 1], [0, 8], [Dd, I])
+    SHB = ("struct", [1, 1], [0, 2], [S16, Bt])
+    for old in (R8, SDI, SHB, ("resized", Bt, -1, 3)):
+        for c, b, s in itertools.product(range(1, 4), range(1, 3), (-2, 1, 3)):
+            out.append(("vector", c, b, s, old))
+        for dp in [(0, 2), (3, 0), (1, 5)]:
+            out.append(("indexed", [1, 2], list(dp), old))
+            out.append(("indexed_block", 2, list(dp), old))
+            out.append(("hindexed", [2, 1], [dp[0] * 5, dp[1] * 7], old))
+    for d0, d1 in itertools.product(range(0, 9, 2), range(0, 9, 3)):
+        out.append(("struct", [1, 1], [d0, d1], [S16, Bt]))
+        out.append(("struct", [2, 1], [d0, d1], [Bt, ("basic", "FLOAT")]))
+    out.append(("contiguous", 3, ("resized", ("vector", 3, 1, 3, Dd), 0, 8)))
     out.append(("contiguous", 3, ("vector", 2, 1, 3, Dd)))
     out.append(("hvector", 2, 2, 64, ("struct", [1, 1], [0, 8], [Dd, I])))
     out.append(("subarray", [3, 4, 2], [2, 2, 1], [1, 0, 1], "F", ("vector", 2, 1, 2, I)))
@@ -325,3 +343,14 @@ def test_addr_of_matches_typemap():
     ext = t.extent
     ps2 = ps + len(addrs)
     assert np.array_equal(oracle.addr_of(t, 2, ps2), addrs[ps] + ext)
+
+
+def test_oracle_mutants_killed():
+    """Each deliberate bug in oracle.c (tools/oracle_mutants.py: extent-vs-size
+    scaling in vector/indexed/hindexed/contiguous, a dropped j*extent term, the struct
+    ε rule) makes at least one pin above fail."""
+    import subprocess
+    import sys
+    tool = os.path.join(os.path.dirname(HERE), "tools", "oracle_mutants.py")
+    r = subprocess.run([sys.executable, tool], capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout + r.stderr
