@@ -173,7 +173,8 @@ dt_status dt_type_deserialize(const void* in, size_t nbytes, dt_t* out);
 enum { DT_XFER_P2P = 0, DT_XFER_NCCL = 1 };
 typedef struct {
   int64_t chunk_bytes; /* pipeline fragment size C (reading A15); 0 = default 1 MiB        */
-  int32_t depth;       /* ring slots D per peer; 0 = default 8                             */
+  int32_t depth;       /* ring slots D (fragments in flight) per (peer, channel), <= 256;
+                          0 = auto: D*C >= 8 MiB, at least 4 slots (NCCL mode: 4)      */
   int32_t mode;        /* DT_XFER_P2P (pack straight into the peer's ring over NVLink) or
                           DT_XFER_NCCL (double-buffered ncclSend/ncclRecv of packed chunks) */
   int32_t ctas;        /* CTAs per direction for the P2P pipeline kernel; 0 = default      */
@@ -182,9 +183,13 @@ typedef struct {
 } dt_xfer_opts;
 
 /* Create this rank's endpoint on `device`: allocates the receive rings
- * (nranks*depth*chunk bytes) and flag words, and (mode NCCL) initialises a
- * NCCL communicator from `nccl_unique_id` (128 B, H; may be NULL for P2P).
- * The handle is single-threaded. */
+ * (nranks*6 channels*depth*chunk bytes) and flag words, and (mode NCCL)
+ * initialises a NCCL communicator from `nccl_unique_id` (128 B, H; may be NULL
+ * for P2P).  Every rank must use the same chunk_bytes, depth and mode
+ * (dt_comm_connect checks; DT_ERR_ARG otherwise).  The handle is single-threaded
+ * and its operations must be stream-ordered (one stream, or joined streams): a
+ * receive posts "start packing" when its kernel starts, which tells the sender
+ * that the previous message on the channel has been consumed. */
 dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int device, const dt_xfer_opts* o,
                        dt_comm_t* out);
 /* NCCL unique id for rank 0 to broadcast (H buffer of 128 bytes). */
@@ -194,7 +199,7 @@ dt_status dt_comm_local_handle(dt_comm_t c, void* out, size_t* nbytes);
 /* After the caller all-gathered every rank's handle blob (H, nranks *
  * nbytes_per_rank, rank-major): map every peer's ring/flags once
  * (cudaIpcOpenMemHandle; [L20:c3807 §4.1]).  Same-process peers (loopback) are
- * recognised and not re-mapped. */
+ * recognised and not re-mapped.  DT_ERR_ARG if a peer's chunk/depth/mode differ. */
 dt_status dt_comm_connect(dt_comm_t c, const void* all_handles, size_t nbytes_per_rank);
 /* Send scount instances of stype from sbuf (D) to rank `dest` and receive into
  * rbuf (D) rcount instances of rtype from rank `source` (either may be -1 =
@@ -202,7 +207,8 @@ dt_status dt_comm_connect(dt_comm_t c, const void* all_handles, size_t nbytes_pe
  * [L26:c1686]).  Signatures may differ as long as the byte counts fit
  * (reading A12): the receive fills a prefix; scount*size(stype) >
  * rcount*size(rtype) of the matching peer is DT_ERR_TRUNCATE, detected before
- * any byte moves (the byte count travels with the first fragment's flag).
+ * any byte moves (the receiver posts its capacity with "start packing"
+ * [L20:c3973], the sender compares before its first fragment).
  * Pipelined in fragments of chunk_bytes through `depth` ring slots: cost ~
  * transfer + one fragment's pack/unpack ([L18:c4932 §4.1]).  Enqueued on
  * `stream`; returns without host synchronisation (P2P mode). */

@@ -1447,6 +1447,22 @@ __device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
 __device__ __forceinline__ void red_release_sys_add(uint64_t* p, uint64_t v) {
   asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+// scope-selected flag operations: .gpu when both sides of a flag run on this GPU
+// (loopback, two processes sharing a device), .sys across GPUs (NVLink peers)
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p, bool sys) {
+  uint64_t v;
+  if (sys) asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  else asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v, bool sys) {
+  if (sys) asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  else asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v, bool sys) {
+  if (sys) asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  else asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -1458,15 +1474,15 @@ enum { XERR_TIMEOUT = 1, XERR_TRUNCATE = 2 };
 // spin until pred(*p) holds; false on timeout (sets *err)
 template <typename Pred>
 __device__ __forceinline__ bool spin(const uint64_t* p, Pred pred, int64_t timeout_ns, int32_t* err, uint64_t* out,
-                                     bool sleep = true) {
-  uint64_t v = ld_acquire_sys(p);
+                                     bool sleep = true, bool sys = true) {
+  uint64_t v = ld_acquire(p, sys);
   if (pred(v)) { *out = v; return true; }
   const uint64_t t0 = gtimer();
   int ns = 32;
   while (true) {
     if (sleep) __nanosleep(ns);
     if (ns < 256) ns <<= 1;
-    v = ld_acquire_sys(p);
+    v = ld_acquire(p, sys);
     if (pred(v)) { *out = v; return true; }
     if ((int64_t)(gtimer() - t0) > timeout_ns) {
       atomicCAS(err, 0, XERR_TIMEOUT);

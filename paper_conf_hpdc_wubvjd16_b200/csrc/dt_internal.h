@@ -153,6 +153,15 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
 int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
                 int64_t* gran);
 void build_levels(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count, KLevels& L);
+// Effective template of one launch: a single-block template whose innermost regular
+// level continues the run (count instances of a contiguous type, a vector of
+// adjacent blocks) becomes one longer run when that makes it a long-run copy.
+struct Eff {
+  KLevels L;
+  int64_t tsize, nblocks, bd0, bl0;
+  bool merged;
+};
+Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count);
 dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out);
 const Form& get_form(dt_type_s* t);
 // xfer.cu: identity of a communicator (direct exchange plans live beside it)

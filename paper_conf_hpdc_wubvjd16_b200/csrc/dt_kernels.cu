@@ -419,12 +419,7 @@ static bool template_fits_int32(const Form& f) {
 // Effective template of one launch: a single-block template whose innermost
 // regular level continues the run (e.g. count instances of a contiguous type)
 // becomes one longer run, when that makes it a long-run copy.
-struct Eff {
-  KLevels L;
-  int64_t tsize, nblocks, bd0, bl0;
-  bool merged;
-};
-static Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count) {
+Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count) {
   Eff E;
   build_levels(f, dd, t, count, E.L);
   E.tsize = f.tsize();

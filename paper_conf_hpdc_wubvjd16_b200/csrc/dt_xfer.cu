@@ -10,17 +10,17 @@
 // ([L20:c3973]); the sender signals "unpack fragment i" ([L20:c3380]) and the
 // receiver acks ([L20:c4133]).
 //
-// B200 design (DESIGN.md §Transfer):
+// B200 design (DESIGN.md §7):
 //  * P2P mode: ONE persistent kernel per call (or per group of calls) whose
-//    send-role CTAs pack fragment k straight into the receiver's ring slot k%D in
-//    peer HBM over NVLink (remote 16-byte stores), then publish it with a
-//    release.sys add of the bytes written to the receiver's ready[slot]; the
-//    receive-role CTAs spin (ld.acquire.sys) on their local ready[slot], unpack
-//    the slot into the user's layout and add the bytes consumed to the sender's
-//    ack[slot].  Chunk != launch: the chunk size only sets flow-control
-//    granularity.  Counters are cumulative bytes per slot; each side keeps its
-//    base per (peer, channel) in device memory, double-buffered by message parity.
-//    Header {seq, nbytes} + "go" word implement the handshake and truncation check.
+//    send-role CTAs pack pieces of fragment k straight into the receiver's ring
+//    slot k%D in peer HBM over NVLink, then publish each piece with a system-scope
+//    release store of a tag (seq, round) into the receiver's ready flag; the
+//    receive-role CTAs spin (ld.acquire.sys) on their local ready flags, unpack the
+//    piece into the user's layout and release the tag into the sender's ack flag.
+//    Chunk != launch: the chunk size only sets flow-control granularity.  The
+//    receiver posts {capacity, seq} ("start packing") at kernel start; the sender
+//    answers with the header {seq, n | abort, pieces, teams}.  The grid is sized to
+//    the message (pieces of >= 32 KiB, teams of CTAs taking alternate fragments).
 //  * NCCL mode: double-buffered chunks: pack(k) -> ncclSend/ncclRecv -> unpack(k)
 //    on three internal streams with per-slot events.
 #include <cuda_runtime.h>
@@ -28,6 +28,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <vector>
@@ -38,9 +39,17 @@
 namespace dt {
 
 constexpr int kMaxOps = 16;
-constexpr int kMaxCh = 6;   // concurrent messages per (pair, direction) inside one group
-constexpr int kMaxSub = 64; // sub-rings (one per sending CTA) per message
+constexpr int kMaxCh = 6;    // concurrent messages per (pair, direction) inside one group
+constexpr int kMaxSub = 64;  // pieces (sub-rings) per fragment
+constexpr int kMaxDepth = 256;  // ring slots per (pair, channel)
 constexpr uint64_t kAbort = 1ull << 63;
+
+// Flag values are tags: (message sequence number << 32) | (round + 1).  They only
+// grow on a (pair, channel), so a waiter compares with >= and nothing is ever reset
+// or carried between messages.  Round r of slot s is fragment r*D + s.
+__host__ __device__ __forceinline__ uint64_t xtag(uint64_t seq, int64_t round) {
+  return (seq << 32) | (uint64_t)(round + 1);
+}
 
 struct XOp {
   KP P;            // pack (send role) or unpack (recv role) over the user's layout
@@ -49,15 +58,15 @@ struct XOp {
   int32_t single;  // segment walk over a single-block template
   int32_t g;       // word granularity
   int64_t n;       // send: bytes; recv: capacity in bytes
-  int64_t chunk;
-  int32_t depth, cta0, ncta, rep;  // rep (send role): CTAs per sub-ring, alternating fragments
+  int64_t chunk;   // C: fragment bytes (one ring slot)
+  int32_t depth, cta0, ncta;
+  int32_t gs, rep;  // send role: pieces per fragment, teams (fragment k -> team k % rep)
+  int32_t sys;      // flag scope: 1 = system (peer on another GPU), 0 = gpu (same device)
   uint8_t* ring;   // slot 0 of the (pair, channel) ring (send: peer memory; recv: local)
-  uint64_t* ready; // [depth]  send: peer; recv: local
-  uint64_t* ack;   // [depth]  send: local; recv: peer
-  uint64_t* hdr;   // [2] {seq, nbytes}  send: peer; recv: local
-  uint64_t* go;    // [1]     send: local; recv: peer
-  const uint64_t* base_in;  // [depth] cumulative bytes per slot before this message
-  uint64_t* base_out;       // [depth] after it
+  uint64_t* ready; // [depth][kMaxSub] tags  send: peer; recv: local
+  uint64_t* ack;   // [depth][kMaxSub] tags  send: local; recv: peer
+  uint64_t* hdr;   // [4] {seq, nbytes|abort, gs, rep}  send: peer; recv: local
+  uint64_t* go;    // [2] {capacity, seq}  send: local; recv: peer
   uint64_t seq;
   int32_t* err;
   RecGeo rg;       // kind 6: record-span geometry (per-fragment element range set on the device)
@@ -66,120 +75,175 @@ struct XOp {
 struct XArgs {
   int32_t nops;
   int32_t wt_off;  // byte offset of the word table in dynamic smem (after the staging buffers)
-  int32_t flags;
-  int32_t pad2;  // tuning switches (DT_XFER_FLAGS): bit1 = no sleep in polls, bit2 = SC system fence before each flag
+  int32_t flags;   // DT_XFER_FLAGS: bit1 = no sleep in polls, bit2 = SC system fence before each flag
+  int32_t pad2;
   int64_t timeout_ns;
+  uint64_t* trace;  // diagnostics (DT_XFER_TRACE): per-piece globaltimer stamps of the first CTAs
   XOp ops[kMaxOps];
 };
+constexpr int kTraceCtas = 4, kTracePieces = 64;
+__device__ __forceinline__ void xtrace(const XArgs& A, int op, int j, int idx, int point) {
+  if (A.trace && j < kTraceCtas && idx < kTracePieces)
+    A.trace[(((size_t)op * kTraceCtas + j) * kTracePieces + idx) * 4 + point] = gtimer();
+}
 
-// pack or unpack stream bytes [lo, lo+len) of the current chunk with this CTA.
-// cb: the slot base such that stream byte x of the message lives at cb + x.  The
-// op's parameters stay in the grid-constant bank (no per-fragment struct copy).
-template <bool UNPACK>
-__device__ __forceinline__ void cta_chunk(const XOp& X, uint8_t* cb, int64_t lo, int64_t len, const int32_t* wt,
-                                          uint8_t* sbuf, uint64_t* mbar) {
-  const KP& P = X.P;
-  const int64_t hi = lo + len;
+// ---- per-family piece copies.  Each is a separate (noinline) function so that
+// ptxas compiles the families one at a time instead of one giant kernel body.
+// The op's parameters stay in the grid-constant bank (X refers to it).
+template <bool UNPACK, bool SINGLE>
+__device__ __noinline__ void xc_seg(const XOp& X, uint8_t* cb, int64_t a, int64_t b, int lane) {
   constexpr int POL = UNPACK ? LD_CG : LD_CS;  // ring slots are rewritten by the peer: bypass L1
-  if (X.kind == 6) {  // record spans: the CTA's warps take RB-record batches of the fragment
-    const int64_t hb = hi - len % X.g;  // a ragged tail (< G bytes, last fragment) is walked below
-    RecGeo R = X.rg;
-    R.e_lo = lo / P.tsize;
-    R.e_hi = (hb + P.tsize - 1) / P.tsize;
-    R.b0 = R.e_lo & ~int64_t(31);
-    R.nbatch = (R.e_hi - R.b0 + R.RB - 1) / R.RB;
-    const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5;
-    uint8_t* buf = sbuf + w * (R.RB * R.spanB);
-    int64_t* sd = reinterpret_cast<int64_t*>(sbuf + nwc * (R.RB * R.spanB)) + w * R.RB;
-    uint16_t* omap = reinterpret_cast<uint16_t*>(sbuf + nwc * (R.RB * R.spanB) + nwc * R.RB * 8);
-    const int lane = threadIdx.x & 31;
+  seg_range<UNPACK, SINGLE, POL>(X.P, cb, a, b, lane);
+}
+
+template <bool UNPACK, int G>
+__device__ __noinline__ void xc_rec(const XOp& X, uint8_t* cb, int64_t lo, int64_t hb, uint8_t* sbuf) {
+  constexpr int POL = UNPACK ? LD_CG : LD_CS;
+  const KP& P = X.P;
+  RecGeo R = X.rg;
+  R.e_lo = lo / P.tsize;
+  R.e_hi = (hb + P.tsize - 1) / P.tsize;
+  R.b0 = R.e_lo & ~int64_t(31);
+  R.nbatch = (R.e_hi - R.b0 + R.RB - 1) / R.RB;
+  const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint8_t* buf = sbuf + w * (R.RB * R.spanB);
+  int64_t* sd = reinterpret_cast<int64_t*>(sbuf + nwc * (R.RB * R.spanB)) + w * R.RB;
+  uint16_t* omap = reinterpret_cast<uint16_t*>(sbuf + nwc * (R.RB * R.spanB) + nwc * R.RB * 8);
+  rec_range<UNPACK, G, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane);
+}
+
+template <bool UNPACK, int G>
+__device__ __noinline__ void xc_span(const XOp& X, uint8_t* cb, int64_t a, int64_t b, uint8_t* sm, int lane) {
+  constexpr int POL = UNPACK ? LD_CG : LD_CS;
+  const PlanEnt st = span_start(X.P, a, lane);
+  span_range<UNPACK, G, POL>(X.P, cb, st, b, lane, sm);
+}
+
+template <bool UNPACK, int G>
+__device__ __noinline__ void xc_stage(const XOp& X, uint8_t* cb, const int32_t* wt, int64_t lo, int64_t bh,
+                                      uint8_t* sbuf, uint64_t* mbar) {
+  if (UNPACK) stage_unpack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf, mbar);
+  else stage_pack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf);
+}
+
+template <bool UNPACK, int G>
+__device__ __noinline__ void xc_word(const XOp& X, uint8_t* cb, int64_t lo, int64_t hi, const int32_t* wt) {
+  constexpr int POL = UNPACK ? LD_CG : LD_CS;
+  // few CTAs carry the whole transfer: keep 4 vectors per thread in flight (512 threads: 32 KiB/CTA)
+  word_range<UNPACK, G, 16, POL, (G >= 4 ? 4 : 2)>(X.P, cb, lo, hi, wt, threadIdx.x, blockDim.x);
+}
+
+// pack or unpack stream bytes [lo, lo+len) of one piece with this CTA.
+// cb: the slot base such that stream byte x of the message lives at cb + x.
+template <bool UNPACK>
+__device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo, int64_t len, const int32_t* wt,
+                                          uint8_t* sbuf, uint64_t* mbar) {
+  const int64_t hi = lo + len;
+  const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (X.kind == 6) {  // record spans: the CTA's warps take RB-record batches of the piece
+    const int64_t hb = hi - len % X.g;  // a ragged tail (< G bytes, last piece) is walked below
     if (lo < hb) {
       switch (X.g) {
-        case 4: rec_range<UNPACK, 4, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane); break;
-        case 8: rec_range<UNPACK, 8, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane); break;
-        default: rec_range<UNPACK, 16, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane); break;
+        case 4: xc_rec<UNPACK, 4>(X, cb, lo, hb, sbuf); break;
+        case 8: xc_rec<UNPACK, 8>(X, cb, lo, hb, sbuf); break;
+        default: xc_rec<UNPACK, 16>(X, cb, lo, hb, sbuf); break;
       }
     }
-    if (hb < hi && w == nwc - 1) seg_range<UNPACK, false, POL>(P, cb, hb, hi, lane);
+    if (hb < hi && w == nwc - 1) xc_seg<UNPACK, false>(X, cb, hb, hi, lane);
     return;
   }
-  if (X.kind == 7) {  // block spans: the CTA's warps take equal 16-byte-multiple slices of the fragment
-    const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int64_t body = len - len % X.g;  // a ragged tail (< G bytes, last fragment) is walked below
+  if (X.kind == 7) {  // block spans: the CTA's warps take equal 16-byte-multiple slices of the piece
+    const int64_t body = len - len % X.g;
     int64_t per = (body + nwc - 1) / nwc;
     per = (per + 15) & ~int64_t(15);
     const int64_t a = lo + (int64_t)w * per, b = min(a + per, lo + body);
     if (a < b) {
-      const PlanEnt st = span_start(P, a, lane);
       uint8_t* sm = sbuf + (size_t)w * kSpanWarpSmem;
       switch (X.g) {
-        case 4: span_range<UNPACK, 4, POL>(P, cb, st, b, lane, sm); break;
-        case 8: span_range<UNPACK, 8, POL>(P, cb, st, b, lane, sm); break;
-        default: span_range<UNPACK, 16, POL>(P, cb, st, b, lane, sm); break;
+        case 4: xc_span<UNPACK, 4>(X, cb, a, b, sm, lane); break;
+        case 8: xc_span<UNPACK, 8>(X, cb, a, b, sm, lane); break;
+        default: xc_span<UNPACK, 16>(X, cb, a, b, sm, lane); break;
       }
     }
-    if (body < len && w == nwc - 1) seg_range<UNPACK, false, POL>(P, cb, lo + body, hi, lane);
+    if (body < len && w == nwc - 1) xc_seg<UNPACK, false>(X, cb, lo + body, hi, lane);
     return;
   }
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
-    const int64_t bh = hi - len % X.g;  // words; a ragged tail (< G bytes, last fragment) is walked below
-    switch (X.g) {
-      case 8:
-        if (UNPACK) stage_unpack<8, kXferStageBufs>(P, cb, wt, lo, bh, sbuf, mbar);
-        else stage_pack<8, kXferStageBufs>(P, cb, wt, lo, bh, sbuf);
-        break;
-      default:
-        if (UNPACK) stage_unpack<16, kXferStageBufs>(P, cb, wt, lo, bh, sbuf, mbar);
-        else stage_pack<16, kXferStageBufs>(P, cb, wt, lo, bh, sbuf);
-        break;
-    }
+    const int64_t bh = hi - len % X.g;
+    if (X.g == 8) xc_stage<UNPACK, 8>(X, cb, wt, lo, bh, sbuf, mbar);
+    else xc_stage<UNPACK, 16>(X, cb, wt, lo, bh, sbuf, mbar);
     if (bh < hi) {
       __syncthreads();
-      if (threadIdx.x < 32) seg_range<UNPACK, false, POL>(P, cb, bh, hi, threadIdx.x & 31);
+      if (threadIdx.x < 32) xc_seg<UNPACK, false>(X, cb, bh, hi, lane);
     }
     return;
   }
   if (X.kind == 2) {
     const int64_t body = len - len % X.g;
-    // few CTAs carry the whole transfer: keep 4 vectors per thread in flight (512 threads: 32 KiB/CTA)
     switch (X.g) {
-      case 1: word_range<UNPACK, 1, 16, POL, 2>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
-      case 2: word_range<UNPACK, 2, 16, POL, 2>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
-      case 4: word_range<UNPACK, 4, 16, POL, 4>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
-      case 8: word_range<UNPACK, 8, 16, POL, 4>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
-      default: word_range<UNPACK, 16, 16, POL, 4>(P, cb, lo, lo + body, wt, threadIdx.x, blockDim.x); break;
+      case 1: xc_word<UNPACK, 1>(X, cb, lo, lo + body, wt); break;
+      case 2: xc_word<UNPACK, 2>(X, cb, lo, lo + body, wt); break;
+      case 4: xc_word<UNPACK, 4>(X, cb, lo, lo + body, wt); break;
+      case 8: xc_word<UNPACK, 8>(X, cb, lo, lo + body, wt); break;
+      default: xc_word<UNPACK, 16>(X, cb, lo, lo + body, wt); break;
     }
-    if (body < len && threadIdx.x < 32)  // ragged tail (< G bytes): one warp walks it
-      seg_range<UNPACK, false, POL>(P, cb, lo + body, hi, threadIdx.x & 31);
+    if (body < len && threadIdx.x < 32) xc_seg<UNPACK, false>(X, cb, lo + body, hi, lane);
     return;
   }
-  const int nw = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  int64_t per = (len + nw - 1) / nw;
+  int64_t per = (len + nwc - 1) / nwc;
   per = (per + 127) & ~int64_t(127);
   const int64_t a = lo + (int64_t)w * per, b = min(a + per, hi);
-  if (X.single) seg_range<UNPACK, true, POL>(P, cb, a, b, lane);
-  else seg_range<UNPACK, false, POL>(P, cb, a, b, lane);
+  if (a < b) {
+    if (X.single) xc_seg<UNPACK, true>(X, cb, a, b, lane);
+    else xc_seg<UNPACK, false>(X, cb, a, b, lane);
+  }
 }
 
+// One persistent kernel per dt_sendrecv / dt_group: send-role and receive-role CTAs
+// of every op (co-resident: cooperative launch).
+//
+// Message protocol on a (pair, channel), sequence number seq:
+//  * receiver CTA 0 posts {capacity, seq} into the sender's `go` words at kernel
+//    start ("start packing", [L20:c3973]) -- its previous kernel on the channel has
+//    finished, so every ring slot is free;
+//  * sender thread 0 of every CTA waits for go >= seq; CTA 0 writes the header
+//    {seq, n | abort, gs, rep}: abort (n > capacity) moves nothing and both sides
+//    report DT_ERR_TRUNCATE, decided before any byte moves ([L26:c4404], A12);
+//  * the message is K = ceil(n/C) fragments ("unpack fragment i", [L20:c3380]);
+//    fragment k uses ring slot k % D, is split into gs pieces of C/gs bytes, and
+//    belongs to team k % rep.  Sender CTA (team t, piece js) packs its pieces of
+//    t's fragments straight into the receiver's slot in peer HBM and publishes each
+//    with a system-scope release store of the tag into ready[slot][js]; before
+//    reusing a slot (round r > 0) it waits for ack[slot][js] >= tag(seq, r-1).
+//  * receiver CTAs take (team, piece) pairs round-robin, wait for ready with an
+//    acquire, unpack the piece from local HBM and release the tag into the sender's
+//    ack[slot][js] ([L20:c4133]).
+// Flags are written by exactly one CTA, so plain release stores suffice, and since
+// tags only grow nothing is carried between messages.
 constexpr int kXferThreads = 512;
 __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
-  // dynamic smem: [staging buffers (if any op stages)] [word table]
+  // dynamic smem: [staging buffers / record or span buffers] [word table]
   extern __shared__ __align__(128) uint8_t xsm[];
   __shared__ uint64_t mbar[kXferStageBufs];
   uint8_t* sbuf = xsm;
   int32_t* wt = reinterpret_cast<int32_t*>(xsm + A.wt_off);
-  __shared__ uint64_t s_val;
-  __shared__ int s_stop, s_gs;
+  __shared__ uint64_t s_n;
+  __shared__ int s_stop, s_gs, s_rep;
   int op = 0;
   for (int i = 0; i < A.nops; i++)
     if ((int)blockIdx.x >= A.ops[i].cta0 && (int)blockIdx.x < A.ops[i].cta0 + A.ops[i].ncta) op = i;
   const XOp& X = A.ops[op];
   const int j = (int)blockIdx.x - X.cta0;
-  if (X.kind == 2)
+  const bool sleep_ok = !(A.flags & 2);
+
+  // the receiver's "start packing" goes out first: it is on the sender's critical path
+  if (X.role == 1 && j == 0 && threadIdx.x == 0) {
+    st_relaxed(X.go, (uint64_t)X.n, X.sys != 0);
+    st_release(X.go + 1, X.seq, X.sys != 0);
+  }
+  if (X.kind == 2 || X.kind == 4)
     for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
-  if (X.kind == 4)
-    for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
-  if (X.kind == 6) {  // record-span maps after the per-warp buffers (same layout as cta_chunk)
+  if (X.kind == 6) {  // record-span maps after the per-warp buffers (same layout as xc_rec)
     const RecGeo& R = X.rg;
     uint16_t* omap = reinterpret_cast<uint16_t*>(xsm + (blockDim.x >> 5) * (R.RB * R.spanB + R.RB * 8));
     if (X.role == 1) {
@@ -190,144 +254,106 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
                      default: rec_maps<false, 16>(R, omap); break; }
     }
   }
+  const uint64_t seq = X.seq;
+  const bool sys = X.sys != 0;
+  if (threadIdx.x == 0) {
+    uint64_t v = 0;
+    s_stop = 0;
+    if (X.role == 0) {
+      const bool ok = spin(X.go + 1, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
+      const uint64_t cap = ok ? *(volatile uint64_t*)X.go : 0;
+      const bool abort = (uint64_t)X.n > cap;
+      if (ok && j == 0) {
+        st_relaxed(X.hdr + 1, (uint64_t)X.n | (abort ? kAbort : 0), sys);
+        st_relaxed(X.hdr + 2, (uint64_t)X.gs, sys);
+        st_relaxed(X.hdr + 3, (uint64_t)X.rep, sys);
+        st_release(X.hdr, seq, sys);
+        if (abort) atomicCAS(X.err, 0, XERR_TRUNCATE);
+      }
+      s_stop = !ok || abort;
+      s_n = (uint64_t)X.n;
+      s_gs = X.gs;
+      s_rep = X.rep;
+    } else {
+      const bool ok = spin(X.hdr, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
+      const uint64_t nv = ok ? *(volatile uint64_t*)(X.hdr + 1) : 0;
+      s_gs = ok ? (int)*(volatile uint64_t*)(X.hdr + 2) : 1;
+      s_rep = ok ? (int)*(volatile uint64_t*)(X.hdr + 3) : 1;
+      s_n = nv & ~kAbort;
+      s_stop = !ok || (nv & kAbort);
+      if (ok && (nv & kAbort) && j == 0) atomicCAS(X.err, 0, XERR_TRUNCATE);
+    }
+  }
+  __syncthreads();
+  if (s_stop) return;
+  const int64_t n = (int64_t)s_n;
+  const int gs = s_gs, rep = s_rep;
   const int64_t C = X.chunk;
   const int D = X.depth;
-  if (threadIdx.x == 0) s_stop = 0;
-  __syncthreads();
-
-  // Sub-rings: step k of the message covers stream bytes [kC, (k+1)C); sub-ring
-  // js in [0, gs) carries [kC + js*Cs, kC + (js+1)*Cs), Cs = C/gs, through its own
-  // D slots and flags, so every CTA pipelines on its own (no cross-CTA wait per
-  // fragment).  The sender runs one CTA per sub-ring; receiver CTA j serves
-  // sub-rings j, j+ncta, ...
-  // Replicas: with an even depth, sub-ring js is served by `rep` CTAs that take alternate
-  // fragments (fragment k -> replica k % rep; slot k % D belongs to one replica), so two
-  // fragments of a sub-ring are in flight at once and each fragment's fixed cost (credit
-  // poll, store completion, publication) overlaps the other's copy.
-  int64_t n = X.n;
-  int gs, rep;
-  __shared__ int s_rep;
-  if (X.role == 0) {
-    rep = X.rep > 1 ? X.rep : 1;
-    gs = X.ncta / rep;
-    // ---- send role: header {seq, nbytes, gs, rep}, wait for "go" (receiver-driven, [L20:c3973])
-    if (j == 0 && threadIdx.x == 0) {
-      st_release_sys(X.hdr + 1, (uint64_t)n);
-      st_release_sys(X.hdr + 2, (uint64_t)gs);
-      st_release_sys(X.hdr + 3, (uint64_t)rep);
-      st_release_sys(X.hdr, X.seq);
-    }
-    if (threadIdx.x == 0) {
-      uint64_t v = 0;
-      const uint64_t seq = X.seq;
-      bool ok = spin(X.go, [seq](uint64_t x) { return (x & ~kAbort) >= seq; }, A.timeout_ns, X.err, &v);
-      s_stop = !ok ? 2 : (v & kAbort) ? 1 : 0;
-      if (s_stop == 1 && j == 0) atomicCAS(X.err, 0, XERR_TRUNCATE);
-    }
-    __syncthreads();
-    if (s_stop == 2) return;
-    if (s_stop == 1) n = 0;  // aborted: move nothing, carry the bases over
-  } else {
-    // ---- recv role: read the header, check capacity, send "go"
-    if (threadIdx.x == 0) {
-      uint64_t v = 0;
-      const uint64_t seq = X.seq;
-      bool ok = spin(X.hdr, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v);
-      s_val = ok ? ld_acquire_sys(X.hdr + 1) : 0;
-      s_gs = ok ? (int)ld_acquire_sys(X.hdr + 2) : 1;
-      s_rep = ok ? (int)ld_acquire_sys(X.hdr + 3) : 1;
-      s_stop = ok ? 0 : 2;
-    }
-    __syncthreads();
-    if (s_stop == 2) return;
-    n = (int64_t)s_val;
-    gs = s_gs;
-    rep = s_rep > 1 ? s_rep : 1;
-    if (n > X.n) {
-      if (j == 0 && threadIdx.x == 0) {
-        atomicCAS(X.err, 0, XERR_TRUNCATE);
-        st_release_sys(X.go, X.seq | kAbort);
-      }
-      n = 0;
-    } else if (j == 0 && threadIdx.x == 0) {
-      st_release_sys(X.go, X.seq);
-    }
-  }
-
   const int64_t Cs = C / gs;
-  const int64_t K = (n + C - 1) / C;
-  // this CTA's replica and sub-rings: sender CTA j = replica j / gs of sub-ring j % gs;
-  // receiver CTAs split into rep groups of nsub (a receiver with fewer CTAs than
-  // replicas serves every fragment)
-  int myrep = 0, js0 = j, jstep = X.ncta;
-  bool all_k = rep == 1;
-  if (X.role == 0) {
-    myrep = j / gs;
-    js0 = j % gs;
-    jstep = gs;
-  } else if (X.ncta >= rep && rep > 1) {
-    const int nsub = X.ncta / rep;
-    myrep = j / nsub;
-    js0 = j % nsub;
-    jstep = nsub;
-    if (myrep >= rep) js0 = gs;  // surplus CTA: no sub-ring
-  } else {
-    all_k = true;
-  }
-  for (int64_t k = 0; k < K; k++) {
-    if (!all_k && (int)(k % rep) != myrep) continue;
-    const int slot = (int)(k % D);
-    const int64_t round = k / D;
-    for (int js = js0; js < gs; js += jstep) {
-      const int64_t off = k * C + (int64_t)js * Cs;
-      if (off >= n) continue;
+  const int K = (int)((n + C - 1) / C);
+  const int npairs = gs * rep;
+  // Pieces of this CTA, in fragment order (32-bit index math, slot/round kept
+  // incrementally: the loop runs between every two pieces, it must cost nothing).
+  // Send role: CTA j = (team j / gs, piece j % gs), fragments j/gs, j/gs + rep, ...
+  // Receive role: pairs j, j + ncta, ... (one pair per CTA when ncta >= pairs).
+  const bool one = X.role == 0 || X.ncta >= npairs;
+  if (one && j >= npairs) return;
+  const int kstep = one ? rep : 1;
+  int k = one ? j / gs : 0;
+  int slot = k % D, round = k / D;
+  int pidx = 0;
+  for (; k < K; k += kstep) {
+    const int team = one ? 0 : k % rep;
+    int js = one ? j % gs : (((j - team * gs) % X.ncta) + X.ncta) % X.ncta;
+    const int jstep = one ? gs : X.ncta;
+    for (; js < gs; js += jstep) {
+      const int64_t off = (int64_t)k * C + (int64_t)js * Cs;
+      if (off >= n) break;
       const int64_t len = min(Cs, n - off);
-      const int fi = js * D + slot;  // flag / base index of (sub-ring, slot)
-      uint8_t* sl = X.ring + (int64_t)fi * Cs - off;  // stream byte `off` lands at the slot start
-      const uint64_t base = X.base_in[fi] + (uint64_t)round * (uint64_t)Cs;
+      const int fi = slot * kMaxSub + js;
+      const uint64_t tag = xtag(seq, round);
+      uint8_t* sl = X.ring + (int64_t)slot * C + (int64_t)js * Cs - off;  // stream byte off -> piece start
       if (threadIdx.x == 0) {
         uint64_t v;
-        bool ok;
-        const bool sl_ok = !(A.flags & 2);
-        if (X.role == 0)
-          ok = spin(X.ack + fi, [base](uint64_t x) { return x >= base; }, A.timeout_ns, X.err, &v, sl_ok);
-        else {
-          const uint64_t need = base + (uint64_t)len;
-          ok = spin(X.ready + fi, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v, sl_ok);
+        bool ok = true;
+        xtrace(A, op, j, pidx, 0);
+        if (X.role == 0) {
+          if (round > 0) {
+            const uint64_t need = xtag(seq, round - 1);
+            ok = spin(X.ack + fi, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
+          }
+        } else {
+          ok = spin(X.ready + fi, [tag](uint64_t x) { return x >= tag; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
+          // the piece is read by TMA bulk loads (staged kernel) too: order them after the acquire
+          if (X.kind == 4 && !(A.flags & 8)) asm volatile("fence.proxy.async.global;" ::: "memory");
         }
-        s_stop = ok ? 0 : 2;
+        s_stop = !ok;
+        xtrace(A, op, j, pidx, 1);
       }
       __syncthreads();
       if (s_stop) return;
-      if (X.role == 0) cta_chunk<false>(X, sl, off, len, wt, sbuf, mbar);
-      else cta_chunk<true>(X, sl, off, len, wt, sbuf, mbar);
+      if (X.role == 0) cta_piece<false>(X, sl, off, len, wt, sbuf, mbar);
+      else cta_piece<true>(X, sl, off, len, wt, sbuf, mbar);
       __syncthreads();
       if (threadIdx.x == 0) {
-        // Publication: the CTA's stores (generic, and TMA bulk stores that thread 0 issued
-        // and waited for) precede this thread's system-scope release through the barrier
-        // above; the release is cumulative, so the peer's acquire of the counter sees them
-        // (the message-passing pattern NCCL's simple protocol uses: barrier, acq_rel fence
-        // at system scope, flag store).  The proxy fence orders the async-proxy writes with
-        // the generic release.  A full SC fence (bit 2 of DT_XFER_FLAGS) cost 20-25 % of
-        // the loopback exchange rate at 1-4 MiB fragments and is not needed for this pattern.
+        xtrace(A, op, j, pidx, 2);
+        // Publication (NCCL simple-protocol pattern): the CTA's stores precede thread 0's
+        // release through the barrier; the release is cumulative.  The proxy fence orders
+        // the TMA bulk stores (async proxy) that thread 0 issued and waited for.
         if (A.flags & 4) __threadfence_system();
-        if (X.kind == 4 && X.role == 0) asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA stores
-        red_release_sys_add(X.role == 0 ? X.ready + fi : X.ack + fi, (uint64_t)len);
-      }
-    }
-  }
-  // cumulative per-(sub-ring, slot) bytes after this message (read by the next
-  // message's kernel from the other parity); every sub-ring is carried over
-  for (int js = j; js < kMaxSub; js += X.ncta) {
-    for (int s = threadIdx.x; s < D; s += blockDim.x) {
-      uint64_t add = 0;
-      if (js < gs)
-        for (int64_t k = s; k < K; k += D) {
-          const int64_t off = k * C + (int64_t)js * Cs;
-          if (off < n) add += (uint64_t)min(Cs, n - off);
+        if (X.role == 0) {
+          if (X.kind == 4) asm volatile("fence.proxy.async.global;" ::: "memory");
+          st_release(X.ready + fi, tag, sys);
+        } else {
+          st_release(X.ack + fi, tag, sys);
         }
-      X.base_out[js * D + s] = X.base_in[js * D + s] + add;
+        xtrace(A, op, j, pidx, 3);
+      }
+      pidx++;
     }
+    slot += kstep;
+    while (slot >= D) { slot -= D; round++; }
   }
 }
 
@@ -385,11 +411,14 @@ struct HandleBlob {
   int32_t rank;
   int64_t pid;
   int32_t device;
-  int32_t pad;
+  int32_t mode;
+  int64_t chunk_bytes;  // the ring geometry every peer must share (checked at connect)
+  int32_t depth, nch;
+  uint8_t uuid[16];     // physical GPU (device ordinals differ between processes)
   uint64_t ring_ptr, flags_ptr;
   cudaIpcMemHandle_t ring_h, flags_h;
 };
-static const uint32_t kMagic = 0xD7A7C0DEu;
+static const uint32_t kMagic = 0xD7A7C0E2u;
 
 struct PendingOp {
   const void* sbuf;
@@ -408,11 +437,11 @@ struct dt_comm_s {
   int nch = kMaxCh;
   uint8_t* ring = nullptr;
   uint64_t* flags = nullptr;
-  uint64_t* bases = nullptr;  // [2 parities][2 dirs][nranks][nch][depth]
   size_t ring_bytes = 0, flag_words = 0;
   std::vector<uint8_t*> peer_ring;
   std::vector<uint64_t*> peer_flags;
   std::vector<bool> opened;
+  std::vector<int> same_dev;  // peer runs on this physical GPU: gpu-scope flags suffice
   bool connected = false;
   std::vector<uint64_t> send_seq, recv_seq;  // [nranks*nch]
   // group
@@ -426,21 +455,18 @@ struct dt_comm_s {
   uint8_t* rstage = nullptr; // recv staging
   int64_t* szbuf = nullptr;  // device size handshake buffers [2][kMaxOps]
   int64_t* szhost = nullptr; // pinned
-  // layout helpers (uint64 flag words): per (peer, channel) kMaxSub*depth ready
-  // counters, a 4-word header {seq, nbytes, sub-rings, replicas}, kMaxSub*depth ack
-  // counters and a go word; then one error word.  The ring of a (source,
-  // channel) pair is depth*chunk bytes, split among the sender's sub-rings.
+  // layout helpers (uint64 flag words): per (peer, channel) depth*kMaxSub ready tags,
+  // a 4-word header {seq, nbytes|abort, pieces, teams}, depth*kMaxSub ack tags and
+  // a 2-word go {capacity, seq}; then one error word.  The ring of a (source,
+  // channel) pair is depth*chunk bytes: D slots of one fragment each.
   size_t per() const { return (size_t)kMaxSub * o.depth; }
   size_t pairs() const { return (size_t)nranks * nch; }
   size_t ready_idx(int src, int ch) const { return ((size_t)src * nch + ch) * per(); }
   size_t hdr_idx(int src, int ch) const { return pairs() * per() + ((size_t)src * nch + ch) * 4; }
   size_t ack_idx(int dst, int ch) const { return pairs() * (per() + 4) + ((size_t)dst * nch + ch) * per(); }
-  size_t go_idx(int dst, int ch) const { return pairs() * (2 * per() + 4) + (size_t)dst * nch + ch; }
-  size_t err_idx() const { return pairs() * (2 * per() + 5); }
+  size_t go_idx(int dst, int ch) const { return pairs() * (2 * per() + 4) + ((size_t)dst * nch + ch) * 2; }
+  size_t err_idx() const { return pairs() * (2 * per() + 6); }
   size_t ring_off(int src, int ch) const { return (((size_t)src * nch + ch) * o.depth) * (size_t)o.chunk_bytes; }
-  uint64_t* base(int parity, int dir, int peer, int ch) const {
-    return bases + ((((size_t)parity * 2 + dir) * nranks + peer) * nch + ch) * per();
-  }
 };
 
 void dt::comm_info(dt_comm_t c, int* rank, int* nranks, int* device) {
@@ -470,7 +496,7 @@ static dt_status cufail(cudaError_t e, const char* what) {
 
 static void fill_opts(dt_xfer_opts& o, const dt_xfer_opts* in) {
   o.chunk_bytes = 1 << 20;
-  o.depth = 8;
+  o.depth = 0;
   o.mode = DT_XFER_P2P;
   o.ctas = 0;
   o.flags = in ? in->flags : 0;
@@ -481,6 +507,15 @@ static void fill_opts(dt_xfer_opts& o, const dt_xfer_opts* in) {
     o.ctas = in->ctas;
   }
   o.chunk_bytes = (o.chunk_bytes + 511) & ~int64_t(511);
+  if ((!in || in->depth <= 0) && o.mode == DT_XFER_NCCL) {
+    o.depth = 4;  // NCCL mode: depth = staging buffers of the pack/net/unpack overlap
+  } else if (!in || in->depth <= 0) {
+    // auto depth: a ring of >= 8 MiB per (pair, channel), at least 4 slots -- the
+    // in-flight bytes must cover link bandwidth x flag round trip (900 GB/s x ~5 us),
+    // so small fragments need many slots (64 KiB: 128)
+    int64_t d = ((int64_t)8 << 20) / o.chunk_bytes;
+    o.depth = (int)std::max<int64_t>(4, std::min<int64_t>(kMaxDepth, d));
+  }
 }
 
 extern "C" {
@@ -516,6 +551,11 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
     set_error("dt_comm_init: unknown mode");
     return DT_ERR_ARG;
   }
+  if (c->o.depth > kMaxDepth) {
+    delete c;
+    set_error("dt_comm_init: depth %d > %d", c->o.depth, kMaxDepth);
+    return DT_ERR_ARG;
+  }
   cudaError_t e = cudaSetDevice(device);
   if (e != cudaSuccess) {
     delete c;
@@ -527,13 +567,9 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
     e = cudaMalloc(&c->ring, c->ring_bytes);
     if (e == cudaSuccess) e = cudaMalloc(&c->flags, c->flag_words * 8);
     if (e == cudaSuccess) e = cudaMemset(c->flags, 0, c->flag_words * 8);
-    const size_t nb = (size_t)2 * 2 * c->pairs() * c->per();
-    if (e == cudaSuccess) e = cudaMalloc(&c->bases, nb * 8);
-    if (e == cudaSuccess) e = cudaMemset(c->bases, 0, nb * 8);
     if (e != cudaSuccess) {
       cudaFree(c->ring);
       cudaFree(c->flags);
-      cudaFree(c->bases);
       delete c;
       return cufail(e, "dt_comm_init alloc");
     }
@@ -574,6 +610,8 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
   c->peer_ring.assign(nranks, nullptr);
   c->peer_flags.assign(nranks, nullptr);
   c->opened.assign(nranks, false);
+  c->same_dev.assign(nranks, 0);
+  c->same_dev[rank] = !getenv("DT_XFER_SYS");  // DT_XFER_SYS: system-scope flags even on one GPU
   c->send_seq.assign((size_t)nranks * c->nch, 0);
   c->recv_seq.assign((size_t)nranks * c->nch, 0);
   c->peer_ring[rank] = c->ring;
@@ -600,6 +638,15 @@ dt_status dt_comm_local_handle(dt_comm_t c, void* out, size_t* nbytes) {
   b.rank = c->rank;
   b.pid = (int64_t)getpid();
   b.device = c->device;
+  b.mode = c->o.mode;
+  b.chunk_bytes = c->o.chunk_bytes;
+  b.depth = c->o.depth;
+  b.nch = c->nch;
+  {
+    cudaDeviceProp pr;
+    CU(cudaGetDeviceProperties(&pr, c->device));
+    std::memcpy(b.uuid, &pr.uuid, 16);
+  }
   b.ring_ptr = (uint64_t)(uintptr_t)c->ring;
   b.flags_ptr = (uint64_t)(uintptr_t)c->flags;
   if (c->o.mode == DT_XFER_P2P) {
@@ -629,7 +676,19 @@ dt_status dt_comm_connect(dt_comm_t c, const void* all, size_t per) {
       set_error("dt_comm_connect: malformed handle of rank %d", r);
       return DT_ERR_ARG;
     }
+    if (b.mode != c->o.mode || b.chunk_bytes != c->o.chunk_bytes || b.depth != c->o.depth || b.nch != c->nch) {
+      // the sender lays fragments out with its own C and D inside the receiver's ring
+      set_error("dt_comm_connect: rank %d uses chunk %lld / depth %d / mode %d, this rank chunk %lld / depth %d / "
+                "mode %d (must match)", r, (long long)b.chunk_bytes, b.depth, b.mode, (long long)c->o.chunk_bytes,
+                c->o.depth, c->o.mode);
+      return DT_ERR_ARG;
+    }
     if (r == c->rank) continue;
+    {
+      cudaDeviceProp pr;
+      CU(cudaGetDeviceProperties(&pr, c->device));
+      c->same_dev[r] = std::memcmp(b.uuid, &pr.uuid, 16) == 0 && !getenv("DT_XFER_SYS");
+    }
     if (b.pid == mypid) {  // same process (e.g. several devices driven by one process)
       c->peer_ring[r] = (uint8_t*)(uintptr_t)b.ring_ptr;
       c->peer_flags[r] = (uint64_t*)(uintptr_t)b.flags_ptr;
@@ -671,23 +730,26 @@ static int64_t lowp2u(uint64_t x) {
 }
 
 // Fill the pack/unpack params of one side of an op (no chunk-specific fields).
+// Contiguous instances are merged into one run first (effective(): count BYTEs, a
+// vector of adjacent blocks), so a piece of a contiguous message is one warp copy
+// per warp slice instead of a walk over count tiny instances.
 static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbytes, int64_t chunk, XOp& X) {
   DeviceDesc* dd = nullptr;
   dt_status st = ensure_committed_on_device(t, &dd);
   if (st != DT_OK) return st;
   const Form& f = get_form(t);
-  KLevels L;
-  build_levels(f, dd, t, count, L);
+  const Eff E = effective(f, dd, t, count);
+  const KLevels& L = E.L;
   KP& P = X.P;
   std::memset(&P, 0, sizeof(P));
   P.nc = (const uint8_t*)nc;
-  P.tsize = f.tsize();
-  P.nblocks = (int64_t)f.bl.size();
+  P.tsize = E.tsize;
+  P.nblocks = E.nblocks;
   P.bd = dd->bd;
   P.bl = dd->bl;
   P.boff = dd->boff;
-  P.bd0 = f.bd.empty() ? 0 : f.bd[0];
-  P.bl0 = f.bl.empty() ? 0 : f.bl[0];
+  P.bd0 = E.bd0;
+  P.bl0 = E.bl0;
   P.nlev = L.n;
   for (int i = 0; i < L.n; i++) {
     P.cnt[i] = L.cnt[i];
@@ -697,9 +759,9 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   }
   P.ftsize = make_fd((uint64_t)P.tsize);
   int64_t g = 1;
-  // chunk starts are multiples of `chunk` (a multiple of 512) and ring slots are aligned
-  int kind = plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
-  if (kind == 6) {  // record spans: fragments start on 512-byte stream boundaries (16-byte aligned)
+  // piece starts are multiples of C/gs (a multiple of 512) and ring slots are aligned
+  int kind = E.merged ? 1 : plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
+  if (kind == 6) {  // record spans: pieces start on 512-byte stream boundaries (16-byte aligned)
     if (!rec_geometry(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, g, &X.rg) || getenv("DT_XFER_NOREC"))
       kind = g >= 8 ? 4 : 2;
   }
@@ -722,16 +784,45 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
 }
 
 // shared memory of a record-span op in the transfer kernel: per-warp record buffers and
-// displacements, then the per-CTA map (layout as in cta_chunk / k_xfer)
+// displacements, then the per-CTA map (layout as in xc_rec / k_xfer)
 static size_t rec_smem_bytes(const RecGeo& R, int g) {
   const size_t nwc = kXferThreads / 32;
   const size_t tab = std::max<size_t>((size_t)R.RB * R.nwr * 2, (size_t)(R.spanB / g) * 2);
   return nwc * ((size_t)R.RB * R.spanB + (size_t)R.RB * 8) + tab;
 }
 
-// CTAs per direction (capped by co-residency across the group's ops); 64 measured best for
-// the loopback C3 exchange (738 vs 428 GB/s at 32, 16 MiB fragments)
-static int default_ctas(const dt_comm_s* c) { return c->o.ctas > 0 ? c->o.ctas : 64; }
+// CTA budget per direction (capped by co-residency across the group's ops)
+static int default_ctas(const dt_comm_s* c) {
+  if (c->o.ctas > 0) return c->o.ctas;
+  const char* e = getenv("DT_XFER_CTAS");
+  return e && atoi(e) > 0 ? atoi(e) : 64;
+}
+
+// Message geometry (gs pieces per fragment, rep teams): pieces of >= kPiece bytes
+// (a CTA moves a piece with one barrier + one flag; smaller pieces are all fixed
+// cost), as many pieces as the budget allows for large fragments, then teams that
+// take alternate fragments so several fragments are in flight at once (each team
+// owns D/rep slots).  Depends only on (n, C, D, budget).
+struct Geo {
+  int gs, rep;
+};
+static Geo geometry(int64_t n, int64_t C, int D, int budget) {
+  static const int64_t kPiece = getenv("DT_XFER_PIECE") ? atoll(getenv("DT_XFER_PIECE")) : (32 << 10);
+  const int64_t eff = std::min<int64_t>(C, std::max<int64_t>(512, (n + 511) & ~int64_t(511)));
+  int gs = 1;
+  while (gs * 2 <= kMaxSub && gs * 2 <= budget && C % ((int64_t)gs * 2 * 512) == 0 && eff / (gs * 2) >= kPiece)
+    gs *= 2;
+  const int64_t K = std::max<int64_t>(1, (n + C - 1) / C);
+  const char* rp = getenv("DT_XFER_REP");
+  int rep = 1;
+  if (rp) {
+    rep = std::max(1, atoi(rp));
+    while (rep > 1 && (D % rep || rep * gs > budget)) rep--;
+  } else {
+    while (rep * 2 <= D && D % (rep * 2) == 0 && rep * 2 * gs <= budget && rep * 2 <= K) rep *= 2;
+  }
+  return Geo{gs, rep};
+}
 
 static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cudaStream_t s) {
   XArgs A;
@@ -739,11 +830,10 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   const char* to = getenv("DT_TIMEOUT_MS");
   A.timeout_ns = (int64_t)(to ? atoll(to) : 30000) * 1000000ll;
   A.flags = getenv("DT_XFER_FLAGS") ? atoi(getenv("DT_XFER_FLAGS")) : 0;
-  int nops = 0, cta = 0;
+  int nops = 0;
   size_t smem = 0, rec_smem = 0;
   bool any_stage = false;
   std::vector<int> sch(c->nranks, 0), rch(c->nranks, 0);
-  const int G = default_ctas(c);
   for (const auto& p : ops) {
     if (p.dest >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
@@ -755,24 +845,14 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       if (st != DT_OK) return st;
       X.role = 0;
       X.n = n;
-      X.chunk = c->o.chunk_bytes;
-      X.depth = c->o.depth;
       uint64_t* pf = c->peer_flags[p.dest];
       X.ring = c->peer_ring[p.dest] + c->ring_off(c->rank, ch);
       X.ready = pf + c->ready_idx(c->rank, ch);
       X.hdr = pf + c->hdr_idx(c->rank, ch);
       X.ack = c->flags + c->ack_idx(p.dest, ch);
       X.go = c->flags + c->go_idx(p.dest, ch);
-      uint64_t& sq = c->send_seq[(size_t)p.dest * c->nch + ch];
-      const int par = (int)(sq & 1);
-      X.base_in = c->base(par, 0, p.dest, ch);
-      X.base_out = c->base(par ^ 1, 0, p.dest, ch);
-      X.seq = ++sq;
-      X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
-      if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
-      any_stage = any_stage || X.kind == 4;
-      if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
-      if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)(kXferThreads / 32) * kSpanWarpSmem);
+      X.seq = ++c->send_seq[(size_t)p.dest * c->nch + ch];
+      X.sys = !c->same_dev[p.dest];
     }
     if (p.source >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
@@ -784,67 +864,84 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       if (st != DT_OK) return st;
       X.role = 1;
       X.n = cap;
-      X.chunk = c->o.chunk_bytes;
-      X.depth = c->o.depth;
       uint64_t* pf = c->peer_flags[p.source];
       X.ring = c->ring + c->ring_off(p.source, ch);
       X.ready = c->flags + c->ready_idx(p.source, ch);
       X.hdr = c->flags + c->hdr_idx(p.source, ch);
       X.ack = pf + c->ack_idx(c->rank, ch);
       X.go = pf + c->go_idx(c->rank, ch);
-      uint64_t& sq = c->recv_seq[(size_t)p.source * c->nch + ch];
-      const int par = (int)(sq & 1);
-      X.base_in = c->base(par, 1, p.source, ch);
-      X.base_out = c->base(par ^ 1, 1, p.source, ch);
-      X.seq = ++sq;
-      X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
-      if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
-      any_stage = any_stage || X.kind == 4;
-      if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
-      if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)(kXferThreads / 32) * kSpanWarpSmem);
+      X.seq = ++c->recv_seq[(size_t)p.source * c->nch + ch];
+      X.sys = !c->same_dev[p.source];
     }
   }
   if (nops == 0) return DT_OK;
+  for (int i = 0; i < nops; i++) {
+    XOp& X = A.ops[i];
+    X.chunk = c->o.chunk_bytes;
+    X.depth = c->o.depth;
+    X.err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
+    if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
+    any_stage = any_stage || X.kind == 4;
+    if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
+    if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)(kXferThreads / 32) * kSpanWarpSmem);
+  }
   A.nops = nops;
   A.wt_off = (int32_t)std::max<size_t>(any_stage ? (size_t)kXferStageBufs * kStageTile : 0, (rec_smem + 127) & ~size_t(127));
   smem += (size_t)A.wt_off;
+  // the attribute is per device (a process may drive several)
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  // every CTA must be co-resident: fit the per-op CTA count to the occupancy
+  // every CTA must be co-resident: fit the per-op CTA budget to the occupancy
   int occ = 0;
   CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_xfer, kXferThreads, smem));
   int sms = 0, dev = 0;
   CU(cudaGetDevice(&dev));
   CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-  const int per_op = std::max(1, std::min(G, occ * sms / nops));
+  const int budget = std::max(1, std::min(default_ctas(c), occ * sms / nops));
+  int cta = 0;
   for (int i = 0; i < nops; i++) {
-    int n_i = per_op;
-    if (A.ops[i].role == 0) {  // rep CTAs per sub-ring; a sub-ring slot is C/gs bytes, a multiple of 512
-      const int64_t C = A.ops[i].chunk;
-      // replicas: each slot must belong to one replica, and each replica keeps >= 2 slots
-      // (with one slot a replica waits a full round trip per fragment: C3 4 MiB, depth 2:
-      // 441 -> 306 GB/s; depth 4 with 2 replicas: 436 -> 487, 1 MiB: 192 -> 296)
-      // default: the most replicas (<= 4) that still leave each >= 2 slots (depth 8: 4
-      // replicas, C3 1 MiB 415 GB/s; depth 4: 2 replicas, 300 GB/s)
-      const char* rp = getenv("DT_XFER_REP");
-      const int dep = A.ops[i].depth;
-      int rep = rp ? std::max(1, atoi(rp)) : 4;
-      if (!rp) {
-        const int64_t K = (A.ops[i].n + C - 1) / C;  // fragments: replicas beyond K would idle
-        while (rep > 1 && (dep % rep != 0 || dep / rep < 2 || rep > K)) rep /= 2;
-      }
-      if (dep % rep != 0 || dep / rep < 2 || per_op < rep) rep = 1;
-      int g = 1;
-      while (g * 2 * rep <= per_op && g * 2 <= kMaxSub && C % ((int64_t)g * 2 * 512) == 0) g *= 2;
-      n_i = g * rep;
-      A.ops[i].rep = rep;
-    }
-    A.ops[i].cta0 = cta;
-    A.ops[i].ncta = n_i;
-    cta += n_i;
+    XOp& X = A.ops[i];
+    // send role: one CTA per (team, piece); receive role: as many as the capacity
+    // would need (the actual geometry arrives in the header; CTAs map onto it)
+    const Geo G = geometry(X.n, X.chunk, X.depth, budget);
+    X.gs = G.gs;
+    X.rep = G.rep;
+    X.cta0 = cta;
+    X.ncta = G.gs * G.rep;
+    cta += X.ncta;
+  }
+  if (getenv("DT_XFER_DEBUG"))
+    for (int i = 0; i < nops; i++)
+      fprintf(stderr, "[dt_xfer] op %d role %d kind %d g %d n %lld C %lld D %d gs %d rep %d ncta %d budget %d\n", i,
+              A.ops[i].role, A.ops[i].kind, A.ops[i].g, (long long)A.ops[i].n, (long long)A.ops[i].chunk,
+              A.ops[i].depth, A.ops[i].gs, A.ops[i].rep, A.ops[i].ncta, budget);
+  static uint64_t* trace = nullptr;
+  const char* tr = getenv("DT_XFER_TRACE");  // diagnostics: dump per-piece timestamps to this file
+  const size_t tn = (size_t)kMaxOps * kTraceCtas * kTracePieces * 4;
+  if (tr) {
+    if (!trace) CU(cudaMalloc(&trace, tn * 8));
+    CU(cudaMemsetAsync(trace, 0, tn * 8, s));
+    A.trace = trace;
   }
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
   CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
+  if (tr) {
+    std::vector<uint64_t> h(tn);
+    CU(cudaMemcpyAsync(h.data(), trace, tn * 8, cudaMemcpyDeviceToHost, s));
+    CU(cudaStreamSynchronize(s));
+    if (FILE* fp = fopen(tr, "a")) {
+      fprintf(fp, "# launch nops %d\n", nops);
+      for (int i = 0; i < nops; i++)
+        for (int jj = 0; jj < kTraceCtas; jj++)
+          for (int p = 0; p < kTracePieces; p++) {
+            const uint64_t* q = &h[(((size_t)i * kTraceCtas + jj) * kTracePieces + p) * 4];
+            if (q[0]) fprintf(fp, "%d %d %d %d %llu %llu %llu %llu\n", i, A.ops[i].role, jj, p,
+                              (unsigned long long)q[0], (unsigned long long)q[1], (unsigned long long)q[2],
+                              (unsigned long long)q[3]);
+          }
+      fclose(fp);
+    }
+  }
   return DT_OK;
 }
 
@@ -1066,7 +1163,6 @@ dt_status dt_comm_free(dt_comm_t* pc) {
   }
   cudaFree(c->ring);
   cudaFree(c->flags);
-  cudaFree(c->bases);
   cudaFree(c->stage);
   cudaFree(c->rstage);
   cudaFree(c->szbuf);

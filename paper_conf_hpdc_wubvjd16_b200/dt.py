@@ -365,7 +365,7 @@ def broadcast_id(idbytes, group=None) -> bytes:
 class Comm:
     """dt_comm_t: this rank's endpoint (receive rings + flags, or a NCCL communicator)."""
 
-    def __init__(self, rank: int, nranks: int, device: int, chunk_bytes: int = 1 << 20, depth: int = 8,
+    def __init__(self, rank: int, nranks: int, device: int, chunk_bytes: int = 1 << 20, depth: int = 0,
                  mode: int = XFER_P2P, ctas: int = 0, nccl_id: bytes | None = None, ring_loopback: bool = False):
         # ring_loopback: send-to-self goes through the ring pipeline instead of the fused dt_copy
         self.opts = XferOpts(chunk_bytes, depth, mode, ctas, 1 if ring_loopback else 0)

@@ -16,7 +16,8 @@ def main():
     src = torch.empty(64 << 20, dtype=torch.uint8, device="cuda").random_(0, 255)
     dst = torch.zeros_like(src)
     s = torch.cuda.current_stream()
-    for chunk, depth in [(1 << 20, 2), (1 << 20, 8), (4 << 20, 2), (256 << 10, 4)]:
+    cfgs = os.environ.get("PROBE_CFGS", "1024:2,1024:0,4096:2,256:4,64:0")
+    for chunk, depth in [(int(a) << 10, int(b)) for a, b in (x.split(":") for x in cfgs.split(","))]:
         comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth, ring_loopback=True,
                        ctas=int(os.environ.get("PROBE_CTAS", 0)))
         row = {}
@@ -32,7 +33,8 @@ def main():
             comm.check()
             assert torch.equal(dst[:n], src[:n])
             row[f"{n >> 10}K"] = round(e0.elapsed_time(e1) / 10 * 1e3, 1)
-        print(f"unit={unit} ctas={os.environ.get('PROBE_CTAS', 0)} chunk={chunk >> 10}K depth={depth}", row, flush=True)
+        print(f"unit={unit} ctas={os.environ.get('PROBE_CTAS', 0)} chunk={chunk >> 10}K depth={depth or 'auto'}", row,
+              flush=True)
         comm.free()
 
 
