@@ -183,8 +183,8 @@ __global__ void __launch_bounds__(256) k_stage(const KP P, int64_t ntiles) {
   const int64_t lo = P.pos + t0 * kStageTile;
   const int64_t hi = P.pos + t1 * kStageTile < end ? P.pos + t1 * kStageTile : end;
   if (lo >= hi) return;
-  if (UNPACK) stage_unpack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf, mbar);
-  else stage_pack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf);
+  if (UNPACK) stage_unpack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf, mbar, threadIdx.x, blockDim.x);
+  else stage_pack<G, kStageBufs>(P, P.c - P.pos, wt, lo, hi, sbuf, threadIdx.x, blockDim.x);
 }
 
 // f1: fused type -> type copies (no packed buffer)

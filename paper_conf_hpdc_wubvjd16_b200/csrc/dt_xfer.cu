@@ -42,6 +42,13 @@ constexpr int kMaxOps = 16;
 constexpr int kMaxCh = 6;    // concurrent messages per (pair, direction) inside one group
 constexpr int kMaxSub = 64;  // pieces (sub-rings) per fragment
 constexpr int kMaxDepth = 256;  // ring slots per (pair, channel)
+// CTA layout: warp 0 = control warp; then kGroups copy groups of kGroupWarps warps.
+// Piece i of a CTA goes to group i % 2, so two pieces are copied concurrently and a
+// piece's fixed latencies (TMA completion, barriers) overlap the other's copy.
+constexpr int kGroups = 2, kGroupWarps = 8;
+constexpr int kCopyWarps = kGroups * kGroupWarps;
+constexpr int kGroupThreads = kGroupWarps * 32;
+constexpr int kXferThreads = 32 + kCopyWarps * 32;
 constexpr uint64_t kAbort = 1ull << 63;
 
 // Flag values are tags: (message sequence number << 32) | (round + 1).  They only
@@ -81,10 +88,12 @@ struct XArgs {
   uint64_t* trace;  // diagnostics (DT_XFER_TRACE): per-piece globaltimer stamps of the first CTAs
   XOp ops[kMaxOps];
 };
-constexpr int kTraceCtas = 4, kTracePieces = 64;
+constexpr int kTraceCtas = 4, kTracePieces = 64, kTracePts = 6;
+// points: 0 control starts waiting for the piece's flag, 1 flag acquired, 2 copy seen
+// done, 3 flag released, 4 copy group starts the piece, 5 copy group done
 __device__ __forceinline__ void xtrace(const XArgs& A, int op, int j, int idx, int point) {
   if (A.trace && j < kTraceCtas && idx < kTracePieces)
-    A.trace[(((size_t)op * kTraceCtas + j) * kTracePieces + idx) * 4 + point] = gtimer();
+    *(volatile uint64_t*)&A.trace[(((size_t)op * kTraceCtas + j) * kTracePieces + idx) * kTracePts + point] = gtimer();
 }
 
 // ---- per-family piece copies.  Each is a separate (noinline) function so that
@@ -97,7 +106,8 @@ __device__ __noinline__ void xc_seg(const XOp& X, uint8_t* cb, int64_t a, int64_
 }
 
 template <bool UNPACK, int G>
-__device__ __noinline__ void xc_rec(const XOp& X, uint8_t* cb, int64_t lo, int64_t hb, uint8_t* sbuf) {
+__device__ __noinline__ void xc_rec(const XOp& X, uint8_t* cb, int64_t lo, int64_t hb, uint8_t* sbuf, int w,
+                                    int nwc, int cw) {
   constexpr int POL = UNPACK ? LD_CG : LD_CS;
   const KP& P = X.P;
   RecGeo R = X.rg;
@@ -105,10 +115,12 @@ __device__ __noinline__ void xc_rec(const XOp& X, uint8_t* cb, int64_t lo, int64
   R.e_hi = (hb + P.tsize - 1) / P.tsize;
   R.b0 = R.e_lo & ~int64_t(31);
   R.nbatch = (R.e_hi - R.b0 + R.RB - 1) / R.RB;
-  const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint8_t* buf = sbuf + w * (R.RB * R.spanB);
-  int64_t* sd = reinterpret_cast<int64_t*>(sbuf + nwc * (R.RB * R.spanB)) + w * R.RB;
-  uint16_t* omap = reinterpret_cast<uint16_t*>(sbuf + nwc * (R.RB * R.spanB) + nwc * R.RB * 8);
+  // per-copy-warp buffers (cw: the warp's index among all copy warps, layout as set up in
+  // k_xfer); the work is split over the nwc warps of the group (w: index in the group)
+  const int lane = threadIdx.x & 31;
+  uint8_t* buf = sbuf + cw * (R.RB * R.spanB);
+  int64_t* sd = reinterpret_cast<int64_t*>(sbuf + kCopyWarps * (R.RB * R.spanB)) + cw * R.RB;
+  uint16_t* omap = reinterpret_cast<uint16_t*>(sbuf + kCopyWarps * (R.RB * R.spanB) + kCopyWarps * R.RB * 8);
   rec_range<UNPACK, G, POL>(P, R, cb, lo, hb, buf, sd, omap, w, nwc, lane);
 }
 
@@ -121,44 +133,50 @@ __device__ __noinline__ void xc_span(const XOp& X, uint8_t* cb, int64_t a, int64
 
 template <bool UNPACK, int G>
 __device__ __noinline__ void xc_stage(const XOp& X, uint8_t* cb, const int32_t* wt, int64_t lo, int64_t bh,
-                                      uint8_t* sbuf, uint64_t* mbar) {
-  if (UNPACK) stage_unpack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf, mbar);
-  else stage_pack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf);
+                                      uint8_t* sbuf, uint64_t* mbar, int ctid, int cnthr, int bar, int64_t tb) {
+  if (UNPACK) stage_unpack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf, mbar, ctid, cnthr, bar, tb);
+  else stage_pack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf, ctid, cnthr, bar);
 }
 
 template <bool UNPACK, int G>
-__device__ __noinline__ void xc_word(const XOp& X, uint8_t* cb, int64_t lo, int64_t hi, const int32_t* wt) {
+__device__ __noinline__ void xc_word(const XOp& X, uint8_t* cb, int64_t lo, int64_t hi, const int32_t* wt, int ctid,
+                                     int cnthr) {
   constexpr int POL = UNPACK ? LD_CG : LD_CS;
-  // few CTAs carry the whole transfer: keep 4 vectors per thread in flight (512 threads: 32 KiB/CTA)
-  word_range<UNPACK, G, 16, POL, (G >= 4 ? 4 : 2)>(X.P, cb, lo, hi, wt, threadIdx.x, blockDim.x);
+  // few CTAs carry the whole transfer: keep 4 vectors per thread in flight (480 threads: 30 KiB/CTA)
+  word_range<UNPACK, G, 16, POL, (G >= 4 ? 4 : 2)>(X.P, cb, lo, hi, wt, ctid, cnthr);
 }
 
-// pack or unpack stream bytes [lo, lo+len) of one piece with this CTA.
-// cb: the slot base such that stream byte x of the message lives at cb + x.
+// pack or unpack stream bytes [lo, lo+len) of one piece with copy group g (warps
+// 1 + 8g .. 8 + 8g of the CTA; warp 0 is the control warp).  cb: the slot base such
+// that stream byte x of the message lives at cb + x.  sbuf: the CTA's dynamic smem
+// (per-warp buffers of kinds 6/7, or this group's staging tiles for kind 4); mbar:
+// this group's TMA mbarriers.
 template <bool UNPACK>
 __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo, int64_t len, const int32_t* wt,
-                                          uint8_t* sbuf, uint64_t* mbar) {
+                                          uint8_t* sbuf, uint64_t* mbar, int g, int64_t& tb) {
   const int64_t hi = lo + len;
-  const int nwc = blockDim.x >> 5, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (X.kind == 6) {  // record spans: the CTA's warps take RB-record batches of the piece
+  const int cw = (threadIdx.x >> 5) - 1;  // copy warp index among all copy warps
+  const int nwc = kGroupWarps, w = cw - g * kGroupWarps, lane = threadIdx.x & 31;
+  const int ctid = threadIdx.x - 32 - g * kGroupThreads, cnthr = kGroupThreads, bar = 1 + g;
+  if (X.kind == 6) {  // record spans: the copy warps take RB-record batches of the piece
     const int64_t hb = hi - len % X.g;  // a ragged tail (< G bytes, last piece) is walked below
     if (lo < hb) {
       switch (X.g) {
-        case 4: xc_rec<UNPACK, 4>(X, cb, lo, hb, sbuf); break;
-        case 8: xc_rec<UNPACK, 8>(X, cb, lo, hb, sbuf); break;
-        default: xc_rec<UNPACK, 16>(X, cb, lo, hb, sbuf); break;
+        case 4: xc_rec<UNPACK, 4>(X, cb, lo, hb, sbuf, w, nwc, cw); break;
+        case 8: xc_rec<UNPACK, 8>(X, cb, lo, hb, sbuf, w, nwc, cw); break;
+        default: xc_rec<UNPACK, 16>(X, cb, lo, hb, sbuf, w, nwc, cw); break;
       }
     }
     if (hb < hi && w == nwc - 1) xc_seg<UNPACK, false>(X, cb, hb, hi, lane);
     return;
   }
-  if (X.kind == 7) {  // block spans: the CTA's warps take equal 16-byte-multiple slices of the piece
+  if (X.kind == 7) {  // block spans: the copy warps take equal 16-byte-multiple slices of the piece
     const int64_t body = len - len % X.g;
     int64_t per = (body + nwc - 1) / nwc;
     per = (per + 15) & ~int64_t(15);
     const int64_t a = lo + (int64_t)w * per, b = min(a + per, lo + body);
     if (a < b) {
-      uint8_t* sm = sbuf + (size_t)w * kSpanWarpSmem;
+      uint8_t* sm = sbuf + (size_t)cw * kSpanWarpSmem;
       switch (X.g) {
         case 4: xc_span<UNPACK, 4>(X, cb, a, b, sm, lane); break;
         case 8: xc_span<UNPACK, 8>(X, cb, a, b, sm, lane); break;
@@ -170,24 +188,28 @@ __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo,
   }
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
     const int64_t bh = hi - len % X.g;
-    if (X.g == 8) xc_stage<UNPACK, 8>(X, cb, wt, lo, bh, sbuf, mbar);
-    else xc_stage<UNPACK, 16>(X, cb, wt, lo, bh, sbuf, mbar);
+    uint8_t* gbuf = sbuf + (size_t)g * kXferStageBufs * kStageTile;
+    if (X.g == 8) xc_stage<UNPACK, 8>(X, cb, wt, lo, bh, gbuf, mbar, ctid, cnthr, bar, tb);
+    else xc_stage<UNPACK, 16>(X, cb, wt, lo, bh, gbuf, mbar, ctid, cnthr, bar, tb);
+    tb += (bh - lo + kStageTile - 1) / kStageTile;  // tiles through this group's mbarriers
     if (bh < hi) {
-      __syncthreads();
-      if (threadIdx.x < 32) xc_seg<UNPACK, false>(X, cb, bh, hi, lane);
+      group_sync(bar, cnthr);
+      if (w == 0) xc_seg<UNPACK, false>(X, cb, bh, hi, lane);
     }
+    // the TMA bulk stores (async proxy) of the piece precede the control warp's release
+    if (!UNPACK && ctid == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
     return;
   }
   if (X.kind == 2) {
     const int64_t body = len - len % X.g;
     switch (X.g) {
-      case 1: xc_word<UNPACK, 1>(X, cb, lo, lo + body, wt); break;
-      case 2: xc_word<UNPACK, 2>(X, cb, lo, lo + body, wt); break;
-      case 4: xc_word<UNPACK, 4>(X, cb, lo, lo + body, wt); break;
-      case 8: xc_word<UNPACK, 8>(X, cb, lo, lo + body, wt); break;
-      default: xc_word<UNPACK, 16>(X, cb, lo, lo + body, wt); break;
+      case 1: xc_word<UNPACK, 1>(X, cb, lo, lo + body, wt, ctid, cnthr); break;
+      case 2: xc_word<UNPACK, 2>(X, cb, lo, lo + body, wt, ctid, cnthr); break;
+      case 4: xc_word<UNPACK, 4>(X, cb, lo, lo + body, wt, ctid, cnthr); break;
+      case 8: xc_word<UNPACK, 8>(X, cb, lo, lo + body, wt, ctid, cnthr); break;
+      default: xc_word<UNPACK, 16>(X, cb, lo, lo + body, wt, ctid, cnthr); break;
     }
-    if (body < len && threadIdx.x < 32) xc_seg<UNPACK, false>(X, cb, lo + body, hi, lane);
+    if (body < len && w == 0) xc_seg<UNPACK, false>(X, cb, lo + body, hi, lane);
     return;
   }
   int64_t per = (len + nwc - 1) / nwc;
@@ -198,6 +220,52 @@ __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo,
     else xc_seg<UNPACK, false>(X, cb, a, b, lane);
   }
 }
+
+// The pieces one CTA handles, in fragment order (32-bit index math, slot and round
+// kept incrementally).  Send role: CTA j = (team j / gs, piece j % gs), fragments
+// j/gs, j/gs + rep, ...  Receive role: pairs j, j + ncta, ... (one pair per CTA
+// when ncta >= pairs).  The control warp and the copy warps walk the same sequence.
+struct PieceIt {
+  int64_t n, C, Cs;
+  int K, D, gs, rep, ncta, j, jstep, kstep, k, js, slot, round;
+  bool one;
+  __device__ __forceinline__ bool init(int role, int64_t n_, int64_t C_, int D_, int gs_, int rep_, int ncta_, int j_) {
+    n = n_; C = C_; D = D_; gs = gs_; rep = rep_; ncta = ncta_; j = j_;
+    Cs = C / gs;
+    K = (int)((n + C - 1) / C);
+    const int npairs = gs * rep;
+    one = role == 0 || ncta >= npairs;
+    if (one && j >= npairs) return false;
+    kstep = one ? rep : 1;
+    jstep = one ? gs : ncta;
+    k = one ? j / gs : 0;
+    slot = k % D;
+    round = k / D;
+    js = first_js();
+    return settle();
+  }
+  __device__ __forceinline__ int first_js() const {
+    return one ? j % gs : (((j - (k % rep) * gs) % ncta) + ncta) % ncta;
+  }
+  // advance to a valid (k, js) at or after the current one; false at the end
+  __device__ __forceinline__ bool settle() {
+    while (k < K) {
+      if (js < gs && (int64_t)k * C + (int64_t)js * Cs < n) return true;
+      k += kstep;
+      slot += kstep;
+      while (slot >= D) { slot -= D; round++; }
+      if (k < K) js = first_js();
+    }
+    return false;
+  }
+  __device__ __forceinline__ bool next() {
+    js += jstep;
+    return settle();
+  }
+  __device__ __forceinline__ int64_t off() const { return (int64_t)k * C + (int64_t)js * Cs; }
+  __device__ __forceinline__ int64_t len() const { return min(Cs, n - off()); }
+  __device__ __forceinline__ int fi() const { return slot * kMaxSub + js; }
+};
 
 // One persistent kernel per dt_sendrecv / dt_group: send-role and receive-role CTAs
 // of every op (co-resident: cooperative launch).
@@ -220,11 +288,10 @@ __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo,
 //    ack[slot][js] ([L20:c4133]).
 // Flags are written by exactly one CTA, so plain release stores suffice, and since
 // tags only grow nothing is carried between messages.
-constexpr int kXferThreads = 512;
 __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
   // dynamic smem: [staging buffers / record or span buffers] [word table]
   extern __shared__ __align__(128) uint8_t xsm[];
-  __shared__ uint64_t mbar[kXferStageBufs];
+  __shared__ __align__(8) uint64_t mbar[kGroups][kXferStageBufs];
   uint8_t* sbuf = xsm;
   int32_t* wt = reinterpret_cast<int32_t*>(xsm + A.wt_off);
   __shared__ uint64_t s_n;
@@ -235,6 +302,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   const XOp& X = A.ops[op];
   const int j = (int)blockIdx.x - X.cta0;
   const bool sleep_ok = !(A.flags & 2);
+  if (threadIdx.x == 0) xtrace(A, op, j, kTracePieces - 1, 0);  // (diagnostics: kernel entry)
 
   // the receiver's "start packing" goes out first: it is on the sender's critical path
   if (X.role == 1 && j == 0 && threadIdx.x == 0) {
@@ -245,7 +313,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
     for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
   if (X.kind == 6) {  // record-span maps after the per-warp buffers (same layout as xc_rec)
     const RecGeo& R = X.rg;
-    uint16_t* omap = reinterpret_cast<uint16_t*>(xsm + (blockDim.x >> 5) * (R.RB * R.spanB + R.RB * 8));
+    uint16_t* omap = reinterpret_cast<uint16_t*>(xsm + kCopyWarps * (R.RB * R.spanB + R.RB * 8));
     if (X.role == 1) {
       switch (X.g) { case 4: rec_maps<true, 4>(R, omap); break; case 8: rec_maps<true, 8>(R, omap); break;
                      default: rec_maps<true, 16>(R, omap); break; }
@@ -257,6 +325,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   const uint64_t seq = X.seq;
   const bool sys = X.sys != 0;
   if (threadIdx.x == 0) {
+    xtrace(A, op, j, kTracePieces - 1, 1);  // setup done
     uint64_t v = 0;
     s_stop = 0;
     if (X.role == 0) {
@@ -287,73 +356,109 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   __syncthreads();
   if (s_stop) return;
   const int64_t n = (int64_t)s_n;
-  const int gs = s_gs, rep = s_rep;
-  const int64_t C = X.chunk;
-  const int D = X.depth;
-  const int64_t Cs = C / gs;
-  const int K = (int)((n + C - 1) / C);
-  const int npairs = gs * rep;
-  // Pieces of this CTA, in fragment order (32-bit index math, slot/round kept
-  // incrementally: the loop runs between every two pieces, it must cost nothing).
-  // Send role: CTA j = (team j / gs, piece j % gs), fragments j/gs, j/gs + rep, ...
-  // Receive role: pairs j, j + ncta, ... (one pair per CTA when ncta >= pairs).
-  const bool one = X.role == 0 || X.ncta >= npairs;
-  if (one && j >= npairs) return;
-  const int kstep = one ? rep : 1;
-  int k = one ? j / gs : 0;
-  int slot = k % D, round = k / D;
-  int pidx = 0;
-  for (; k < K; k += kstep) {
-    const int team = one ? 0 : k % rep;
-    int js = one ? j % gs : (((j - team * gs) % X.ncta) + X.ncta) % X.ncta;
-    const int jstep = one ? gs : X.ncta;
-    for (; js < gs; js += jstep) {
-      const int64_t off = (int64_t)k * C + (int64_t)js * Cs;
-      if (off >= n) break;
-      const int64_t len = min(Cs, n - off);
-      const int fi = slot * kMaxSub + js;
-      const uint64_t tag = xtag(seq, round);
-      uint8_t* sl = X.ring + (int64_t)slot * C + (int64_t)js * Cs - off;  // stream byte off -> piece start
-      if (threadIdx.x == 0) {
-        uint64_t v;
-        bool ok = true;
-        xtrace(A, op, j, pidx, 0);
-        if (X.role == 0) {
-          if (round > 0) {
-            const uint64_t need = xtag(seq, round - 1);
-            ok = spin(X.ack + fi, [need](uint64_t x) { return x >= need; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
-          }
-        } else {
-          ok = spin(X.ready + fi, [tag](uint64_t x) { return x >= tag; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
-          // the piece is read by TMA bulk loads (staged kernel) too: order them after the acquire
-          if (X.kind == 4 && !(A.flags & 8)) asm volatile("fence.proxy.async.global;" ::: "memory");
-        }
-        s_stop = !ok;
-        xtrace(A, op, j, pidx, 1);
-      }
-      __syncthreads();
-      if (s_stop) return;
-      if (X.role == 0) cta_piece<false>(X, sl, off, len, wt, sbuf, mbar);
-      else cta_piece<true>(X, sl, off, len, wt, sbuf, mbar);
-      __syncthreads();
-      if (threadIdx.x == 0) {
-        xtrace(A, op, j, pidx, 2);
-        // Publication (NCCL simple-protocol pattern): the CTA's stores precede thread 0's
-        // release through the barrier; the release is cumulative.  The proxy fence orders
-        // the TMA bulk stores (async proxy) that thread 0 issued and waited for.
+  // Warp specialisation: warp 0 (lane 0) is the control warp -- it waits for each
+  // piece's flag, hands the piece to the copy warps through full[b], waits for the
+  // copy through empty[b] and publishes it -- so the flag latency and the release
+  // (a system-scope release waits for every store of the piece to be acknowledged,
+  // ~4 us over the system fabric) overlap the copy of the next piece.  Two pieces
+  // in flight per CTA (b = piece index % 2).
+  __shared__ __align__(8) uint64_t full[2], empty[2];
+  __shared__ int s_abort;
+  if (threadIdx.x == 0) {
+    mbar_init(full + 0, 1);
+    mbar_init(full + 1, 1);
+    mbar_init(empty + 0, kGroupThreads);
+    mbar_init(empty + 1, kGroupThreads);
+    for (int g = 0; g < kGroups; g++)  // the staged unpack's TMA barriers: initialised once per kernel
+      for (int b = 0; b < kXferStageBufs; b++) mbar_init(&mbar[g][b], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    s_abort = 0;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) xtrace(A, op, j, kTracePieces - 1, 2);  // handshake done
+  PieceIt it;
+  bool more = it.init(X.role, n, X.chunk, X.depth, s_gs, s_rep, X.ncta, j);
+  if (threadIdx.x < 32) {  // ---- control warp
+    if (threadIdx.x != 0) return;
+    // Event loop over two conditions, never blocking on one while the other could
+    // progress (a receiver must publish piece i-1 before it can get piece i when the
+    // sender has one slot per lane): release the oldest acquired piece once copied;
+    // acquire the next piece when its flag is set (at most 2 pieces outstanding).
+    int i_acq = 0, i_rel = 0;
+    int q_fi[2] = {0, 0};
+    uint64_t q_tag[2] = {0, 0};
+    uint64_t t_idle = 0;
+    int ns = 0;
+    while (more || i_rel < i_acq) {
+      bool progress = false;
+      if (i_rel < i_acq && mbar_test(empty + (i_rel & 1), (uint32_t)((i_rel >> 1) & 1))) {
+        xtrace(A, op, j, i_rel, 2);
         if (A.flags & 4) __threadfence_system();
-        if (X.role == 0) {
-          if (X.kind == 4) asm volatile("fence.proxy.async.global;" ::: "memory");
-          st_release(X.ready + fi, tag, sys);
-        } else {
-          st_release(X.ack + fi, tag, sys);
-        }
-        xtrace(A, op, j, pidx, 3);
+        const int b = i_rel & 1;
+        st_release(X.role == 0 ? X.ready + q_fi[b] : X.ack + q_fi[b], q_tag[b], sys);
+        xtrace(A, op, j, i_rel, 3);
+        i_rel++;
+        progress = true;
       }
-      pidx++;
+      if (more && i_acq - i_rel < ((A.flags & 16) ? 1 : 2)) {
+        const int fi = it.fi();
+        const uint64_t tag = xtag(seq, it.round);
+        bool ok;
+        if (i_acq == 0 || ns == 0) xtrace(A, op, j, i_acq, 0);
+        if (X.role == 0) ok = it.round == 0 || ld_acquire(X.ack + fi, sys) >= xtag(seq, it.round - 1);
+        else ok = ld_acquire(X.ready + fi, sys) >= tag;
+        if (ok) {
+          xtrace(A, op, j, i_acq, 1);
+          const int b = i_acq & 1;
+          q_fi[b] = fi;
+          q_tag[b] = tag;
+          mbar_arrive(full + b);  // piece i_acq may be copied (the arrive releases the acquire)
+          i_acq++;
+          more = it.next();
+          progress = true;
+        }
+      }
+      if (progress) {
+        t_idle = 0;
+        ns = 0;
+        continue;
+      }
+      if (sleep_ok) __nanosleep(ns);
+      ns = ns < 32 ? 32 : (ns < 256 ? 2 * ns : 256);
+      const uint64_t now = gtimer();
+      if (!t_idle) t_idle = now;
+      else if ((int64_t)(now - t_idle) > A.timeout_ns) {
+        atomicCAS(X.err, 0, XERR_TIMEOUT);
+        s_abort = 1;
+        __threadfence_block();
+        // wake both copy groups (each waits on its own barrier); they see s_abort and leave.
+        // A group still copying its piece leaves at its next wait: that phase completes by
+        // these arrivals or by the one below.
+        mbar_arrive(full + 0);
+        mbar_arrive(full + 1);
+        return;
+      }
     }
-    slot += kstep;
-    while (slot >= D) { slot -= D; round++; }
+    xtrace(A, op, j, kTracePieces - 1, 3);  // control loop done
+    return;
+  }
+  // ---- copy groups: group g takes the CTA's pieces g, g + 2, g + 4, ...
+  const int g = (threadIdx.x - 32) / kGroupThreads;
+  int64_t tb = 0;  // tiles this group has moved through its TMA barriers (staged unpack)
+  if (more && g == 1) more = it.next();
+  for (int i = g; more; i += 2) {
+    mbar_wait(full + g, (uint32_t)((i >> 1) & 1));
+    if (s_abort) return;
+    const int64_t off = it.off();
+    uint8_t* sl = X.ring + (int64_t)it.slot * X.chunk + (int64_t)it.js * it.Cs - off;  // stream byte off -> piece
+    if (X.role == 1 && X.kind == 4 && !(A.flags & 8))  // TMA bulk loads of the ring after the acquire
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+    if (threadIdx.x == 32 + g * kGroupThreads) xtrace(A, op, j, i, 4);
+    if (X.role == 0) cta_piece<false>(X, sl, off, it.len(), wt, sbuf, mbar[g], g, tb);
+    else cta_piece<true>(X, sl, off, it.len(), wt, sbuf, mbar[g], g, tb);
+    if (threadIdx.x == 32 + g * kGroupThreads) xtrace(A, op, j, i, 5);
+    mbar_arrive(empty + g);  // release.cta: this thread's stores precede the control warp's wait
+    more = it.next() && it.next();
   }
 }
 
@@ -770,6 +875,11 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   if (kind == 7 && getenv("DT_XFER_NOSPAN")) kind = 1;
   // the block-window kernel (3) is not used inside the pipeline
   X.kind = (kind == 2 || kind == 4 || kind == 6 || kind == 7) ? kind : 1;
+  if (const char* fk = getenv("DT_XFER_KIND")) {  // tuning: force a family where it applies
+    const int k = atoi(fk);
+    const bool wt_ok = f.tsize() / g <= kMaxWordTable && f.tsize() % g == 0 && !E.merged;
+    if ((k == 2 && wt_ok) || (k == 4 && wt_ok && g >= 8) || k == 1) X.kind = k;
+  }
   if (X.kind == 7) P.fnb = make_fd((uint64_t)P.nblocks);
   X.single = P.nblocks == 1;
   X.g = (int32_t)g;
@@ -786,7 +896,7 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
 // shared memory of a record-span op in the transfer kernel: per-warp record buffers and
 // displacements, then the per-CTA map (layout as in xc_rec / k_xfer)
 static size_t rec_smem_bytes(const RecGeo& R, int g) {
-  const size_t nwc = kXferThreads / 32;
+  const size_t nwc = kCopyWarps;
   const size_t tab = std::max<size_t>((size_t)R.RB * R.nwr * 2, (size_t)(R.spanB / g) * 2);
   return nwc * ((size_t)R.RB * R.spanB + (size_t)R.RB * 8) + tab;
 }
@@ -883,10 +993,11 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
     if (X.kind == 2 || X.kind == 4) smem = std::max(smem, sizeof(int32_t) * (size_t)X.P.nwords);
     any_stage = any_stage || X.kind == 4;
     if (X.kind == 6) rec_smem = std::max(rec_smem, rec_smem_bytes(X.rg, X.g));
-    if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)(kXferThreads / 32) * kSpanWarpSmem);
+    if (X.kind == 7) rec_smem = std::max(rec_smem, (size_t)kCopyWarps * kSpanWarpSmem);
   }
   A.nops = nops;
-  A.wt_off = (int32_t)std::max<size_t>(any_stage ? (size_t)kXferStageBufs * kStageTile : 0, (rec_smem + 127) & ~size_t(127));
+  A.wt_off = (int32_t)std::max<size_t>(any_stage ? (size_t)kGroups * kXferStageBufs * kStageTile : 0,
+                                       (rec_smem + 127) & ~size_t(127));
   smem += (size_t)A.wt_off;
   // the attribute is per device (a process may drive several)
   if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -916,30 +1027,39 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
               A.ops[i].depth, A.ops[i].gs, A.ops[i].rep, A.ops[i].ncta, budget);
   static uint64_t* trace = nullptr;
   const char* tr = getenv("DT_XFER_TRACE");  // diagnostics: dump per-piece timestamps to this file
-  const size_t tn = (size_t)kMaxOps * kTraceCtas * kTracePieces * 4;
-  if (tr) {
-    if (!trace) CU(cudaMalloc(&trace, tn * 8));
-    CU(cudaMemsetAsync(trace, 0, tn * 8, s));
+  const size_t tn = (size_t)kMaxOps * kTraceCtas * kTracePieces * kTracePts;
+  if (tr) {  // host-mapped, so a hung kernel's progress is readable
+    if (!trace) CU(cudaHostAlloc(&trace, tn * 8, cudaHostAllocMapped));
+    CU(cudaStreamSynchronize(s));
+    std::memset(trace, 0, tn * 8);
     A.trace = trace;
   }
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
   CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
   if (tr) {
-    std::vector<uint64_t> h(tn);
-    CU(cudaMemcpyAsync(h.data(), trace, tn * 8, cudaMemcpyDeviceToHost, s));
-    CU(cudaStreamSynchronize(s));
+    bool hung = false;
+    for (int w = 0; cudaStreamQuery(s) == cudaErrorNotReady; w++) {
+      if (w > 5000) { hung = true; break; }  // ~5 s
+      usleep(1000);
+    }
     if (FILE* fp = fopen(tr, "a")) {
-      fprintf(fp, "# launch nops %d\n", nops);
+      fprintf(fp, "# launch nops %d%s\n", nops, hung ? " HUNG" : "");
       for (int i = 0; i < nops; i++)
         for (int jj = 0; jj < kTraceCtas; jj++)
           for (int p = 0; p < kTracePieces; p++) {
-            const uint64_t* q = &h[(((size_t)i * kTraceCtas + jj) * kTracePieces + p) * 4];
-            if (q[0]) fprintf(fp, "%d %d %d %d %llu %llu %llu %llu\n", i, A.ops[i].role, jj, p,
-                              (unsigned long long)q[0], (unsigned long long)q[1], (unsigned long long)q[2],
-                              (unsigned long long)q[3]);
+            const volatile uint64_t* q = &trace[(((size_t)i * kTraceCtas + jj) * kTracePieces + p) * kTracePts];
+            if (q[0] || q[4]) {
+              fprintf(fp, "%d %d %d %d", i, A.ops[i].role, jj, p);
+              for (int k = 0; k < kTracePts; k++) fprintf(fp, " %llu", (unsigned long long)q[k]);
+              fprintf(fp, "\n");
+            }
           }
       fclose(fp);
+    }
+    if (hung) {
+      fprintf(stderr, "[dt_xfer] kernel hung; trace written to %s\n", tr);
+      _exit(3);
     }
   }
   return DT_OK;

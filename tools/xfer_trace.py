@@ -10,10 +10,19 @@ import numpy as np
 def main():
     rows = [ln.split() for ln in open(sys.argv[1]) if ln.strip() and not ln.startswith("#")]
     by = defaultdict(list)
+    stamps = {}
     for r in rows:
         op, role, j, p, *t = map(int, r)
+        t = t[:4] if len(t) < 6 else t
+        if p == 63:  # kernel-level stamps: entry, setup done, handshake done, control loop done
+            stamps[(op, role, j)] = t
+            continue
         by[(op, role, j)].append((p, t))
-    base = min(t[0] for v in by.values() for _, t in v)
+    base = min([t[0] for v in by.values() for _, t in v] + [t[0] for t in stamps.values() if t[0]])
+    for key, t in sorted(stamps.items()):
+        print(f"op {key[0]} {'send' if key[1] == 0 else 'recv'} cta {key[2]}: entry {(t[0] - base) / 1e3:6.2f} "
+              f"setup {(t[1] - base) / 1e3:6.2f} handshake {(t[2] - base) / 1e3:6.2f} "
+              f"end {(t[3] - base) / 1e3 if t[3] else float('nan'):6.2f} us")
     for (op, role, j), v in sorted(by.items()):
         v.sort()
         t = np.array([x[1] for x in v], dtype=np.float64) - base
