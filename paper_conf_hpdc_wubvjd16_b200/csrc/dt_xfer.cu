@@ -72,8 +72,9 @@ struct XOp {
   uint8_t* ring;   // slot 0 of the (pair, channel) ring (send: peer memory; recv: local)
   uint64_t* ready; // [depth][kMaxSub] tags  send: peer; recv: local
   uint64_t* ack;   // [depth][kMaxSub] tags  send: local; recv: peer
-  uint64_t* hdr;   // [4] {seq, nbytes|abort, gs, rep}  send: peer; recv: local
-  uint64_t* go;    // [2] {capacity, seq}  send: local; recv: peer
+  uint64_t* hdr;   // [4] {seq, nbytes, gs, rep}  send: peer; recv: local
+  uint64_t* go;    // [2] {consumed seq, aborted seq}  send: local; recv: peer
+  uint32_t* done;  // recv: local counter of CTAs finished with the message (last one posts consumed)
   uint64_t seq;
   int32_t* err;
   RecGeo rg;       // kind 6: record-span geometry (per-fragment element range set on the device)
@@ -227,30 +228,34 @@ __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo,
 // when ncta >= pairs).  The control warp and the copy warps walk the same sequence.
 struct PieceIt {
   int64_t n, C, Cs;
-  int K, D, gs, rep, ncta, j, jstep, kstep, k, js, slot, round;
+  int K, D, gs, gu, rep, ncta, j, jstep, kstep, k, js, slot, round;
   bool one;
+  // gs: pieces per ring slot (layout, Cs = C/gs); gu: pieces of a fragment in use
+  // (fewer than gs when the whole message is shorter than one slot)
   __device__ __forceinline__ bool init(int role, int64_t n_, int64_t C_, int D_, int gs_, int rep_, int ncta_, int j_) {
     n = n_; C = C_; D = D_; gs = gs_; rep = rep_; ncta = ncta_; j = j_;
     Cs = C / gs;
     K = (int)((n + C - 1) / C);
-    const int npairs = gs * rep;
+    gu = (int)min((int64_t)gs, ((n < C ? n : C) + Cs - 1) / Cs);
+    if (gu < 1) gu = 1;
+    const int npairs = gu * rep;
     one = role == 0 || ncta >= npairs;
     if (one && j >= npairs) return false;
     kstep = one ? rep : 1;
-    jstep = one ? gs : ncta;
-    k = one ? j / gs : 0;
+    jstep = one ? gu : ncta;
+    k = one ? j / gu : 0;
     slot = k % D;
     round = k / D;
     js = first_js();
     return settle();
   }
   __device__ __forceinline__ int first_js() const {
-    return one ? j % gs : (((j - (k % rep) * gs) % ncta) + ncta) % ncta;
+    return one ? j % gu : (((j - (k % rep) * gu) % ncta) + ncta) % ncta;
   }
   // advance to a valid (k, js) at or after the current one; false at the end
   __device__ __forceinline__ bool settle() {
     while (k < K) {
-      if (js < gs && (int64_t)k * C + (int64_t)js * Cs < n) return true;
+      if (js < gu && (int64_t)k * C + (int64_t)js * Cs < n) return true;
       k += kstep;
       slot += kstep;
       while (slot >= D) { slot -= D; round++; }
@@ -271,23 +276,40 @@ struct PieceIt {
 // of every op (co-resident: cooperative launch).
 //
 // Message protocol on a (pair, channel), sequence number seq:
-//  * receiver CTA 0 posts {capacity, seq} into the sender's `go` words at kernel
-//    start ("start packing", [L20:c3973]) -- its previous kernel on the channel has
-//    finished, so every ring slot is free;
-//  * sender thread 0 of every CTA waits for go >= seq; CTA 0 writes the header
-//    {seq, n | abort, gs, rep}: abort (n > capacity) moves nothing and both sides
-//    report DT_ERR_TRUNCATE, decided before any byte moves ([L26:c4404], A12);
+//  * the sender does not wait for the receiver's kernel: the receiver posted
+//    "consumed = seq-1" when its previous kernel on the channel finished (the last
+//    of its CTAs, [L20:c4133]), so every ring slot is free; sender CTA 0 writes the
+//    header {seq, n, gs, rep} and the pieces start at once;
 //  * the message is K = ceil(n/C) fragments ("unpack fragment i", [L20:c3380]);
-//    fragment k uses ring slot k % D, is split into gs pieces of C/gs bytes, and
-//    belongs to team k % rep.  Sender CTA (team t, piece js) packs its pieces of
-//    t's fragments straight into the receiver's slot in peer HBM and publishes each
-//    with a system-scope release store of the tag into ready[slot][js]; before
-//    reusing a slot (round r > 0) it waits for ack[slot][js] >= tag(seq, r-1).
-//  * receiver CTAs take (team, piece) pairs round-robin, wait for ready with an
-//    acquire, unpack the piece from local HBM and release the tag into the sender's
-//    ack[slot][js] ([L20:c4133]).
+//    fragment k uses ring slot k % D, is split into gs pieces of C/gs bytes (gu of
+//    them used: fewer for a message shorter than C), and belongs to team k % rep.
+//    Sender CTA (team t, piece js) packs its pieces of t's fragments straight into
+//    the receiver's slot in peer HBM and publishes each with a release store of the
+//    tag into ready[slot][js]; before reusing a slot (round r > 0) it waits for
+//    ack[slot][js] >= tag(seq, r-1);
+//  * receiver CTAs read the header, take (team, piece) pairs round-robin, wait for
+//    ready with an acquire, unpack the piece from local HBM and release the tag into
+//    the sender's ack[slot][js];
+//  * truncation (n > the receive capacity, [L26:c4404], reading A12) is decided by
+//    the receiver from the header before any byte reaches the receive buffer: it
+//    reports DT_ERR_TRUNCATE (an MPI receive-side error), unpacks nothing and posts
+//    "aborted = seq" so a sender waiting for a slot stops (the bytes it staged are
+//    never read; the next message's tags supersede their flags).
 // Flags are written by exactly one CTA, so plain release stores suffice, and since
 // tags only grow nothing is carried between messages.
+// Receiver CTA finished its part of message seq (every piece it owns unpacked and
+// acked, by this thread): the last CTA of the op posts "consumed = seq" to the
+// sender -- the ring is free for the next message on the channel.
+__device__ __forceinline__ void recv_done(const XOp& X, uint64_t seq, bool sys) {
+  __threadfence();  // this CTA's reads of the ring are complete (their values were stored)
+  const uint32_t old = atomicAdd(X.done, 1u);
+  if (old + 1 == (uint32_t)X.ncta) {
+    atomicExch(X.done, 0u);
+    __threadfence();
+    st_release(X.go, seq, sys);
+  }
+}
+
 __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
   // dynamic smem: [staging buffers / record or span buffers] [word table]
   extern __shared__ __align__(128) uint8_t xsm[];
@@ -304,11 +326,6 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   const bool sleep_ok = !(A.flags & 2);
   if (threadIdx.x == 0) xtrace(A, op, j, kTracePieces - 1, 0);  // (diagnostics: kernel entry)
 
-  // the receiver's "start packing" goes out first: it is on the sender's critical path
-  if (X.role == 1 && j == 0 && threadIdx.x == 0) {
-    st_relaxed(X.go, (uint64_t)X.n, X.sys != 0);
-    st_release(X.go + 1, X.seq, X.sys != 0);
-  }
   if (X.kind == 2 || X.kind == 4)
     for (int i = threadIdx.x; i < X.P.nwords; i += blockDim.x) wt[i] = X.P.wtab[i];
   if (X.kind == 6) {  // record-span maps after the per-warp buffers (same layout as xc_rec)
@@ -329,17 +346,16 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
     uint64_t v = 0;
     s_stop = 0;
     if (X.role == 0) {
-      const bool ok = spin(X.go + 1, [seq](uint64_t x) { return x >= seq; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
-      const uint64_t cap = ok ? *(volatile uint64_t*)X.go : 0;
-      const bool abort = (uint64_t)X.n > cap;
+      // the receiver consumed the previous message on the channel: every slot is free
+      const uint64_t prev = seq - 1;
+      const bool ok = spin(X.go, [prev](uint64_t x) { return x >= prev; }, A.timeout_ns, X.err, &v, sleep_ok, sys);
       if (ok && j == 0) {
-        st_relaxed(X.hdr + 1, (uint64_t)X.n | (abort ? kAbort : 0), sys);
+        st_relaxed(X.hdr + 1, (uint64_t)X.n, sys);
         st_relaxed(X.hdr + 2, (uint64_t)X.gs, sys);
         st_relaxed(X.hdr + 3, (uint64_t)X.rep, sys);
         st_release(X.hdr, seq, sys);
-        if (abort) atomicCAS(X.err, 0, XERR_TRUNCATE);
       }
-      s_stop = !ok || abort;
+      s_stop = !ok;
       s_n = (uint64_t)X.n;
       s_gs = X.gs;
       s_rep = X.rep;
@@ -348,13 +364,20 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       const uint64_t nv = ok ? *(volatile uint64_t*)(X.hdr + 1) : 0;
       s_gs = ok ? (int)*(volatile uint64_t*)(X.hdr + 2) : 1;
       s_rep = ok ? (int)*(volatile uint64_t*)(X.hdr + 3) : 1;
-      s_n = nv & ~kAbort;
-      s_stop = !ok || (nv & kAbort);
-      if (ok && (nv & kAbort) && j == 0) atomicCAS(X.err, 0, XERR_TRUNCATE);
+      s_n = nv;
+      const bool trunc = ok && nv > (uint64_t)X.n;
+      s_stop = !ok || trunc;
+      if (trunc && j == 0) {
+        atomicCAS(X.err, 0, XERR_TRUNCATE);
+        st_release(X.go + 1, seq, sys);  // aborted: a sender waiting for a slot stops
+      }
     }
   }
   __syncthreads();
-  if (s_stop) return;
+  if (s_stop) {
+    if (X.role == 1 && threadIdx.x == 0) recv_done(X, seq, sys);
+    return;
+  }
   const int64_t n = (int64_t)s_n;
   // Warp specialisation: warp 0 (lane 0) is the control warp -- it waits for each
   // piece's flag, hands the piece to the copy warps through full[b], waits for the
@@ -423,8 +446,17 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
         ns = 0;
         continue;
       }
+      // a sender waiting for a slot: has the receiver aborted the message (truncation)?
+      if (X.role == 0 && i_rel == i_acq && ld_acquire(X.go + 1, sys) >= seq) {
+        atomicCAS(X.err, 0, XERR_TRUNCATE);
+        s_abort = 1;
+        __threadfence_block();
+        mbar_arrive(full + 0);
+        mbar_arrive(full + 1);
+        return;
+      }
       if (sleep_ok) __nanosleep(ns);
-      ns = ns < 32 ? 32 : (ns < 256 ? 2 * ns : 256);
+      ns = ns < 16 ? 16 : (ns < 64 ? 2 * ns : 64);
       const uint64_t now = gtimer();
       if (!t_idle) t_idle = now;
       else if ((int64_t)(now - t_idle) > A.timeout_ns) {
@@ -440,6 +472,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
       }
     }
     xtrace(A, op, j, kTracePieces - 1, 3);  // control loop done
+    if (X.role == 1) recv_done(X, seq, sys);
     return;
   }
   // ---- copy groups: group g takes the CTA's pieces g, g + 2, g + 4, ...
@@ -562,7 +595,8 @@ struct dt_comm_s {
   int64_t* szhost = nullptr; // pinned
   // layout helpers (uint64 flag words): per (peer, channel) depth*kMaxSub ready tags,
   // a 4-word header {seq, nbytes|abort, pieces, teams}, depth*kMaxSub ack tags and
-  // a 2-word go {capacity, seq}; then one error word.  The ring of a (source,
+  // a 2-word go {consumed seq, aborted seq}, a receiver-local CTA counter; then one
+  // error word.  The ring of a (source,
   // channel) pair is depth*chunk bytes: D slots of one fragment each.
   size_t per() const { return (size_t)kMaxSub * o.depth; }
   size_t pairs() const { return (size_t)nranks * nch; }
@@ -570,7 +604,8 @@ struct dt_comm_s {
   size_t hdr_idx(int src, int ch) const { return pairs() * per() + ((size_t)src * nch + ch) * 4; }
   size_t ack_idx(int dst, int ch) const { return pairs() * (per() + 4) + ((size_t)dst * nch + ch) * per(); }
   size_t go_idx(int dst, int ch) const { return pairs() * (2 * per() + 4) + ((size_t)dst * nch + ch) * 2; }
-  size_t err_idx() const { return pairs() * (2 * per() + 6); }
+  size_t done_idx(int src, int ch) const { return pairs() * (2 * per() + 6) + (size_t)src * nch + ch; }
+  size_t err_idx() const { return pairs() * (2 * per() + 7); }
   size_t ring_off(int src, int ch) const { return (((size_t)src * nch + ch) * o.depth) * (size_t)o.chunk_bytes; }
 };
 
@@ -914,24 +949,31 @@ static int default_ctas(const dt_comm_s* c) {
 // take alternate fragments so several fragments are in flight at once (each team
 // owns D/rep slots).  Depends only on (n, C, D, budget).
 struct Geo {
-  int gs, rep;
+  int gs, gu, rep;
 };
 static Geo geometry(int64_t n, int64_t C, int D, int budget) {
   static const int64_t kPiece = getenv("DT_XFER_PIECE") ? atoll(getenv("DT_XFER_PIECE")) : (32 << 10);
   const int64_t eff = std::min<int64_t>(C, std::max<int64_t>(512, (n + 511) & ~int64_t(511)));
+  // p: CTAs per fragment, pieces of >= kPiece bytes
+  int p = 1;
+  while (p * 2 <= kMaxSub && p * 2 <= budget && eff / (p * 2) >= kPiece) p *= 2;
+  // gs: the slot layout, pieces of C/gs >= eff/p bytes (a message shorter than C uses
+  // gu < gs of them)
+  const int64_t want = (((eff + p - 1) / p) + 511) & ~int64_t(511);
   int gs = 1;
-  while (gs * 2 <= kMaxSub && gs * 2 <= budget && C % ((int64_t)gs * 2 * 512) == 0 && eff / (gs * 2) >= kPiece)
-    gs *= 2;
+  while (gs * 2 <= kMaxSub && C % ((int64_t)gs * 2 * 512) == 0 && C / (gs * 2) >= want) gs *= 2;
+  const int64_t Cs = C / gs;
+  const int gu = (int)std::max<int64_t>(1, std::min<int64_t>(gs, (std::min(n, C) + Cs - 1) / Cs));
   const int64_t K = std::max<int64_t>(1, (n + C - 1) / C);
   const char* rp = getenv("DT_XFER_REP");
   int rep = 1;
   if (rp) {
     rep = std::max(1, atoi(rp));
-    while (rep > 1 && (D % rep || rep * gs > budget)) rep--;
+    while (rep > 1 && (D % rep || rep * gu > budget)) rep--;
   } else {
-    while (rep * 2 <= D && D % (rep * 2) == 0 && rep * 2 * gs <= budget && rep * 2 <= K) rep *= 2;
+    while (rep * 2 <= D && D % (rep * 2) == 0 && rep * 2 * gu <= budget && rep * 2 <= K) rep *= 2;
   }
-  return Geo{gs, rep};
+  return Geo{gs, gu, rep};
 }
 
 static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cudaStream_t s) {
@@ -980,6 +1022,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.hdr = c->flags + c->hdr_idx(p.source, ch);
       X.ack = pf + c->ack_idx(c->rank, ch);
       X.go = pf + c->go_idx(c->rank, ch);
+      X.done = reinterpret_cast<uint32_t*>(c->flags + c->done_idx(p.source, ch));
       X.seq = ++c->recv_seq[(size_t)p.source * c->nch + ch];
       X.sys = !c->same_dev[p.source];
     }
@@ -1007,24 +1050,37 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   int sms = 0, dev = 0;
   CU(cudaGetDevice(&dev));
   CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-  const int budget = std::max(1, std::min(default_ctas(c), occ * sms / nops));
+  // Co-resident CTAs are shared among the ops in proportion to their estimated cost:
+  // bytes x a per-family factor (4-byte words gathered one by one cost ~4x a long-run
+  // copy per byte; the C4 halo's x faces next to its y/z faces).
+  // Unpacking G-byte words scatters partial-sector writes (each a DRAM read-modify-write
+  // when G < 32): measured ~2x the pack cost, so the factor doubles on the receive side.
+  auto cost = [](const XOp& X) {
+    double w = X.kind == 2 ? 16.0 / X.g : (X.kind == 6 || X.kind == 7) ? 2.0 : 1.0;
+    if (X.role == 1 && X.g < 16 && X.kind != 1) w *= 2;
+    return (double)std::max<int64_t>(X.n, 4096) * w;
+  };
+  double csum = 0;
+  for (int i = 0; i < nops; i++) csum += cost(A.ops[i]);
+  const int total = occ * sms;
   int cta = 0;
   for (int i = 0; i < nops; i++) {
     XOp& X = A.ops[i];
+    const int budget = std::max(1, std::min(default_ctas(c), (int)(total * cost(X) / csum)));
     // send role: one CTA per (team, piece); receive role: as many as the capacity
     // would need (the actual geometry arrives in the header; CTAs map onto it)
     const Geo G = geometry(X.n, X.chunk, X.depth, budget);
     X.gs = G.gs;
     X.rep = G.rep;
     X.cta0 = cta;
-    X.ncta = G.gs * G.rep;
+    X.ncta = G.gu * G.rep;
     cta += X.ncta;
   }
   if (getenv("DT_XFER_DEBUG"))
     for (int i = 0; i < nops; i++)
-      fprintf(stderr, "[dt_xfer] op %d role %d kind %d g %d n %lld C %lld D %d gs %d rep %d ncta %d budget %d\n", i,
+      fprintf(stderr, "[dt_xfer] op %d role %d kind %d g %d n %lld C %lld D %d gs %d rep %d ncta %d total %d\n", i,
               A.ops[i].role, A.ops[i].kind, A.ops[i].g, (long long)A.ops[i].n, (long long)A.ops[i].chunk,
-              A.ops[i].depth, A.ops[i].gs, A.ops[i].rep, A.ops[i].ncta, budget);
+              A.ops[i].depth, A.ops[i].gs, A.ops[i].rep, A.ops[i].ncta, total);
   static uint64_t* trace = nullptr;
   const char* tr = getenv("DT_XFER_TRACE");  // diagnostics: dump per-piece timestamps to this file
   const size_t tn = (size_t)kMaxOps * kTraceCtas * kTracePieces * kTracePts;
@@ -1036,7 +1092,9 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   }
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
-  CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
+  static const bool coop = !getenv("DT_XFER_NOCOOP");
+  if (coop) CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
+  else CU(cudaLaunchKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
   if (tr) {
     bool hung = false;
     for (int w = 0; cudaStreamQuery(s) == cudaErrorNotReady; w++) {

@@ -111,6 +111,22 @@ def test_truncation_detected(torch_cuda):
     torch.cuda.synchronize()
     comm.check()
     assert torch.equal(r[:7992], s2[:7992])
+    # a message longer than the whole ring (16 x 64 KiB fragments through 2 slots): the
+    # sender must be released by the receiver's abort instead of waiting for slots
+    big = dt.Type.basic("BYTE").contiguous(1 << 20).commit()
+    small = dt.Type.basic("BYTE").contiguous((1 << 20) - 1).commit()
+    s3 = torch.randint(0, 255, (1 << 20,), dtype=torch.uint8, device="cuda")
+    r3 = torch.full((1 << 20,), 0xA5, dtype=torch.uint8, device="cuda")
+    comm.sendrecv(s3, 1, big, 0, r3, 1, small, 0)
+    torch.cuda.synchronize()
+    with pytest.raises(dt.DTError) as e:
+        comm.check()
+    assert e.value.name == "DT_ERR_TRUNCATE"
+    assert torch.all(r3 == 0xA5)
+    comm.sendrecv(s3, 1, big, 0, r3, 1, big, 0)
+    torch.cuda.synchronize()
+    comm.check()
+    assert torch.equal(r3, s3)
     comm.free()
 
 

@@ -16,7 +16,7 @@ def main():
     n, h = 512, 1
     L = n + 2 * h
     chunk = int(os.environ.get("PROBE_CHUNK", 1 << 20))
-    depth = int(os.environ.get("PROBE_DEPTH", 2))
+    depth = int(os.environ.get("PROBE_DEPTH", 0))
     comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth, ring_loopback=True)
     plan = make_plan(0, n, h, (1, 1, 1))
     buf = torch.empty(L ** 3 * 4, dtype=torch.uint8, device="cuda")
