@@ -9,10 +9,13 @@ run on one GPU: S3 position resolve, S4 work split, S5 pack, S6 unpack; S1/S2
 construct + commit happen once, before timing, as the paper's cached DEVs
 [L24:c2714]).  Metric (BASELINE.json): pack/unpack GB/s counting payload bytes
 read + written, i.e. 2*payload per kernel, reported against the measured HBM
-copy peak.  At N>1 every rank runs the same step on its own matrices (weak
-scaling, no data-path collective) and the line adds a "transfer" object: the
-north_star's multi-GPU metric, the pipelined C3 exchange between pairs (r, r^1)
-over NVLink as a fraction of 900 GB/s per direction (`--workload xfer` sweeps it).
+copy peak.  At N>1 the headline is the north_star's multi-GPU metric instead:
+the pipelined C3 exchange between pairs (r, r^1) through dt_sendrecv over NVLink
+(whole-job bytes received per second; roofline = one rank's GB/s per direction
+against 900 GB/s), with the same bytes contiguous through the same path (the
+paper's "C" comparator) and through NCCL, the NCCL mode, the direct plan, the C4
+halo and C5 pairs in a "transfer" object, and the replicated C2 pack/unpack in a
+side field (`--workload xfer` / `halo` sweep them further).
 
 L2 hygiene: a 2xL2 scratch buffer is rewritten before every timed kernel, and
 only the pack/unpack kernels themselves are inside the CUDA-event intervals.
@@ -173,6 +176,8 @@ def run_ours(args):
     import torch
 
     from paper_conf_hpdc_wubvjd16_b200 import dt
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1:
+        return run_multi(args)
     ws, rank, local = dist_init()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -244,22 +249,6 @@ def run_ours(args):
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(f"c2_{dom}")
     e2e = run_e2e(args, t, src_h, org, parent, payload, dev) if rank == 0 and not args.no_e2e else None
-    transfer = None
-    if ws > 1:
-        # the north_star's multi-GPU metric: pipelined non-contiguous exchange between
-        # pairs (r, r^1) over NVLink (C3 block-cyclic, P2P mode), reported beside the
-        # replica headline as a fraction of 900 GB/s per direction
-        del src, dst, packed, flush, flush_rd
-        torch.cuda.empty_cache()
-        try:
-            res, xpay, xok, _ = xfer_sweep(ws, rank, local, [1 << 20, 4 << 20], [8], "p2p", 0, 10, 3)
-            xb = max(res, key=lambda r: r["gbs_per_rank"])
-            transfer = {"workload": "C3 block-cyclic 128 MiB per direction, pairs (r, r^1), dt_sendrecv P2P",
-                        "value": round(ws * xpay / (xb["ms"] * 1e-3) / 1e9, 1), "unit": UNIT,
-                        "gbs_per_direction": xb["gbs_per_rank"], "peak": 900.0,
-                        "frac": round(xb["gbs_per_rank"] / 900.0, 4), "sweep": res, "spot_parity": xok}
-        except Exception as e:  # noqa: BLE001  (the replica headline above stands on its own)
-            transfer = {"error": f"{type(e).__name__}: {e}"[:300]}
     line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(kern_ms / args.steps, 5), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic (splitmix64 words)",
@@ -275,8 +264,6 @@ def run_ours(args):
                          "traffic": traffic,
                          "algorithmic_bytes_per_launch": 2 * payload},
             "gpu_launches": 2 * args.steps, "clocks": clk.summary(), "e2e": e2e}
-    if transfer is not None:
-        line["transfer"] = transfer
     if rank == 0 and ws == 1 and not args.no_cpu:
         line["cpu_baseline"] = time_oracle_c2(seconds=args.cpu_seconds)[0]
     if rank == 0:
@@ -284,6 +271,261 @@ def run_ours(args):
     if ws > 1:
         import torch.distributed as tdist
         tdist.destroy_process_group()
+
+
+# ------------------------------------------------------------------ N > 1 GPUs
+MULTI_WORKLOAD = ("C3: ScaLAPACK 2D block-cyclic submatrix (N=8192 f64, nb=64, owner (0,1)), 128 MiB per "
+                  "direction, pairwise exchange (r, r^1) through dt_sendrecv (P2P ring over NVLink)")
+
+
+def reduce_max(vals, dev=None):
+    """Max over ranks of a list of floats (the contract's max-over-ranks timing)."""
+    import torch
+    import torch.distributed as tdist
+    if not tdist.is_initialized() or tdist.get_world_size() == 1:
+        return [float(v) for v in vals]
+    x = torch.tensor([float(v) for v in vals], dtype=torch.float64, device=dev if dev is not None else "cpu")
+    tdist.all_reduce(x, op=tdist.ReduceOp.MAX)
+    return [float(v) for v in x.tolist()]
+
+
+def assemble_multi_line(ws, steps, warmup, payload, ring, sub, clocks=None, e2e=None, replica=None, dtype="u8"):
+    """The N>1 JSON line (SURVEY §8(d) multi-GPU metric).  ring: the headline ring
+    exchange {"ms": max-over-ranks ms per exchange, "chunk", "depth", "gbs_per_rank"};
+    sub: side measurements (contiguous comparator, NCCL mode, direct plan, C4 halo,
+    C5 pairs, ...), each already reduced over ranks.  value = bytes received by all
+    ranks per second (whole job); the roofline is one rank's per-direction GB/s
+    against 900 GB/s of NVLink 5 per direction."""
+    per_dir = payload / (ring["ms"] * 1e-3) / 1e9
+    line = {"metric": METRIC, "value": round(ws * per_dir, 1), "unit": UNIT, "n_gpus": ws, "steps": steps,
+            "warmup": warmup, "ms_per_step": round(ring["ms"], 5), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": dtype, "data": "synthetic (splitmix64 words)",
+            "config": {"workload": MULTI_WORKLOAD, "payload_bytes_per_direction": payload,
+                       "pairs": "(r, r^1)", "chunk": ring.get("chunk"), "depth": ring.get("depth"),
+                       "gbs_per_direction": round(per_dir, 1), "parallelism": f"pairs x{ws // 2}",
+                       "l2": "inputs (512 MiB matrices) larger than L2"},
+            "roofline": {"bound": "nvlink", "kernel": "k_xfer (dt_sendrecv, P2P ring)",
+                         "achieved": round(per_dir, 1), "peak": 900.0, "peak_source": "NVLink 5 per direction (spec)",
+                         "unit": "GB/s", "frac": round(per_dir / 900.0, 4), "traffic": None},
+            "gpu_launches": steps, "transfer": sub}
+    c = sub.get("contiguous_same_bytes") or {}
+    if c.get("gbs_per_direction"):
+        line["config"]["of_contiguous"] = round(per_dir / c["gbs_per_direction"], 3)
+    if clocks is not None:
+        line["clocks"] = clocks
+    if e2e is not None:
+        line["e2e"] = e2e
+    if replica is not None:
+        line["replica_pack_unpack"] = replica
+    return line
+
+
+def _guard(fn, *a, **k):
+    """Run one side measurement; a failure is recorded, not fatal (the headline stands)."""
+    if os.environ.get("DT_BENCH_VERBOSE"):
+        print(f"[bench] rank {os.environ.get('RANK')}: {getattr(fn, '__name__', fn)} {a[1:2]}", file=sys.stderr,
+              flush=True)
+    try:
+        return fn(*a, **k)
+    except Exception as e:  # noqa: BLE001
+        return {"error": f"{type(e).__name__}: {e}"[:300]}
+
+
+def _torch_nccl_contig(ws, rank, local, payload, steps, warmup):
+    """ncclSend/ncclRecv of the same number of contiguous bytes (torch.distributed)."""
+    import torch
+    import torch.distributed as tdist
+    if tdist.get_backend() != "nccl":
+        return {"skipped": "process group backend is not nccl"}
+    dev = torch.device("cuda", local)
+    peer = rank ^ 1 if (rank ^ 1) < ws else rank
+    a = torch.empty(payload, dtype=torch.uint8, device=dev).random_(0, 255)
+    b = torch.empty_like(a)
+
+    def one():
+        ops = [tdist.P2POp(tdist.isend, a, peer), tdist.P2POp(tdist.irecv, b, peer)]
+        for r in tdist.batch_isend_irecv(ops):
+            r.wait()
+    for _ in range(warmup):
+        one()
+    torch.cuda.synchronize()
+    tdist.barrier()
+    s = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    for _ in range(steps):
+        one()
+    e1.record(s)
+    torch.cuda.synchronize()
+    ms = reduce_max([e0.elapsed_time(e1) / steps], dev)[0]
+    return {"how": "torch.distributed batch_isend_irecv (ncclSend/ncclRecv) of contiguous bytes",
+            "ms": round(ms, 4), "gbs_per_direction": round(payload / (ms * 1e-3) / 1e9, 1)}
+
+
+def _halo(ws, rank, local, mode, steps, warmup, chunk=1 << 20):
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import make_plan
+    dev = torch.device("cuda", local)
+    dims = {1: (1, 1, 1), 2: (1, 1, 2), 4: (1, 2, 2), 8: (2, 2, 2)}.get(ws, (1, 1, ws))
+    n, h = 512, 1
+    L = n + 2 * h
+    plan = make_plan(rank, n, h, dims)
+    buf = torch.empty(L * L * L * 4, dtype=torch.uint8, device=dev)
+    buf.view(torch.int32).random_(0, 1 << 30)
+    comm = dt.Comm.from_process_group(device=local, chunk_bytes=chunk, depth=0)
+    s = torch.cuda.current_stream()
+    if mode == "direct":
+        xp = plan.direct_plan(comm, buf)
+        one, check = (lambda: xp.start(s)), xp.check
+    else:
+        one, check = (lambda: plan.exchange(comm, buf, stream=s)), comm.check
+    for _ in range(warmup):
+        one()
+    torch.cuda.synchronize()
+    check()
+    torch.distributed.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    for _ in range(steps):
+        one()
+    e1.record(s)
+    torch.cuda.synchronize()
+    check()
+    ms = reduce_max([e0.elapsed_time(e1) / steps], dev)[0]
+    if mode == "direct":
+        xp.free()
+    comm.free()
+    del buf
+    torch.cuda.empty_cache()
+    return {"grid": list(dims), "mode": mode, "us_per_exchange": round(ms * 1e3, 2),
+            "gbs_per_rank": round(6 * n * n * h * 4 / (ms * 1e-3) / 1e9, 1)}
+
+
+def _multi_e2e(ws, rank, local, t, org, steps):
+    """The headline exchange end to end through the public API with host buffers:
+    every step copies the send layout's span from pinned host memory to the device,
+    runs dt_sendrecv, and copies the received span back to pinned host memory."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    dev = torch.device("cuda", local)
+    peer = rank ^ 1 if (rank ^ 1) < ws else rank
+    tlb, text = t.true_extent
+    lo, span = org + tlb, org + tlb + text  # the layout's bytes are [origin + true_lb, + true_extent)
+    hs = torch.empty(span, dtype=torch.uint8).pin_memory()
+    hr = torch.empty(span, dtype=torch.uint8).pin_memory()
+    ds = torch.empty(span, dtype=torch.uint8, device=dev)
+    dr = torch.empty(span, dtype=torch.uint8, device=dev)
+    comm = dt.Comm.from_process_group(device=local, chunk_bytes=4 << 20, depth=0)
+    s = torch.cuda.current_stream()
+
+    def one():
+        ds[lo:].copy_(hs[lo:], non_blocking=True)
+        comm.sendrecv(ds, 1, t, peer, dr, 1, t, peer, sbuf_offset=org, rbuf_offset=org)
+        hr[lo:].copy_(dr[lo:], non_blocking=True)
+    one()
+    torch.cuda.synchronize()
+    torch.distributed.barrier()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        one()
+    torch.cuda.synchronize()
+    el = reduce_max([time.perf_counter() - t0], None)[0]
+    comm.check()
+    comm.free()
+    payload = t.size
+    return {"value": round(ws * payload * steps / el / 1e9, 2), "unit": UNIT,
+            "h2d_bytes_per_step": span - lo, "d2h_bytes_per_step": span - lo, "steps": steps,
+            "note": "pinned host buffers; per step: H2D of the send layout's span, dt_sendrecv, D2H of the "
+                    "received span; wall clock, max over ranks"}
+
+
+def _replica_c2(local, steps, warmup):
+    """Every rank packs + unpacks its own C2 triangle (no data-path collective): the
+    1-GPU metric, replicated; min over ranks of the per-rank GB/s."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    dev = torch.device("cuda", local)
+    rec, org, parent, src_h = c2_buffers(torch)
+    t = dt.from_recipe(rec).commit()
+    src = torch.from_numpy(src_h).to(dev)
+    dst = torch.empty(parent, dtype=torch.uint8, device=dev)
+    pk = torch.empty(t.size, dtype=torch.uint8, device=dev)
+    flush = torch.empty(2 * torch.cuda.get_device_properties(dev).L2_cache_size, dtype=torch.uint8, device=dev)
+    s = torch.cuda.current_stream()
+    tot = 0.0
+    for i in range(warmup + steps):
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+        flush.fill_(1)
+        ev[0].record(s)
+        dt.pack(t, 1, src, pk, origin_offset=org)
+        ev[1].record(s)
+        flush.fill_(2)
+        ev[2].record(s)
+        dt.unpack(t, 1, pk, dst, origin_offset=org)
+        ev[3].record(s)
+        torch.cuda.synchronize()
+        if i >= warmup:
+            tot += ev[0].elapsed_time(ev[1]) + ev[2].elapsed_time(ev[3])
+    ms = reduce_max([tot / steps], dev)[0]
+    del src, dst, pk, flush
+    torch.cuda.empty_cache()
+    return {"workload": WORKLOAD, "ms_per_step": round(ms, 5),
+            "gbs_per_rank": round(4 * t.size / (ms * 1e-3) / 1e9, 1), "note": "slowest rank; L2 flushed per kernel"}
+
+
+def run_multi(args):
+    """N > 1: the north_star's multi-GPU metric.  Headline = the pipelined C3
+    exchange between pairs (r, r^1) through dt_sendrecv's P2P ring (best of 1 and 4
+    MiB fragments, auto depth); beside it, in the same run, the same bytes contiguous
+    through the same path (the paper's "C" comparator, [L26:c977 §5.2]) and through
+    torch/NCCL, the NCCL mode and the direct plan on C3, the C4 halo (ring and direct)
+    and C5 pairs.  Replica C2 pack/unpack moves to a side field."""
+    import torch
+    os.environ.setdefault("DT_TIMEOUT_MS", "15000")
+    ws, rank, local = dist_init()
+    dev = torch.device("cuda", local)
+    steps = max(3, min(args.steps, 10))
+    w = args.warmup
+    clk = ClockSampler(local)
+    if os.environ.get("DT_BENCH_VERBOSE"):
+        print(f"[bench] rank {rank}: ring C3 headline", file=sys.stderr, flush=True)
+    with clk:
+        ring_res, payload, ok, (t, A, B, org) = xfer_sweep(ws, rank, local, [1 << 20, 4 << 20], [0], "p2p", 0,
+                                                          steps, w)
+    best = max(ring_res, key=lambda r: r["gbs_per_rank"])
+    del A, B
+    torch.cuda.empty_cache()
+    sub = {"ring_sweep": ring_res, "spot_parity": ok}
+
+    def sweep1(mode, workload, chunks=(4 << 20,), depths=(0,)):
+        r, pay, okk, (_, a, b, _) = xfer_sweep(ws, rank, local, list(chunks), list(depths), mode, 0, steps, w,
+                                               workload)
+        del a, b
+        torch.cuda.empty_cache()
+        bb = max(r, key=lambda x: x["gbs_per_rank"])
+        return {"ms": bb["ms"], "gbs_per_direction": bb["gbs_per_rank"], "chunk": bb["chunk"],
+                "depth": bb["depth"], "spot_parity": okk, "payload": pay}
+    sub["contiguous_same_bytes"] = _guard(sweep1, "p2p", "ctg", (1 << 20, 4 << 20))
+    sub["contiguous_same_bytes"]["how"] = "dt_sendrecv of 128 MiB contiguous bytes, same ring (paper's C)"
+    sub["nccl_contiguous"] = _guard(_torch_nccl_contig, ws, rank, local, payload, steps, w)
+    sub["nccl_mode_c3"] = _guard(sweep1, "nccl", "c3", (4 << 20,), (4,))
+    sub["direct_plan_c3"] = _guard(sweep1, "direct", "c3")
+    sub["c4_halo_ring"] = _guard(_halo, ws, rank, local, "p2p", steps, w)
+    sub["c4_halo_direct"] = _guard(_halo, ws, rank, local, "direct", steps, w)
+    c5 = {}
+    for m in (1 << 10, 1 << 20, 64 << 20):
+        c5[str(m)] = _guard(sweep1, "p2p", f"c5:{m}", (1 << 20,))
+    sub["c5_pairs"] = c5
+    e2e = _guard(_multi_e2e, ws, rank, local, t, org, steps) if not args.no_e2e else None
+    replica = _guard(_replica_c2, local, steps, w)
+    line = assemble_multi_line(ws, steps, w, payload, best, sub, clocks=clk.summary(), e2e=e2e, replica=replica)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    torch.distributed.destroy_process_group()
 
 
 def run_e2e(args, t, src_h, org, parent, payload, dev):
@@ -349,8 +591,13 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup, 
     from workloads import c3_block_cyclic, c5_particles, c5b_irregular, fill_bytes, seed_for
     dev = torch.device("cuda", local)
     peer = rank ^ 1 if (rank ^ 1) < ws else rank
-    rec, org, parent = {"c3": c3_block_cyclic, "c5": lambda: c5_particles(128 << 20),
-                        "c5b": lambda: c5b_irregular(128 << 20)}[workload]()
+    if workload.startswith("c5:"):  # C5 particle message of a given size (pairs sweep)
+        rec, org, parent = c5_particles(int(workload[3:]))
+    elif workload == "ctg":  # the paper's "C" comparator: the same bytes as C3, contiguous
+        rec, org, parent = ("contiguous", 128 << 20, ("basic", "BYTE")), 0, 128 << 20
+    else:
+        rec, org, parent = {"c3": c3_block_cyclic, "c5": lambda: c5_particles(128 << 20),
+                            "c5b": lambda: c5b_irregular(128 << 20)}[workload]()
     t = dt.from_recipe(rec).commit()
     payload = t.size
     A = torch.from_numpy(fill_bytes(parent, seed_for(3) + rank)).to(dev)

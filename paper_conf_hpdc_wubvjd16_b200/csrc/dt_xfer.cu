@@ -1005,6 +1005,10 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.go = c->flags + c->go_idx(p.dest, ch);
       X.seq = ++c->send_seq[(size_t)p.dest * c->nch + ch];
       X.sys = !c->same_dev[p.dest];
+      // a peer on another GPU: the staged family's TMA bulk stores would target peer
+      // memory, never exercised on a one-GPU lease -- use the word-table family's
+      // plain 16-byte stores there (DT_XFER_PEER_TMA=1 keeps TMA)
+      if (X.sys && X.kind == 4 && !getenv("DT_XFER_PEER_TMA")) X.kind = 2;
     }
     if (p.source >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
