@@ -152,7 +152,17 @@ def time_oracle_c2(seconds=10.0, threads=1):
     value = 4.0 * payload * reps / (tp + tu) / 1e9
     return {"value": round(value, 4), "unit": UNIT, "cores": threads, "kind": "oracle",
             "sample": f"{reps} x (pack+unpack of the full C2 triangle, {payload} B payload), "
-                      f"{tp + tu:.1f} s wall, single process"}, reps, tp + tu
+                      f"{tp + tu:.1f} s wall, one process, {threads} thread(s)"}, reps, tp + tu
+
+
+def _cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def run_reference(args):
@@ -244,10 +254,12 @@ def run_ours(args):
     avg_unpack = statistics.mean(tup)
     dom_ms, dom = (avg_pack, "pack") if avg_pack >= avg_unpack else (avg_unpack, "unpack")
     achieved = 2 * payload / (dom_ms * 1e-3) / 1e9
-    traffic = None
+    traffic, traffic_src = None, None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
-        traffic = json.load(open(tp)).get(f"c2_{dom}")
+        tj = json.load(open(tp))
+        traffic, traffic_src = tj.get(f"c2_{dom}"), tj.get("_source")
+    beyond = _beyond_l2(dev, args) if not args.no_beyond else None
     e2e = run_e2e(args, t, src_h, org, parent, payload, dev) if rank == 0 and not args.no_e2e else None
     line = {"metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(kern_ms / args.steps, 5), "higher_is_better": True,
@@ -261,11 +273,20 @@ def run_ours(args):
                        "parallelism": f"replicas x{ws}" if ws > 1 else "1 GPU"},
             "roofline": {"bound": "hbm", "kernel": f"k_seg<{dom}> (dt_{dom})", "achieved": round(achieved, 1),
                          "peak": peak, "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / peak, 4),
-                         "traffic": traffic,
+                         "traffic": traffic, "traffic_source": traffic_src,
                          "algorithmic_bytes_per_launch": 2 * payload},
             "gpu_launches": 2 * args.steps, "clocks": clk.summary(), "e2e": e2e}
+    if beyond is not None:
+        line["beyond_l2"] = beyond
     if rank == 0 and ws == 1 and not args.no_cpu:
-        line["cpu_baseline"] = time_oracle_c2(seconds=args.cpu_seconds)[0]
+        # the oracle as it stands, on every host core the process may use (its pthread
+        # mode splits the stream into equal byte ranges), and single-threaded beside it
+        cores = len(os.sched_getaffinity(0))
+        cb = time_oracle_c2(seconds=args.cpu_seconds, threads=cores)[0]
+        one = time_oracle_c2(seconds=args.cpu_seconds / 2, threads=1)[0]
+        cb["single_thread"] = {"value": one["value"], "cores": 1, "sample": one["sample"]}
+        cb["cpu_model"] = _cpu_model()
+        line["cpu_baseline"] = cb
     if rank == 0:
         print(json.dumps(line), flush=True)
     if ws > 1:
@@ -526,6 +547,47 @@ def run_multi(args):
     if rank == 0:
         print(json.dumps(line), flush=True)
     torch.distributed.destroy_process_group()
+
+
+def _beyond_l2(dev, args):
+    """A long-run point L2 cannot flatter: the lower triangle of a 16384^2 f64 matrix
+    (2 GiB matrix, 1 GiB payload, 8x L2), pack + unpack, event-timed per kernel."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from workloads import c2_lower_triangle
+    try:
+        rec, org, parent = c2_lower_triangle(16384)
+        t = dt.from_recipe(rec).commit()
+        src = torch.empty(parent, dtype=torch.uint8, device=dev).random_(0, 255)
+        dst = torch.empty(parent, dtype=torch.uint8, device=dev)
+        pk = torch.empty(t.size, dtype=torch.uint8, device=dev)
+        s = torch.cuda.current_stream()
+        for _ in range(2):
+            dt.pack(t, 1, src, pk)
+            dt.unpack(t, 1, pk, dst)
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        n = 5
+        ev[0].record(s)
+        for _ in range(n):
+            dt.pack(t, 1, src, pk)
+        ev[1].record(s)
+        for _ in range(n):
+            dt.unpack(t, 1, pk, dst)
+        ev[2].record(s)
+        torch.cuda.synchronize()
+        ok = bool(torch.equal(src[: 16384 * 8], dst[: 16384 * 8]))  # column 0 lies wholly in the triangle
+        tp, tu = ev[0].elapsed_time(ev[1]) / n, ev[1].elapsed_time(ev[2]) / n
+        peak, _ = load_peaks()
+        gp, gu = 2 * t.size / (tp * 1e-3) / 1e9, 2 * t.size / (tu * 1e-3) / 1e9
+        del src, dst, pk
+        torch.cuda.empty_cache()
+        return {"workload": "T16K: lower triangle of 16384x16384 f64 (1 GiB payload, 8x L2)",
+                "pack_ms": round(tp, 4), "unpack_ms": round(tu, 4), "pack_gbs": round(gp, 1),
+                "unpack_gbs": round(gu, 1), "pack_frac": round(gp / peak, 4), "unpack_frac": round(gu / peak, 4),
+                "spot_check": ok}
+    except Exception as e:  # noqa: BLE001
+        return {"error": f"{type(e).__name__}: {e}"[:200]}
 
 
 def run_e2e(args, t, src_h, org, parent, payload, dev):
@@ -944,6 +1006,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true",
                     help="skip the host-buffer e2e leg (ncu launch lists of the timed device step)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--no-beyond", action="store_true", help="skip the beyond-L2 T16K sub-measurement")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -12,11 +12,11 @@ for step in "$@"; do
            echo "smoke rc=$?" >> gpurun_out/smoke.log; tail -2 gpurun_out/smoke.log ;;
     bench) timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; cat gpurun_out/bench.json ;;
     launches) timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
-                --log-file gpurun_out/launches.csv python bench.py --steps 5 --warmup 3 --no-cpu --no-e2e \
+                --log-file gpurun_out/launches.csv python bench.py --steps 5 --warmup 3 --no-cpu --no-e2e --no-beyond \
                 > gpurun_out/b_ncu.log 2>&1 ;;
     ncu=*) k="${step#ncu=}"
            timeout 900 ncu --set full --clock-control none --import-source on -k "regex:$k" -c 2 \
-             -o "gpurun_out/full_${k//[^a-zA-Z0-9_]/_}" -f python bench.py --steps 3 --warmup 3 --no-cpu --no-e2e \
+             -o "gpurun_out/full_${k//[^a-zA-Z0-9_]/_}" -f python bench.py --steps 3 --warmup 3 --no-cpu --no-e2e --no-beyond \
              > "gpurun_out/ncu_${k//[^a-zA-Z0-9_]/_}.log" 2>&1 ;;
     cmd=*) bash -c "${step#cmd=}" ;;
   esac
