@@ -21,6 +21,7 @@ def main():
     ap.add_argument("--configs", default="C1,C1b,C2,C3,C4x,C4y,C4z,C5_64M,C5_1G,C5b_64M,V4K,V8K,V16K,T16K")
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--l2fetch", type=int, default=0, help="cudaLimitMaxL2FetchGranularity (bytes) for the run")
+    ap.add_argument("--naive", default="", help="configs that also time the per-block cudaMemcpyAsync baseline")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -36,6 +37,7 @@ def main():
         "V4K": lambda: W.c1_submatrix(4096, 8192), "V8K": lambda: W.c1_submatrix(8192, 16384),
         "V16K": lambda: W.c1_submatrix(16384, 16384),
         "T16K": lambda: W.c2_lower_triangle(16384), "Tstair8K": lambda: W.stair_triangle(8192, 256),
+        "T8K": lambda: W.c2_lower_triangle(8192), "C5b_1M": lambda: W.c5b_irregular(1 << 20),
     }
     dev = torch.device("cuda")
     torch.zeros(1, device=dev)
@@ -108,6 +110,35 @@ def main():
             tm = timeit(m2d)
             row.update({"memcpy2d_us": round(tm * 1e3, 2), "memcpy2d_gbs": gb(tm),
                         "pack_vs_memcpy2d": round(tm / tp, 3)})
+        if args.naive and name in args.naive.split(","):
+            # f4 naive baseline (Fig. 1c, [L14:c4769 §3]): one device-to-device cudaMemcpyAsync per
+            # contiguous block of the flattened typemap -- issued from a host loop (what a user gets),
+            # and captured once into a CUDA graph and replayed (the copy engine's per-block floor
+            # without host launch cost)
+            from cuda.bindings import runtime as cudart
+            disp, lens = t.flatten(1)
+            offs = np.concatenate([[0], np.cumsum(lens)[:-1]])
+            base_s, base_p = src.data_ptr() + org, pk.data_ptr()
+            D2D = cudart.cudaMemcpyKind.cudaMemcpyDeviceToDevice
+
+            def loop():
+                for d, ln, o in zip(disp.tolist(), lens.tolist(), offs.tolist()):
+                    cudart.cudaMemcpyAsync(base_p + o, base_s + d, ln, D2D, s.cuda_stream)
+            tl = timeit(loop)
+            g = torch.cuda.CUDAGraph()
+            cs = torch.cuda.Stream()
+            with torch.cuda.stream(cs):
+                with torch.cuda.graph(g, stream=cs):
+                    for d, ln, o in zip(disp.tolist(), lens.tolist(), offs.tolist()):
+                        cudart.cudaMemcpyAsync(base_p + o, base_s + d, ln, D2D, cs.cuda_stream)
+            tg = timeit(g.replay)
+            dt.pack(t, 1, src, a, origin_offset=org, stream=s)  # the naive copies must build the same stream
+            torch.cuda.synchronize()
+            row["naive_parity"] = bool(torch.equal(pk, a))
+            row.update({"naive_blocks": int(len(lens)), "naive_loop_us": round(tl * 1e3, 1),
+                        "naive_loop_gbs": gb(tl), "naive_graph_us": round(tg * 1e3, 1), "naive_graph_gbs": gb(tg),
+                        "pack_vs_naive_loop": round(tl / tp, 1), "pack_vs_naive_graph": round(tg / tp, 1)})
+            del g
         print(json.dumps(row), flush=True)
         del src, pk, dst, a, b
         torch.cuda.empty_cache()
