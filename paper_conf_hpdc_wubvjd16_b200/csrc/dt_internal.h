@@ -119,7 +119,8 @@ struct dt_type_s {
   dt::Kind kind = dt::K_BASIC;
   int basic = 0;
   int64_t count = 0, blocklen = 0, stride = 0;           // stride in bytes
-  std::vector<int64_t> bls, dps;                          // bytes
+  std::vector<int64_t> bls, dps;                          // bytes (struct; hindexed: bls only when not uniform)
+  std::shared_ptr<std::vector<int64_t>> hdps;             // hindexed displacements (bytes), shared with the form
   std::vector<dt_type_s*> types;                          // struct components
   int ndims = 0, order = 0;
   std::vector<int64_t> sizes, subsizes, starts;

@@ -449,6 +449,7 @@ static int64_t host_cost(const KP& P, const Form& f, int64_t alpha, int64_t p) {
   const int64_t ce = P.tsize + alpha * P.nblocks;
   const int64_t e = p / P.tsize;
   const int64_t rem = p - e * P.tsize;
+  if (rem == 0) return e * ce;  // element boundary (pos 0, a whole stream): no block search
   int64_t b = 0, bo = 0;
   if (P.nblocks > 1) {
     const auto& h = f.hoff();

@@ -15,6 +15,8 @@
 #include <cstring>
 #include <numeric>
 
+#include <sys/mman.h>
+
 #include "dt_internal.h"
 
 namespace dt {
@@ -28,6 +30,22 @@ void set_error(const char* fmt, ...) {
 }
 
 static const int64_t kBasicSize[8] = {1, 1, 1, 2, 4, 8, 4, 8};
+
+// Reserve a large vector on transparent huge pages (first-use cost, f2): a 1 GB
+// index list has ~2e7-3e7 entries, and faulting 240 MB in 4 KiB pages costs more
+// than the flattening arithmetic itself.
+static void huge_reserve(std::vector<int64_t>& v, size_t n) {
+  v.reserve(n);
+  const size_t bytes = n * sizeof(int64_t), hp = size_t(2) << 20;
+  if (bytes < 4 * hp) return;
+  const uintptr_t a = ((uintptr_t)v.data() + hp - 1) & ~(uintptr_t)(hp - 1);
+  const uintptr_t e = ((uintptr_t)v.data() + bytes) & ~(uintptr_t)(hp - 1);
+  if (e > a) madvise((void*)a, e - a, MADV_HUGEPAGE);
+}
+static void huge_assign(std::vector<int64_t>& v, const int64_t* p, size_t n) {
+  huge_reserve(v, n);
+  v.assign(p, p + n);
+}
 
 // ------------------------------------------------------------------ bounds
 // Bounds of a constructed type from the range of shifts its copies of T take
@@ -170,32 +188,36 @@ static dt_status create_hindexed(int64_t count, const int64_t* bls, int64_t ubl,
   CHECK_ARG(old && out, "NULL argument");
   CHECK_ARG(count >= 0, "negative count");
   CHECK_ARG(count == 0 || dps, "NULL arrays");
-  if (bls) {
-    for (int64_t i = 0; i < count; i++) CHECK_ARG(bls[i] >= 0, "negative blocklen");
-  } else {
-    CHECK_ARG(ubl >= 0, "negative blocklen");
-  }
-  auto* t = new dt_type_s;
-  t->kind = K_HINDEXED;
-  t->count = count;
-  if (bls) t->bls.assign(bls, bls + count);
-  else t->bls.assign((size_t)count, ubl);
-  t->dps.assign(dps, dps + count);
-  t->old = retain(old);
+  if (!bls) CHECK_ARG(ubl >= 0, "negative blocklen");
   // every copy is of the same type `old`, so the bounds need only the range of the
-  // shifts over all copies and their number (one pass, no per-entry Bounds update)
-  Bounds b;
+  // shifts over all copies and their number: one pass over the arrays (which also
+  // validates the block lengths), before anything is allocated
   const int64_t e = old->extent();
   int64_t smin = INT64_MAX, smax = INT64_MIN, ncopies = 0;
+  bool neg = false;
   for (int64_t i = 0; i < count; i++) {
     const int64_t n = bls ? bls[i] : ubl;
-    if (n == 0) continue;
+    neg |= n < 0;
+    if (n <= 0) continue;
     const int64_t last = (n - 1) * e;
     const int64_t lo = dps[i] + (last < 0 ? last : 0), hi = dps[i] + (last > 0 ? last : 0);
     smin = lo < smin ? lo : smin;
     smax = hi > smax ? hi : smax;
     ncopies += n;
   }
+  CHECK_ARG(!neg, "negative blocklen");
+  auto* t = new dt_type_s;
+  t->kind = K_HINDEXED;
+  t->count = count;
+  // f2 (first-use cost): a uniform block length is kept as one number, and the
+  // displacement list is held once and shared with the flattened form's list level
+  // (a 1 GB index list has ~2e7 entries; every extra copy of it is page faults)
+  if (bls) huge_assign(t->bls, bls, (size_t)count);
+  t->blocklen = bls ? -1 : ubl;
+  t->hdps = std::make_shared<std::vector<int64_t>>();
+  huge_assign(*t->hdps, dps, (size_t)count);
+  t->old = retain(old);
+  Bounds b;
   if (ncopies > 0) b.add(old, smin, smax, ncopies);
   b.finish(t, false);
   *out = t;
@@ -366,17 +388,22 @@ static void prepend_list(Form& f, const std::vector<int64_t>& tab) {
   f.lv.insert(f.lv.begin(), l);
 }
 
+// merge adjacent blocks, drop empty ones -- in place (a list of 3e7 blocks must not be
+// copied again)
 static void merge_template(Form& f) {
-  std::vector<int64_t> d, l;
-  d.reserve(f.bd.size());
-  l.reserve(f.bl.size());
+  size_t w = 0;
   for (size_t i = 0; i < f.bd.size(); i++) {
     if (f.bl[i] == 0) continue;
-    if (!d.empty() && d.back() + l.back() == f.bd[i]) l.back() += f.bl[i];
-    else { d.push_back(f.bd[i]); l.push_back(f.bl[i]); }
+    if (w > 0 && f.bd[w - 1] + f.bl[w - 1] == f.bd[i]) {
+      f.bl[w - 1] += f.bl[i];
+    } else {
+      f.bd[w] = f.bd[i];
+      f.bl[w] = f.bl[i];
+      w++;
+    }
   }
-  f.bd.swap(d);
-  f.bl.swap(l);
+  f.bd.resize(w);
+  f.bl.resize(w);
 }
 
 void normalize(Form& f) {
@@ -524,31 +551,47 @@ static Form build_form(const dt_type_s* t) {
       break;
     }
     case K_HINDEXED: {
-      // entries with blocklen 0 contribute nothing; the common case (none) avoids the
-      // filtered copies (a 1 GB index list has ~2e7 entries: first-use cost, f2)
+      // entries with blocklen 0 contribute nothing; the common cases (a uniform block
+      // length, or no zero entries) use the type's arrays as they are -- no filtered
+      // copies (first-use cost, f2)
+      const std::vector<int64_t>& dps = *t->hdps;
+      Form sub = build_form(t->old);
+      normalize(sub);
+      if (t->count == 0 || sub.empty()) break;
+      if (t->blocklen >= 0) {  // hindexed_block: uniform
+        if (t->blocklen == 0) break;
+        f = sub;
+        prepend_regular(f, t->blocklen, t->old->extent());
+        Level l;  // the list level shares the type's displacement array
+        l.cnt = t->count;
+        l.table = t->hdps;
+        f.lv.insert(f.lv.begin(), l);
+        break;
+      }
       const bool all_pos = std::all_of(t->bls.begin(), t->bls.end(), [](int64_t x) { return x > 0; });
       std::vector<int64_t> B, D;
       if (!all_pos) {
         for (int64_t i = 0; i < t->count; i++)
-          if (t->bls[i] > 0) { B.push_back(t->bls[i]); D.push_back(t->dps[i]); }
+          if (t->bls[i] > 0) { B.push_back(t->bls[i]); D.push_back(dps[i]); }
       }
       const std::vector<int64_t>& Bv = all_pos ? t->bls : B;
-      const std::vector<int64_t>& Dv = all_pos ? t->dps : D;
-      Form sub = build_form(t->old);
-      normalize(sub);
-      if (Bv.empty() || sub.empty()) break;
+      const std::vector<int64_t>& Dv = all_pos ? dps : D;
+      if (Bv.empty()) break;
       bool uniform = std::all_of(Bv.begin(), Bv.end(), [&](int64_t x) { return x == Bv[0]; });
       if (uniform) {
         f = sub;
         prepend_regular(f, Bv[0], t->old->extent());
         prepend_list(f, Dv);
       } else if (is_simple_run(sub, t->old->extent())) {
-        // indexed of a contiguous element: one block per entry (the triangle, C2)
-        f.bd.resize(Bv.size());
-        f.bl.resize(Bv.size());
+        // indexed of a contiguous element: one block per entry (the triangle C2, the
+        // irregular list C5b), adjacent blocks merged in the same pass
+        const int64_t d0 = sub.bd[0], l0 = sub.bl[0];
+        huge_reserve(f.bd, Bv.size());
+        huge_reserve(f.bl, Bv.size());
         for (size_t i = 0; i < Bv.size(); i++) {
-          f.bd[i] = Dv[i] + sub.bd[0];
-          f.bl[i] = Bv[i] * sub.bl[0];
+          const int64_t d = Dv[i] + d0, l = Bv[i] * l0;
+          if (!f.bd.empty() && f.bd.back() + f.bl.back() == d) f.bl.back() += l;
+          else { f.bd.push_back(d); f.bl.push_back(l); }
         }
       } else {
         int64_t e = t->old->extent();

@@ -1,0 +1,71 @@
+"""f2: first-use (uncached) cost vs cached, per workload.
+
+The paper prepares its CUDA DEVs on the CPU for every call unless cached and
+overlaps that preparation with the pack kernels ([L18:c1121]-[L18:c1649 §3.2];
+uncached vs cached T, Fig. 7, [L24:c2562 §5.1]).  Here the preparation is the
+commit: host flattening into levels + template, then the device upload (with the
+device prefix scan); the first pack also builds its launch plan.  For each
+workload this prints, in ms: type construction, host flattening, device upload,
+the first pack (upload pipelined with it when the list is large), a cached pack,
+and first-use total vs cached.
+"""
+import json
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+from paper_conf_hpdc_wubvjd16_b200 import dt  # noqa: E402
+import workloads as W  # noqa: E402
+
+
+def main():
+    names = os.environ.get("FU_CONFIGS", "C2,T16K,C5_1G,C5b_1G").split(",")
+    mk = {"C2": lambda: W.c2_lower_triangle(4096), "T16K": lambda: W.c2_lower_triangle(16384),
+          "C5_1G": lambda: W.c5_particles(1 << 30), "C5b_1G": lambda: W.c5b_irregular(1 << 30),
+          "C5_64M": lambda: W.c5_particles(64 << 20)}
+    dev = torch.device("cuda")
+    torch.zeros(1, device=dev)
+    s = torch.cuda.current_stream()
+    for name in names:
+        rec, org, parent = mk[name]()
+        src = torch.empty(parent, dtype=torch.uint8, device=dev).random_(0, 255)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        t = dt.from_recipe(rec)
+        t1 = time.perf_counter()
+        t.form()  # host flattening only
+        t2 = time.perf_counter()
+        t.commit()  # device upload (+ the pipelined first-use path when it applies)
+        torch.cuda.synchronize()
+        t3 = time.perf_counter()
+        pk = torch.empty(t.size, dtype=torch.uint8, device=dev)
+        torch.cuda.synchronize()
+        t4 = time.perf_counter()
+        dt.pack(t, 1, src, pk, origin_offset=org, stream=s)
+        torch.cuda.synchronize()
+        t5 = time.perf_counter()
+        first = pk.clone()
+        reps = 5
+        c0 = time.perf_counter()
+        for _ in range(reps):
+            dt.pack(t, 1, src, pk, origin_offset=org, stream=s)
+        torch.cuda.synchronize()
+        cached = (time.perf_counter() - c0) / reps
+        same = bool(torch.equal(first, pk))
+        ms = lambda x: round(x * 1e3, 3)  # noqa: E731
+        print(json.dumps({"config": name, "bytes": t.size, "create_ms": ms(t1 - t0), "host_flatten_ms": ms(t2 - t1),
+                          "commit_upload_ms": ms(t3 - t2), "first_pack_ms": ms(t5 - t4),
+                          "cached_pack_ms": ms(cached),
+                          "first_use_ms": ms((t2 - t1) + (t3 - t2) + (t5 - t4)),
+                          "first_use_over_cached": round(((t2 - t1) + (t3 - t2) + (t5 - t4)) / cached, 1),
+                          "first_equals_cached": same}), flush=True)
+        del src, pk, first
+        del t
+        torch.cuda.empty_cache()
+
+
+if __name__ == "__main__":
+    main()
