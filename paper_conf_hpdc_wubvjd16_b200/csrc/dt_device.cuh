@@ -51,6 +51,10 @@ struct KP {
   FastDiv fnb;  // division by nblocks (short-block window kernel)
   int64_t per_warp;
   const int32_t* wtab;
+  // compact block descriptors (block-span kernel): block i = (len << 32) | (uint32)(disp
+  // - wbase[i / 32]); 8 bytes per block instead of 16 (nullptr: use bd/bl)
+  const uint64_t* sdesc;
+  const int64_t* wbase;
 };
 
 // byte displacement of element e: mixed radix over the levels, last fastest
@@ -1046,11 +1050,25 @@ __device__ __forceinline__ uint64_t span_desc_issue(const KP& P, const SpanCur& 
   if (P.nblocks == 1) {
     dsc[2 * lane] = P.bl0;
     dsc[2 * lane + 1] = P.bd0;
+  } else if (P.sdesc) {  // compact: (len, disp - group base) + the 32-block group's base
+    cp_async<8>(dsc + 2 * lane, P.sdesc + b);
+    cp_async<8>(dsc + 2 * lane + 1, P.wbase + (b >> 5));
   } else {
     cp_async<8>(dsc + 2 * lane, P.bl + b);
     cp_async<8>(dsc + 2 * lane + 1, P.bd + b);
   }
   return e;
+}
+// a landed descriptor pair -> (len, disp)
+__device__ __forceinline__ void span_desc_get(const KP& P, const int64_t* dsc, int lane, int64_t& len, int64_t& disp) {
+  const int64_t x = dsc[2 * lane], y = dsc[2 * lane + 1];
+  if (P.sdesc && P.nblocks != 1) {
+    len = (int64_t)((uint64_t)x >> 32);
+    disp = y + (int64_t)(int32_t)(uint32_t)x;
+  } else {
+    len = x;
+    disp = y;
+  }
 }
 // One window's geometry (per lane: its block's share).
 struct SpanWin {
@@ -1067,8 +1085,10 @@ __device__ __forceinline__ SpanWin span_geom(const KP& P, SpanCur& c, uint64_t e
   constexpr int32_t kClamp = 1 << 30;
   SpanWin w;
   const int64_t skip = lane == 0 ? c.r : 0;
+  int64_t dlen, ddisp;
+  span_desc_get(P, dsc, lane, dlen, ddisp);
   // lengths clamped to 4 KiB for the 32-bit scan: a window never exceeds kSpanOut
-  const int32_t len = (int32_t)min(dsc[2 * lane] - skip, (int64_t)4096);
+  const int32_t len = (int32_t)min(dlen - skip, (int64_t)4096);
   int32_t inc = len;
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
@@ -1079,7 +1099,7 @@ __device__ __forceinline__ SpanWin span_geom(const KP& P, SpanCur& c, uint64_t e
   w.L = (int32_t)min((int64_t)min(kSpanOut, __shfl_sync(FULL, inc, 31)), p1 - c.p);
   w.n = max(0, min(inc, w.L) - w.off);  // lanes with n > 0 are a prefix (lane 0 always)
   w.a = 0;
-  if (w.n > 0) w.a = (int64_t)(uintptr_t)P.nc + (e == c.ce ? c.ced : elem_disp(P, e)) + dsc[2 * lane + 1] + skip;
+  if (w.n > 0) w.a = (int64_t)(uintptr_t)P.nc + (e == c.ce ? c.ced : elem_disp(P, e)) + ddisp + skip;
   const int64_t a0 = __shfl_sync(FULL, w.a, 0);
   const int32_t rel = (int32_t)max((int64_t)-kClamp, min((int64_t)kClamp, w.a - a0));
   int32_t rlo = w.n > 0 ? rel : INT32_MAX, rhi = w.n > 0 ? rel + w.n : INT32_MIN;

@@ -96,6 +96,11 @@ struct DeviceDesc {
   std::vector<int64_t*> tables;  // per level (nullptr for regular levels)
   // word tables for the short kernel, keyed by granularity (1,2,4,8,16)
   int32_t* wtab[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
+  // compact block descriptors of the block-span kernel (built on first use; state
+  // -1 unknown, 0 not representable, 1 built)
+  uint64_t* sdesc = nullptr;
+  int64_t* wbase = nullptr;
+  int sdesc_state = -1;
   // cached cost-balanced warp plans of the long-run kernel, keyed by the launch shape
   struct PlanSlot {
     int64_t count = -1, pos = 0, len = 0, nw = 0, alpha = 0, tsize = 0, gran = 1;
@@ -168,4 +173,7 @@ const Form& get_form(dt_type_s* t);
 // xfer.cu: identity of a communicator (direct exchange plans live beside it)
 void comm_info(dt_comm_t c, int* rank, int* nranks, int* device);
 dt_status ensure_wtab_pub(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out);
+// compact (8-byte) block descriptors for the block-span kernel, or nullptrs when a
+// block does not fit (|disp - group base| >= 2^31 or len >= 2^32)
+dt_status ensure_sdesc(const Form& f, DeviceDesc& dd, const uint64_t** sdesc, const int64_t** wbase);
 }  // namespace dt

@@ -295,6 +295,11 @@ void free_desc(DeviceDesc& dd) {
   cudaFree(dd.boff);
   for (auto* p : dd.tables) cudaFree(p);
   for (auto*& w : dd.wtab) { cudaFree(w); w = nullptr; }
+  cudaFree(dd.sdesc);
+  cudaFree(dd.wbase);
+  dd.sdesc = nullptr;
+  dd.wbase = nullptr;
+  dd.sdesc_state = -1;
   dd.bd = dd.bl = dd.boff = nullptr;
   dd.tables.clear();
   for (auto& sl : dd.plans) {
@@ -369,6 +374,44 @@ static dt_status ensure_wtab(const Form& f, DeviceDesc& dd, int64_t g, const int
 
 dt_status ensure_wtab_pub(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out) {
   return ensure_wtab(f, dd, g, out);
+}
+
+__global__ void k_build_sdesc(const int64_t* __restrict__ bd, const int64_t* __restrict__ bl, int64_t n,
+                              uint64_t* __restrict__ sdesc, int64_t* __restrict__ wbase) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t base = bd[i & ~int64_t(31)];
+    if ((i & 31) == 0) wbase[i >> 5] = base;
+    sdesc[i] = ((uint64_t)bl[i] << 32) | (uint32_t)(int32_t)(bd[i] - base);
+  }
+}
+
+dt_status ensure_sdesc(const Form& f, DeviceDesc& dd, const uint64_t** sdesc, const int64_t** wbase) {
+  if (dd.sdesc_state < 0) {
+    // representable? (host check once per descriptor, O(n))
+    const char* no = getenv("DT_NO_SDESC");  // (A/B switch)
+    bool ok = !(no && *no && *no != '0');
+    const size_t n = f.bd.size();
+    for (size_t i = 0; i < n && ok; i++) {
+      const int64_t r = f.bd[i] - f.bd[i & ~size_t(31)];
+      ok = r >= INT32_MIN && r <= INT32_MAX && f.bl[i] < (int64_t(1) << 32) && f.bl[i] >= 0;
+    }
+    dd.sdesc_state = 0;
+    if (ok && n > 1) {
+      CU(cudaMalloc(&dd.sdesc, sizeof(uint64_t) * n));
+      CU(cudaMalloc(&dd.wbase, sizeof(int64_t) * ((n + 31) / 32)));
+      const unsigned grid = (unsigned)std::min<int64_t>((int64_t)(n + 255) / 256, 4096);
+      cudaStream_t s;  // a private non-blocking stream: never waits for the caller's work
+      CU(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+      k_build_sdesc<<<grid, 256, 0, s>>>(dd.bd, dd.bl, (int64_t)n, dd.sdesc, dd.wbase);
+      CU(cudaGetLastError());
+      CU(cudaStreamSynchronize(s));  // once per committed type and device
+      CU(cudaStreamDestroy(s));
+      dd.sdesc_state = 1;
+    }
+  }
+  *sdesc = dd.sdesc_state == 1 ? dd.sdesc : nullptr;
+  *wbase = dd.sdesc_state == 1 ? dd.wbase : nullptr;
+  return DT_OK;
 }
 
 static int64_t lowp2(uint64_t x) {
@@ -786,6 +829,10 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
 #undef LS
   } else if (kind == 7) {
     P.fnb = make_fd((uint64_t)P.nblocks);
+    {
+      dt_status sst = ensure_sdesc(f, dd, &P.sdesc, &P.wbase);
+      if (sst != DT_OK) return sst;
+    }
     const size_t smem = 8 * (size_t)kSpanWarpSmem;
     bool& attr = devl().span_attr;
     if (!attr) {

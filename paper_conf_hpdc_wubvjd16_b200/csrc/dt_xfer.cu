@@ -915,7 +915,11 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
     const bool wt_ok = f.tsize() / g <= kMaxWordTable && f.tsize() % g == 0 && !E.merged;
     if ((k == 2 && wt_ok) || (k == 4 && wt_ok && g >= 8) || k == 1) X.kind = k;
   }
-  if (X.kind == 7) P.fnb = make_fd((uint64_t)P.nblocks);
+  if (X.kind == 7) {
+    P.fnb = make_fd((uint64_t)P.nblocks);
+    st = ensure_sdesc(f, *dd, &P.sdesc, &P.wbase);
+    if (st != DT_OK) return st;
+  }
   X.single = P.nblocks == 1;
   X.g = (int32_t)g;
   if (X.kind == 2 || X.kind == 4) {
