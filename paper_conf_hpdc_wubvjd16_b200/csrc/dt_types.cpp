@@ -14,6 +14,7 @@
 #include <cstdio>
 #include <cstring>
 #include <numeric>
+#include <thread>
 
 #include <sys/mman.h>
 
@@ -42,9 +43,33 @@ static void huge_reserve(std::vector<int64_t>& v, size_t n) {
   const uintptr_t e = ((uintptr_t)v.data() + bytes) & ~(uintptr_t)(hp - 1);
   if (e > a) madvise((void*)a, e - a, MADV_HUGEPAGE);
 }
+// Host threads for O(n) passes over huge index lists (first-use cost, f2): fn(lo, hi,
+// thread) over [0, n) split into equal ranges; serial below 1M entries.
+template <typename F>
+static int parallel_for(size_t n, F fn) {
+  const size_t kMin = size_t(1) << 20;
+  int nt = 1;
+  if (n >= kMin) {
+    const unsigned hw = std::thread::hardware_concurrency();
+    nt = (int)std::max(1u, std::min(16u, hw ? hw : 1u));
+    const char* e = getenv("DT_HOST_THREADS");
+    if (e && atoi(e) > 0) nt = std::min(64, atoi(e));
+  }
+  if (nt == 1) {
+    fn((size_t)0, n, 0);
+    return 1;
+  }
+  std::vector<std::thread> th;
+  for (int t = 1; t < nt; t++) th.emplace_back(fn, n * t / nt, n * (t + 1) / nt, t);
+  fn((size_t)0, n / nt, 0);
+  for (auto& x : th) x.join();
+  return nt;
+}
 static void huge_assign(std::vector<int64_t>& v, const int64_t* p, size_t n) {
   huge_reserve(v, n);
-  v.assign(p, p + n);
+  v.resize(n);
+  int64_t* d = v.data();
+  parallel_for(n, [=](size_t lo, size_t hi, int) { std::memcpy(d + lo, p + lo, (hi - lo) * sizeof(int64_t)); });
 }
 
 // ------------------------------------------------------------------ bounds
@@ -193,17 +218,32 @@ static dt_status create_hindexed(int64_t count, const int64_t* bls, int64_t ubl,
   // shifts over all copies and their number: one pass over the arrays (which also
   // validates the block lengths), before anything is allocated
   const int64_t e = old->extent();
+  struct Part {
+    int64_t smin = INT64_MAX, smax = INT64_MIN, ncopies = 0;
+    bool neg = false;
+  };
+  Part parts[64];
+  const int nt = parallel_for((size_t)count, [&](size_t i0, size_t i1, int t) {
+    Part q;
+    for (size_t i = i0; i < i1; i++) {
+      const int64_t n = bls ? bls[i] : ubl;
+      q.neg |= n < 0;
+      if (n <= 0) continue;
+      const int64_t last = (n - 1) * e;
+      const int64_t lo = dps[i] + (last < 0 ? last : 0), hi = dps[i] + (last > 0 ? last : 0);
+      q.smin = lo < q.smin ? lo : q.smin;
+      q.smax = hi > q.smax ? hi : q.smax;
+      q.ncopies += n;
+    }
+    parts[t] = q;
+  });
   int64_t smin = INT64_MAX, smax = INT64_MIN, ncopies = 0;
   bool neg = false;
-  for (int64_t i = 0; i < count; i++) {
-    const int64_t n = bls ? bls[i] : ubl;
-    neg |= n < 0;
-    if (n <= 0) continue;
-    const int64_t last = (n - 1) * e;
-    const int64_t lo = dps[i] + (last < 0 ? last : 0), hi = dps[i] + (last > 0 ? last : 0);
-    smin = lo < smin ? lo : smin;
-    smax = hi > smax ? hi : smax;
-    ncopies += n;
+  for (int t = 0; t < nt; t++) {
+    smin = std::min(smin, parts[t].smin);
+    smax = std::max(smax, parts[t].smax);
+    ncopies += parts[t].ncopies;
+    neg |= parts[t].neg;
   }
   CHECK_ARG(!neg, "negative blocklen");
   auto* t = new dt_type_s;
@@ -585,6 +625,8 @@ static Form build_form(const dt_type_s* t) {
       } else if (is_simple_run(sub, t->old->extent())) {
         // indexed of a contiguous element: one block per entry (the triangle C2, the
         // irregular list C5b), adjacent blocks merged in the same pass
+        // (one pass; host threads did not pay here: the joined ranges cost a serial copy
+        // and concurrent huge-page faults compact memory -- measured slower)
         const int64_t d0 = sub.bd[0], l0 = sub.bl[0];
         huge_reserve(f.bd, Bv.size());
         huge_reserve(f.bl, Bv.size());

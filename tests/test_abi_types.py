@@ -186,3 +186,24 @@ def test_type_serialize_roundtrip():
         with pytest.raises(dt.DTError) as e:
             dt.Type.deserialize(bad)
         assert e.value.name == "DT_ERR_ARG"
+
+
+@pytest.mark.parametrize("threads", ["1", "7"])
+def test_parallel_flatten_matches_numpy(threads, monkeypatch):
+    """f2: type construction of a huge block list runs its bounds pass and copies on
+    several host threads; the bounds and the flattened (merged) blocks must equal
+    numpy's, for any thread count."""
+    monkeypatch.setenv("DT_HOST_THREADS", threads)
+    rng = np.random.default_rng(5)
+    n = 3_000_000
+    lens = rng.integers(1, 5, size=n) * 4
+    gaps = rng.integers(0, 3, size=n) * 4  # a third of the gaps are 0: merges, also across ranges
+    d = np.concatenate([[0], np.cumsum(lens + gaps)[:-1]])
+    t = dt.Type.basic("BYTE").hindexed(lens, d)
+    bd, bl = t.flatten(1)
+    end = d + lens
+    m = np.ones(n, bool)
+    m[1:] = d[1:] != end[:-1]
+    starts = np.flatnonzero(m)
+    assert np.array_equal(bd, d[starts]) and np.array_equal(bl, np.add.reduceat(lens, starts))
+    assert t.size == int(lens.sum()) and t.true_extent == (0, int(d[-1] + lens[-1]))
