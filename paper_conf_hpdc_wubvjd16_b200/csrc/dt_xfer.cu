@@ -484,7 +484,9 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
     if (s_abort) return;
     const int64_t off = it.off();
     uint8_t* sl = X.ring + (int64_t)it.slot * X.chunk + (int64_t)it.js * it.Cs - off;  // stream byte off -> piece
-    if (X.role == 1 && X.kind == 4 && !(A.flags & 8))  // TMA bulk loads of the ring after the acquire
+    // the staged (4) and block-span (7) unpacks read the ring slot with TMA bulk loads
+    // (async proxy): order them after the control warp's generic-proxy acquire
+    if (X.role == 1 && (X.kind == 4 || X.kind == 7) && !(A.flags & 8))
       asm volatile("fence.proxy.async.global;" ::: "memory");
     if (threadIdx.x == 32 + g * kGroupThreads) xtrace(A, op, j, i, 4);
     if (X.role == 0) cta_piece<false>(X, sl, off, it.len(), wt, sbuf, mbar[g], g, tb);
@@ -1071,10 +1073,13 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   double csum = 0;
   for (int i = 0; i < nops; i++) csum += cost(A.ops[i]);
   const int total = occ * sms;
+  // every op gets the default budget when all of them fit; otherwise shares by cost
+  const bool fits = (int64_t)nops * default_ctas(c) <= total;
   int cta = 0;
   for (int i = 0; i < nops; i++) {
     XOp& X = A.ops[i];
-    const int budget = std::max(1, std::min(default_ctas(c), (int)(total * cost(X) / csum)));
+    const int budget = fits ? default_ctas(c)
+                            : std::max(1, std::min(default_ctas(c), (int)(total * cost(X) / csum)));
     // send role: one CTA per (team, piece); receive role: as many as the capacity
     // would need (the actual geometry arrives in the header; CTAs map onto it)
     const Geo G = geometry(X.n, X.chunk, X.depth, budget);
