@@ -41,6 +41,7 @@ struct Form {
   mutable int64_t gran_cache = -1, tsize_cache = -1, lvl_gran_cache = -1;
   mutable int fits32_cache = -1;
   mutable int span_local_cache = -1;  // block-span kernel: are 32-block windows locally dense?
+  mutable int sdesc_ok_cache = -1;    // do the blocks fit the compact span descriptors?
   mutable int64_t span_lo = 0, span_hi = -1;  // cached min bd / max bd+bl (span_hi < span_lo: not computed)
   void span(int64_t* lo, int64_t* hi) const {
     if (span_hi < span_lo) {
@@ -64,6 +65,7 @@ struct Form {
     gran_cache = tsize_cache = lvl_gran_cache = -1;
     fits32_cache = -1;
     span_local_cache = -1;
+    sdesc_ok_cache = -1;
     span_lo = 0;
     span_hi = -1;
     hoff_cache.clear();
@@ -138,6 +140,9 @@ struct dt_type_s {
   bool committed = false;
   std::unique_ptr<dt::Form> form;        // host form (built lazily)
   std::vector<dt::DeviceDesc> devs;      // per device uploads
+  // f2: commit deferred the flattening of a huge block list to the first whole-stream
+  // pack, which flattens, uploads and packs it in a pipeline
+  bool lazy_pipe = false;
   // overlap cache (unpack legality) for the last count checked
   int64_t ovl_count = -1;
   int ovl_result = 0;
@@ -168,6 +173,13 @@ struct Eff {
   bool merged;
 };
 Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count);
+// f2 pipelined first use (dt_types.cpp): is t an hindexed list of a contiguous element
+// with per-entry lengths (the block list flattens entry by entry)?  d0/l0: the element's
+// run.  install_form: adopt a form built outside build_form.  huge_reserve: reserve a
+// large vector on transparent huge pages.
+bool pipe_list(dt_type_s* t, int64_t* d0, int64_t* l0);
+void install_form(dt_type_s* t, Form&& f);
+void huge_reserve(std::vector<int64_t>& v, size_t n);
 dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out);
 const Form& get_form(dt_type_s* t);
 // xfer.cu: identity of a communicator (direct exchange plans live beside it)

@@ -20,6 +20,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <thread>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -80,8 +83,8 @@ __global__ void __launch_bounds__(kScanNT) k_scan_local(const int64_t* __restric
   if (threadIdx.x == 0) sums[blockIdx.x] = tot;
 }
 
-__global__ void __launch_bounds__(kScanNT) k_scan_sums(int64_t* sums, int64_t nb) {
-  int64_t carry = 0;
+__global__ void __launch_bounds__(kScanNT) k_scan_sums(int64_t* sums, int64_t nb, int64_t carry0 = 0) {
+  int64_t carry = carry0;
   for (int64_t b0 = 0; b0 < nb; b0 += kScanNT) {
     int64_t i = b0 + threadIdx.x;
     int64_t v = i < nb ? sums[i] : 0, tot;
@@ -391,9 +394,13 @@ dt_status ensure_sdesc(const Form& f, DeviceDesc& dd, const uint64_t** sdesc, co
     const char* no = getenv("DT_NO_SDESC");  // (A/B switch)
     bool ok = !(no && *no && *no != '0');
     const size_t n = f.bd.size();
-    for (size_t i = 0; i < n && ok; i++) {
-      const int64_t r = f.bd[i] - f.bd[i & ~size_t(31)];
-      ok = r >= INT32_MIN && r <= INT32_MAX && f.bl[i] < (int64_t(1) << 32) && f.bl[i] >= 0;
+    if (ok && f.sdesc_ok_cache >= 0) {
+      ok = f.sdesc_ok_cache == 1;  // (known from the flattening pass)
+    } else {
+      for (size_t i = 0; i < n && ok; i++) {
+        const int64_t r = f.bd[i] - f.bd[i & ~size_t(31)];
+        ok = r >= INT32_MIN && r <= INT32_MAX && f.bl[i] < (int64_t(1) << 32) && f.bl[i] >= 0;
+      }
     }
     dd.sdesc_state = 0;
     if (ok && n > 1) {
@@ -1012,6 +1019,204 @@ static bool host_mapped(const void* p, void** dptr) {
   return true;
 }
 
+// f2: the first whole-stream pack of a huge block list (an hindexed list of a
+// contiguous element with per-entry lengths, >= DT_PIPE_MIN entries) flattens, uploads
+// and packs it in a pipeline -- the paper's T-d2d-pipeline, DEV preparation overlapped
+// with the pack kernels ([L18:c1121]-[L18:c1649 §3.2], "almost doubling" uncached,
+// [L24:c2562 §5.1]).  A host thread flattens (merges adjacent entries) chunk by chunk into
+// the form's arrays; the calling thread uploads each finished run of blocks, scans its
+// lengths on the device with the host-known carry, and launches the block-window pack of
+// exactly that stream range on the caller's stream (waiting on the upload's event).  A
+// chunk's last block stays open until the next chunk (it may still merge).  At the end
+// the form and the device descriptor are installed as if committed normally.
+static int64_t pipe_min() {
+  const char* e = getenv("DT_PIPE_MIN");
+  return e ? atoll(e) : (int64_t(1) << 20);
+}
+
+static dt_status pipelined_first_pack(dt_type_s* t, int64_t d0, int64_t l0, const void* nc, void* c,
+                                      cudaStream_t s) {
+  const std::vector<int64_t>& B = t->bls;
+  const std::vector<int64_t>& Dv = *t->hdps;
+  const size_t n = B.size();
+  const char* ce = getenv("DT_PIPE_CHUNK");
+  const size_t chunk = ce && atoll(ce) > 0 ? (size_t)atoll(ce) : (size_t(1) << 21);
+  int dev = 0;
+  CU(cudaGetDevice(&dev));
+  Form f;
+  huge_reserve(f.bd, n);
+  huge_reserve(f.bl, n);
+  const int64_t* BD = f.bd.data();  // stable: the capacity covers every merged block
+  const int64_t* BL = f.bl.data();
+  DeviceDesc dd;
+  dd.device = dev;
+  cudaStream_t up = nullptr;
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  int64_t* sums = nullptr;
+  const size_t maxtile = (std::max(chunk, size_t(1) << 20) * 2 + kScanTile - 1) / kScanTile + 1;
+  auto fail = [&](cudaError_t e, const char* what) {
+    set_error("pipelined first pack: %s: %s", what, cudaGetErrorString(e));
+    return DT_ERR_CUDA;
+  };
+#define PU(call)                                 \
+  do {                                           \
+    cudaError_t _e = (call);                     \
+    if (_e != cudaSuccess) { st = fail(_e, #call); goto out; } \
+  } while (0)
+  std::atomic<size_t> published{0};
+  std::atomic<bool> done{false};
+  std::thread producer;
+  dt_status st = DT_OK;
+  size_t upto = 0;
+  int64_t carry = 0, s0 = 0;  // lengths of the uploaded blocks; stream bytes packed so far
+  uint64_t orr = 0;
+  int launches = 0;
+  // the facts later launches ask of the form (granularity, 32-bit template, compact span
+  // descriptors) are gathered in the same pass instead of three more passes afterwards
+  uint64_t p_or = 0;
+  int64_t p_lo = INT64_MAX, p_hi = INT64_MIN;
+  bool p_sdesc = true;
+  PU(cudaMalloc(&dd.bd, sizeof(int64_t) * n));
+  PU(cudaMalloc(&dd.bl, sizeof(int64_t) * n));
+  PU(cudaMalloc(&dd.boff, sizeof(int64_t) * n));
+  PU(cudaMalloc(&sums, sizeof(int64_t) * maxtile));
+  PU(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
+  PU(cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming));
+  PU(cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming));
+  producer = std::thread([&] {
+    for (size_t i0 = 0; i0 < n; i0 += chunk) {
+      const size_t i1 = std::min(n, i0 + chunk);
+      for (size_t i = i0; i < i1; i++) {
+        const int64_t l = B[i] * l0;
+        if (l == 0) continue;
+        const int64_t d = Dv[i] + d0;
+        if (!f.bd.empty() && f.bd.back() + f.bl.back() == d) {
+          f.bl.back() += l;
+        } else {
+          const size_t w = f.bd.size();
+          const int64_t r = d - (w & 31 ? f.bd[w & ~size_t(31)] : d);
+          p_sdesc = p_sdesc && r >= INT32_MIN && r <= INT32_MAX;
+          p_or |= (uint64_t)d;
+          p_lo = std::min(p_lo, d);
+          f.bd.push_back(d);
+          f.bl.push_back(l);
+        }
+      }
+      const size_t w = f.bd.size();
+      published.store(w > 0 ? w - 1 : 0, std::memory_order_release);  // the last block may still grow
+    }
+    for (size_t i = 0; i < f.bd.size(); i++) {  // merged lengths are final now
+      p_or |= (uint64_t)f.bl[i];
+      p_hi = std::max(p_hi, f.bd[i] + f.bl[i]);
+      p_sdesc = p_sdesc && f.bl[i] < (int64_t(1) << 32);
+    }
+    published.store(f.bd.size(), std::memory_order_release);
+    done.store(true, std::memory_order_release);
+  });
+  while (true) {
+    const bool fin = done.load(std::memory_order_acquire);
+    const size_t pub = published.load(std::memory_order_acquire);
+    if (pub == upto) {
+      if (fin) break;
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+      continue;
+    }
+    if (!fin && pub - upto < chunk / 2) {  // wait for a worthwhile batch
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+      continue;
+    }
+    const size_t m = pub - upto;
+    int64_t bsum = 0;
+    for (size_t i = upto; i < pub; i++) {
+      bsum += BL[i];
+      orr |= (uint64_t)BD[i] | (uint64_t)BL[i];  // (cumulative: a batch may start inside an earlier block)
+    }
+    // this batch packs stream bytes [s0, s1): s1 16-byte aligned (the block-window kernel
+    // stores 16-byte vectors), the last batch ends the stream
+    const int64_t s1 = fin ? carry + bsum : ((carry + bsum) & ~int64_t(15));  // (fin: pub is the final count)
+    const int64_t blen = s1 - s0;
+    PU(cudaMemcpyAsync(dd.bd + upto, BD + upto, sizeof(int64_t) * m, cudaMemcpyHostToDevice, up));
+    PU(cudaMemcpyAsync(dd.bl + upto, BL + upto, sizeof(int64_t) * m, cudaMemcpyHostToDevice, up));
+    {
+      const int64_t nt = ((int64_t)m + kScanTile - 1) / kScanTile;
+      k_scan_local<<<(unsigned)nt, kScanNT, 0, up>>>(dd.bl + upto, dd.boff + upto, sums, (int64_t)m);
+      k_scan_sums<<<1, kScanNT, 0, up>>>(sums, nt, carry);  // carry: lengths of the blocks before `upto`
+      k_scan_add<<<(unsigned)nt, kScanNT, 0, up>>>(dd.boff + upto, sums, (int64_t)m);
+      PU(cudaGetLastError());
+    }
+    PU(cudaEventRecord(ev[launches & 1], up));
+    PU(cudaStreamWaitEvent(s, ev[launches & 1], 0));
+    {
+      // block-window pack of stream bytes [carry, carry + blen): blocks [0, pub) are valid
+      KP P;
+      std::memset(&P, 0, sizeof(P));
+      P.nc = (const uint8_t*)nc;
+      P.c = (uint8_t*)c + s0;
+      P.pos = s0;
+      P.len = blen;
+      P.tsize = t->size;
+      P.nblocks = (int64_t)pub;
+      P.bd = dd.bd;
+      P.bl = dd.bl;
+      P.boff = dd.boff;
+      P.nlev = 0;
+      P.ftsize = make_fd((uint64_t)P.tsize);
+      P.fnb = make_fd((uint64_t)P.nblocks);
+      const int64_t g =
+          lowp2(orr | (uint64_t)(uintptr_t)nc | (uint64_t)(uintptr_t)c | (uint64_t)s0 | (uint64_t)blen);
+      const int sms = num_sms();
+      const int64_t max_warps = (int64_t)sms * 4 * 8;
+      int64_t nw = std::min<int64_t>(max_warps, std::max<int64_t>(1, (blen + 4095) / 4096));
+      int64_t per = (blen + nw - 1) / nw;
+      per = (per + kBlkWin - 1) / kBlkWin * kBlkWin;
+      nw = (blen + per - 1) / per;
+      P.per_warp = per;
+      const unsigned grid = (unsigned)((nw + 7) / 8);
+      const size_t smem = 8 * (kBlkWin / g) * sizeof(int64_t);
+      if (blen > 0) switch (g) {
+        case 1: k_blk<false, 1><<<grid, 256, smem, s>>>(P); break;
+        case 2: k_blk<false, 2><<<grid, 256, smem, s>>>(P); break;
+        case 4: k_blk<false, 4><<<grid, 256, smem, s>>>(P); break;
+        case 8: k_blk<false, 8><<<grid, 256, smem, s>>>(P); break;
+        default: k_blk<false, 16><<<grid, 256, smem, s>>>(P); break;
+      }
+      PU(cudaGetLastError());
+    }
+    PU(cudaStreamSynchronize(up));  // (sums is reused by the next batch)
+    carry += bsum;
+    s0 = s1;
+    upto = pub;
+    launches++;
+  }
+  if (carry != t->size || s0 != t->size) {
+    set_error("pipelined first pack: %lld of %lld bytes", (long long)s0, (long long)t->size);
+    st = DT_ERR_ARG;
+    goto out;
+  }
+out:
+  if (producer.joinable()) producer.join();
+#undef PU
+  if (sums) cudaFree(sums);
+  if (up) cudaStreamDestroy(up);
+  for (auto e : ev)
+    if (e) cudaEventDestroy(e);
+  if (st != DT_OK) {
+    free_desc(dd);
+    return st;
+  }
+  if (getenv("DT_PIPE_DEBUG")) fprintf(stderr, "[dt] pipelined first pack: %zu blocks, %d batches\n", f.bd.size(), launches);
+  f.gran_cache = std::min<int64_t>(16, lowp2(p_or));
+  f.fits32_cache = (p_lo >= INT32_MIN && p_hi <= INT32_MAX) ? 1 : 0;
+  f.sdesc_ok_cache = p_sdesc ? 1 : 0;
+  {
+    std::lock_guard<std::mutex> g(t->mu);
+    t->devs.push_back(dd);
+    t->lazy_pipe = false;
+  }
+  install_form(t, std::move(f));
+  return DT_OK;
+}
+
 static dt_status pack_common(bool unpack, dt_t t, int64_t count, const void* nc, void* c, int64_t pos, int64_t* len,
                              void* stream, bool check_ptrs = true) {
   if (!t || !len || count < 0 || pos < 0 || *len < 0) {
@@ -1035,6 +1240,12 @@ static dt_status pack_common(bool unpack, dt_t t, int64_t count, const void* nc,
     if (st != DT_OK) return st;
     st = check_dev_ptr(c, "packed");
     if (st != DT_OK) return st;
+  }
+  if (t->lazy_pipe) {  // f2: the first whole-stream pack of a huge block list, pipelined
+    int64_t d0 = 0, l0 = 0;
+    if (!unpack && count == 1 && pos == 0 && n == t->size && pipe_list(t, &d0, &l0))
+      return pipelined_first_pack(t, d0, l0, nc, c, (cudaStream_t)stream);
+    t->lazy_pipe = false;  // any other first use flattens and uploads as usual
   }
   DeviceDesc* dd = nullptr;
   dt_status st = ensure_committed_on_device(t, &dd);
@@ -1064,6 +1275,17 @@ dt_status dt_commit(dt_t t) {
   if (!t) {
     set_error("dt_commit: NULL type");
     return DT_ERR_ARG;
+  }
+  {
+    // f2: a huge block list is flattened by its first whole-stream pack, pipelined with it
+    int64_t d0, l0;
+    if (!t->committed && !t->form && t->kind == K_HINDEXED && t->count >= pipe_min() && !getenv("DT_NO_PIPE") &&
+        pipe_list(t, &d0, &l0)) {
+      t->lazy_pipe = true;
+      t->committed = true;
+      if (const char* e = getenv("DT_NOCHECK")) g_check_ptrs = (e[0] == '0');
+      return DT_OK;
+    }
   }
   try {
     get_form(t);

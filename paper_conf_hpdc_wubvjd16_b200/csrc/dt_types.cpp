@@ -35,7 +35,7 @@ static const int64_t kBasicSize[8] = {1, 1, 1, 2, 4, 8, 4, 8};
 // Reserve a large vector on transparent huge pages (first-use cost, f2): a 1 GB
 // index list has ~2e7-3e7 entries, and faulting 240 MB in 4 KiB pages costs more
 // than the flattening arithmetic itself.
-static void huge_reserve(std::vector<int64_t>& v, size_t n) {
+void huge_reserve(std::vector<int64_t>& v, size_t n) {
   v.reserve(n);
   const size_t bytes = n * sizeof(int64_t), hp = size_t(2) << 20;
   if (bytes < 4 * hp) return;
@@ -708,6 +708,21 @@ static Form build_form(const dt_type_s* t) {
     normalize(f);
   }
   return f;
+}
+
+bool pipe_list(dt_type_s* t, int64_t* d0, int64_t* l0) {
+  if (t->kind != K_HINDEXED || t->blocklen >= 0 || t->count < 2) return false;
+  Form sub = build_form(t->old);
+  normalize(sub);
+  if (!is_simple_run(sub, t->old->extent())) return false;
+  *d0 = sub.bd[0];
+  *l0 = sub.bl[0];
+  return true;
+}
+
+void install_form(dt_type_s* t, Form&& f) {
+  std::lock_guard<std::mutex> g(t->mu);
+  if (!t->form) t->form.reset(new Form(std::move(f)));
 }
 
 const Form& get_form(dt_type_s* t) {

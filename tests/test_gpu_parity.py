@@ -568,3 +568,49 @@ def test_count_or_size_zero(torch_cuda, recipe):
     check_empty(torch_cuda, recipe, 0)
     check_empty(torch_cuda, recipe, 0, nbytes=0)
     check_empty(torch_cuda, recipe, 2, pos=1 << 20)
+
+
+# ------------------------------------------------------------------ f2: pipelined first use
+@pytest.mark.parametrize("first", ["pack", "unpack"])
+@pytest.mark.parametrize("seed", [0, 1])
+def test_pipelined_first_pack(torch_cuda, first, seed, monkeypatch):
+    """f2: a huge irregular block list is flattened by its first whole-stream pack, in
+    chunks pipelined with uploads, device scans and block-window packs of each
+    finished range ([L18:c1121]-[L18:c1649 §3.2]).  Small thresholds force it on a
+    120k-entry list with many zero gaps (merges across chunk boundaries, batches that
+    end inside a block); the stream must equal the oracle's, the cached second pack
+    too, and an unpack as first use must take the ordinary path."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    monkeypatch.setenv("DT_PIPE_MIN", "1000")
+    monkeypatch.setenv("DT_PIPE_CHUNK", "7001")
+    rng = np.random.default_rng(40 + seed)
+    n = 120_000
+    lens = rng.integers(1, 17, size=n) * (4 if seed == 0 else 1)
+    gaps = rng.integers(0, 4, size=n) * (4 if seed == 0 else 3)
+    d = np.concatenate([[0], np.cumsum(lens + gaps)[:-1]]) + 64
+    rec = ("hindexed", lens, d, ("basic", "BYTE"))
+    parent = int(d[-1] + lens[-1] + 128)
+    org = seed * 3  # misaligned origin for seed 1
+    ot = oracle.from_recipe(rec)
+    src_h = fill_bytes(parent + 16, 77 + seed)
+    exp = oracle.pack(ot, 1, src_h, org)
+    t = dt.from_recipe(rec).commit()
+    src = _dev(torch, src_h)
+    out = _poisoned(torch, len(exp))
+    if first == "unpack":
+        dst = torch.full((parent + 16,), 0xA5, dtype=torch.uint8, device="cuda")
+        dt.unpack(t, 1, _dev(torch, exp), dst, origin_offset=org)
+        ref = np.full(parent + 16, 0xA5, dtype=np.uint8)
+        oracle.unpack(ot, 1, exp, ref, org)
+        torch.cuda.synchronize()
+        assert np.array_equal(dst.cpu().numpy(), ref)
+    for _ in range(2):  # first (pipelined when `first` is pack) and cached
+        dt.pack(t, 1, src, out.data_ptr() + GUARD, origin_offset=org)
+        torch.cuda.synchronize()
+        o = out.cpu().numpy()
+        assert np.all(o[:GUARD] == 0xA5) and np.all(o[GUARD + len(exp):] == 0xA5)
+        assert np.array_equal(o[GUARD:GUARD + len(exp)], exp)
+    # the installed form is the ordinary one
+    bd, bl = t.flatten(1)
+    assert int(bl.sum()) == len(exp)
