@@ -552,3 +552,66 @@ def test_ring_replicas(torch_cuda, rep, depth, monkeypatch):
     rec5, org5, parent5 = c5_particles(3 << 20)
     _loop_check(torch_cuda, comm, rec5, org5, parent5, rec5, org5, parent5, seed=7)
     comm.free()
+
+
+@pytest.mark.parametrize("chunk", [1 << 20, 4 << 20])
+def test_full_size_c3_exchange_sampled(torch_cuda, chunk):
+    """BASELINE configs C3 at full size in the launch configuration the bench times
+    (8192^2 f64, nb 64, 128 MiB per direction, auto depth, 1 and 4 MiB fragments):
+    sampled received bytes against the oracle's per-position addresses, gap bytes of the
+    receive layout untouched, repeated exchanges on the same channel."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c3_block_cyclic(8192, 64)
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=0, ring_loopback=True)
+    src_h = fill_bytes(parent, 0x5EED0003)
+    A = torch.from_numpy(src_h).cuda()
+    B = torch.full((parent,), 0xA5, dtype=torch.uint8, device="cuda")
+    for _ in range(3):
+        comm.sendrecv(A, 1, t, 0, B, 1, t, 0, sbuf_offset=org, rbuf_offset=org)
+    torch.cuda.synchronize()
+    comm.check()
+    rng = np.random.default_rng(3)
+    n = ot.size
+    ps = np.unique(np.concatenate([rng.integers(0, n, size=300000), [0, n - 1]]))
+    addr = org + oracle.addr_of(ot, 1, ps)
+    got = B[torch.from_numpy(addr).cuda()].cpu().numpy()
+    assert np.array_equal(got, src_h[addr])
+    # bytes outside the typemap: the other processes' blocks of the block-cyclic layout
+    # (rows nb..2nb of each owned column) keep their poison
+    gaps = org + np.arange(64) * 8 + 64 * 8
+    assert np.all(B[torch.from_numpy(gaps).cuda()].cpu().numpy() == 0xA5)
+    comm.free()
+
+
+def test_full_size_c4_halo_ring(torch_cuda):
+    """C4 at full size (512^3 f32 per rank, ghost width 1, periodic on one GPU), all 12
+    transfers through the ring group as the bench times them: every ghost cell equals
+    the periodic neighbour's interior value (closed form), the interior is untouched."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from paper_conf_hpdc_wubvjd16_b200.halo import make_plan
+    n, h = 512, 1
+    L = n + 2 * h
+    comm = dt.Comm(0, 1, 0, chunk_bytes=1 << 20, depth=0, ring_loopback=True)
+    plan = make_plan(0, n, h, dims=(1, 1, 1))
+    buf = torch.empty(L ** 3 * 4, dtype=torch.uint8, device="cuda")
+    A = buf.view(torch.int32).view(L, L, L)
+    A.random_(0, 1 << 30)
+    before = A[h:h + n, h:h + n, h:h + n].clone()
+    for _ in range(2):
+        plan.exchange(comm, buf)
+    torch.cuda.synchronize()
+    comm.check()
+    assert torch.equal(A[h:h + n, h:h + n, 0], A[h:h + n, h:h + n, n])          # x- ghost = x+ boundary
+    assert torch.equal(A[h:h + n, h:h + n, L - 1], A[h:h + n, h:h + n, h])      # x+ ghost = x- boundary
+    assert torch.equal(A[h:h + n, 0, h:h + n], A[h:h + n, n, h:h + n])
+    assert torch.equal(A[h:h + n, L - 1, h:h + n], A[h:h + n, h, h:h + n])
+    assert torch.equal(A[0, h:h + n, h:h + n], A[n, h:h + n, h:h + n])
+    assert torch.equal(A[L - 1, h:h + n, h:h + n], A[h, h:h + n, h:h + n])
+    assert torch.equal(A[h:h + n, h:h + n, h:h + n], before)
+    comm.free()
