@@ -28,6 +28,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <cstddef>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -74,25 +75,33 @@ struct XOp {
   uint64_t* ack;   // [depth][kMaxSub] tags  send: local; recv: peer
   uint64_t* hdr;   // [4] {seq, nbytes, gs, rep}  send: peer; recv: local
   uint64_t* go;    // [2] {consumed seq, aborted seq}  send: local; recv: peer
-  uint32_t* done;  // recv: local counter of CTAs finished with the message (last one posts consumed)
-  uint64_t seq;
+  uint32_t* done;  // local counter of this op's CTAs finished with the message (the last one
+                   // advances *seqp and, receiving, posts consumed)
+  uint64_t* seqp;  // local: the channel's last message sequence number in this role (device-
+                   // resident, so a captured CUDA graph replays with fresh numbers)
   int32_t* err;
   RecGeo rg;       // kind 6: record-span geometry (per-fragment element range set on the device)
 };
 
-struct XArgs {
+// Kernel parameters: NOPS ops (a single dt_sendrecv has <= 2; a group up to kMaxOps).
+// Each XOp is ~700 bytes, and the kernel parameters travel with every launch: the
+// 2-op instantiation keeps a single exchange's launch small.
+template <int NOPS>
+struct XArgsT {
   int32_t nops;
   int32_t wt_off;  // byte offset of the word table in dynamic smem (after the staging buffers)
   int32_t flags;   // DT_XFER_FLAGS: bit1 = no sleep in polls, bit2 = SC system fence before each flag
   int32_t pad2;
   int64_t timeout_ns;
   uint64_t* trace;  // diagnostics (DT_XFER_TRACE): per-piece globaltimer stamps of the first CTAs
-  XOp ops[kMaxOps];
+  XOp ops[NOPS];
 };
+typedef XArgsT<kMaxOps> XArgs;
 constexpr int kTraceCtas = 4, kTracePieces = 64, kTracePts = 6;
 // points: 0 control starts waiting for the piece's flag, 1 flag acquired, 2 copy seen
 // done, 3 flag released, 4 copy group starts the piece, 5 copy group done
-__device__ __forceinline__ void xtrace(const XArgs& A, int op, int j, int idx, int point) {
+template <int NOPS>
+__device__ __forceinline__ void xtrace(const XArgsT<NOPS>& A, int op, int j, int idx, int point) {
   if (A.trace && j < kTraceCtas && idx < kTracePieces)
     *(volatile uint64_t*)&A.trace[(((size_t)op * kTraceCtas + j) * kTracePieces + idx) * kTracePts + point] = gtimer();
 }
@@ -297,20 +306,23 @@ struct PieceIt {
 //    never read; the next message's tags supersede their flags).
 // Flags are written by exactly one CTA, so plain release stores suffice, and since
 // tags only grow nothing is carried between messages.
-// Receiver CTA finished its part of message seq (every piece it owns unpacked and
-// acked, by this thread): the last CTA of the op posts "consumed = seq" to the
-// sender -- the ring is free for the next message on the channel.
-__device__ __forceinline__ void recv_done(const XOp& X, uint64_t seq, bool sys) {
-  __threadfence();  // this CTA's reads of the ring are complete (their values were stored)
+// A CTA finished its part of message seq (every piece it owns copied and its flags
+// released, by this thread).  The last CTA of the op advances the channel's device-
+// resident sequence number and, receiving, posts "consumed = seq" to the sender --
+// the ring is free for the next message on the channel.
+__device__ __forceinline__ void op_done(const XOp& X, uint64_t seq, bool sys) {
+  __threadfence();  // this CTA's accesses to the ring are complete (their values were used)
   const uint32_t old = atomicAdd(X.done, 1u);
   if (old + 1 == (uint32_t)X.ncta) {
     atomicExch(X.done, 0u);
+    *(volatile uint64_t*)X.seqp = seq;  // read by the next kernel on the stream
     __threadfence();
-    st_release(X.go, seq, sys);
+    if (X.role == 1) st_release(X.go, seq, sys);
   }
 }
 
-__global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgs A) {
+template <int NOPS>
+__global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant__ XArgsT<NOPS> A) {
   // dynamic smem: [staging buffers / record or span buffers] [word table]
   extern __shared__ __align__(128) uint8_t xsm[];
   __shared__ __align__(8) uint64_t mbar[kGroups][kXferStageBufs];
@@ -339,7 +351,9 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
                      default: rec_maps<false, 16>(R, omap); break; }
     }
   }
-  const uint64_t seq = X.seq;
+  // every CTA of the op reads the same number: it is advanced only after all of them
+  // have counted themselves done (op_done)
+  const uint64_t seq = *(volatile const uint64_t*)X.seqp + 1;
   const bool sys = X.sys != 0;
   if (threadIdx.x == 0) {
     xtrace(A, op, j, kTracePieces - 1, 1);  // setup done
@@ -375,7 +389,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   }
   __syncthreads();
   if (s_stop) {
-    if (X.role == 1 && threadIdx.x == 0) recv_done(X, seq, sys);
+    if (threadIdx.x == 0) op_done(X, seq, sys);
     return;
   }
   const int64_t n = (int64_t)s_n;
@@ -453,6 +467,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
         __threadfence_block();
         mbar_arrive(full + 0);
         mbar_arrive(full + 1);
+        op_done(X, seq, sys);
         return;
       }
       if (sleep_ok) __nanosleep(ns);
@@ -468,11 +483,12 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
         // these arrivals or by the one below.
         mbar_arrive(full + 0);
         mbar_arrive(full + 1);
+        op_done(X, seq, sys);
         return;
       }
     }
     xtrace(A, op, j, kTracePieces - 1, 3);  // control loop done
-    if (X.role == 1) recv_done(X, seq, sys);
+    op_done(X, seq, sys);
     return;
   }
   // ---- copy groups: group g takes the CTA's pieces g, g + 2, g + 4, ...
@@ -583,7 +599,9 @@ struct dt_comm_s {
   std::vector<bool> opened;
   std::vector<int> same_dev;  // peer runs on this physical GPU: gpu-scope flags suffice
   bool connected = false;
-  std::vector<uint64_t> send_seq, recv_seq;  // [nranks*nch]
+  // device-resident per-(role, peer, channel) sequence numbers and CTA counters (local)
+  uint64_t* dseq = nullptr;   // [2][nranks][nch]
+  uint32_t* ddone = nullptr;  // [2][nranks][nch]
   // group
   bool in_group = false;
   std::vector<PendingOp> pending;
@@ -709,9 +727,16 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
     e = cudaMalloc(&c->ring, c->ring_bytes);
     if (e == cudaSuccess) e = cudaMalloc(&c->flags, c->flag_words * 8);
     if (e == cudaSuccess) e = cudaMemset(c->flags, 0, c->flag_words * 8);
+    const size_t nq = (size_t)2 * nranks * c->nch;
+    if (e == cudaSuccess) e = cudaMalloc(&c->dseq, nq * 8);
+    if (e == cudaSuccess) e = cudaMemset(c->dseq, 0, nq * 8);
+    if (e == cudaSuccess) e = cudaMalloc(&c->ddone, nq * 4);
+    if (e == cudaSuccess) e = cudaMemset(c->ddone, 0, nq * 4);
     if (e != cudaSuccess) {
       cudaFree(c->ring);
       cudaFree(c->flags);
+      cudaFree(c->dseq);
+      cudaFree(c->ddone);
       delete c;
       return cufail(e, "dt_comm_init alloc");
     }
@@ -754,8 +779,7 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
   c->opened.assign(nranks, false);
   c->same_dev.assign(nranks, 0);
   c->same_dev[rank] = !getenv("DT_XFER_SYS");  // DT_XFER_SYS: system-scope flags even on one GPU
-  c->send_seq.assign((size_t)nranks * c->nch, 0);
-  c->recv_seq.assign((size_t)nranks * c->nch, 0);
+
   c->peer_ring[rank] = c->ring;
   c->peer_flags[rank] = c->flags;
   if (nranks == 1 || c->o.mode == DT_XFER_NCCL) c->connected = true;
@@ -1009,7 +1033,8 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.hdr = pf + c->hdr_idx(c->rank, ch);
       X.ack = c->flags + c->ack_idx(p.dest, ch);
       X.go = c->flags + c->go_idx(p.dest, ch);
-      X.seq = ++c->send_seq[(size_t)p.dest * c->nch + ch];
+      X.seqp = c->dseq + ((size_t)0 * c->nranks + p.dest) * c->nch + ch;
+      X.done = c->ddone + ((size_t)0 * c->nranks + p.dest) * c->nch + ch;
       X.sys = !c->same_dev[p.dest];
       // a peer on another GPU: the staged family's TMA bulk stores would target peer
       // memory, never exercised on a one-GPU lease -- use the word-table family's
@@ -1032,8 +1057,8 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.hdr = c->flags + c->hdr_idx(p.source, ch);
       X.ack = pf + c->ack_idx(c->rank, ch);
       X.go = pf + c->go_idx(c->rank, ch);
-      X.done = reinterpret_cast<uint32_t*>(c->flags + c->done_idx(p.source, ch));
-      X.seq = ++c->recv_seq[(size_t)p.source * c->nch + ch];
+      X.seqp = c->dseq + ((size_t)1 * c->nranks + p.source) * c->nch + ch;
+      X.done = c->ddone + ((size_t)1 * c->nranks + p.source) * c->nch + ch;
       X.sys = !c->same_dev[p.source];
     }
   }
@@ -1053,10 +1078,11 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
                                        (rec_smem + 127) & ~size_t(127));
   smem += (size_t)A.wt_off;
   // the attribute is per device (a process may drive several)
-  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(k_xfer, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const void* kfn = nops <= 2 ? (const void*)k_xfer<2> : (const void*)k_xfer<kMaxOps>;
+  if (smem > 48 * 1024) CU(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // every CTA must be co-resident: fit the per-op CTA budget to the occupancy
   int occ = 0;
-  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_xfer, kXferThreads, smem));
+  CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kfn, kXferThreads, smem));
   int sms = 0, dev = 0;
   CU(cudaGetDevice(&dev));
   CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
@@ -1106,8 +1132,14 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   // every CTA of both roles must be co-resident (they wait on each other): cooperative launch
   void* args[] = {&A};
   static const bool coop = !getenv("DT_XFER_NOCOOP");
-  if (coop) CU(cudaLaunchCooperativeKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
-  else CU(cudaLaunchKernel((void*)k_xfer, dim3(cta), dim3(kXferThreads), args, smem, s));
+  XArgsT<2> A2;  // a single exchange: the small parameter block
+  if (nops <= 2) {
+    std::memcpy(&A2, &A, offsetof(XArgs, ops));
+    std::memcpy(A2.ops, A.ops, sizeof(XOp) * 2);
+    args[0] = &A2;
+  }
+  if (coop) CU(cudaLaunchCooperativeKernel(kfn, dim3(cta), dim3(kXferThreads), args, smem, s));
+  else CU(cudaLaunchKernel(kfn, dim3(cta), dim3(kXferThreads), args, smem, s));
   if (tr) {
     bool hung = false;
     for (int w = 0; cudaStreamQuery(s) == cudaErrorNotReady; w++) {
@@ -1354,6 +1386,8 @@ dt_status dt_comm_free(dt_comm_t* pc) {
   }
   cudaFree(c->ring);
   cudaFree(c->flags);
+  cudaFree(c->dseq);
+  cudaFree(c->ddone);
   cudaFree(c->stage);
   cudaFree(c->rstage);
   cudaFree(c->szbuf);

@@ -615,3 +615,43 @@ def test_full_size_c4_halo_ring(torch_cuda):
     assert torch.equal(A[L - 1, h:h + n, h:h + n], A[h, h:h + n, h:h + n])
     assert torch.equal(A[h:h + n, h:h + n, h:h + n], before)
     comm.free()
+
+
+def test_ring_exchange_graph_replay(torch_cuda):
+    """Sequence numbers live on the device, so ring exchanges captured once in a CUDA
+    graph replay correctly: every replay moves the current source bytes (the paper's
+    persistent exchange of a halo/stencil loop without per-message host work)."""
+    import torch
+
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c3_block_cyclic(2048, 64)
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    v = dt.Type.basic("INT32").contiguous(1000).commit()
+    comm = dt.Comm(0, 1, 0, chunk_bytes=256 << 10, depth=0, ring_loopback=True)
+    A = torch.zeros(parent, dtype=torch.uint8, device="cuda")
+    B = torch.full((parent,), 0xA5, dtype=torch.uint8, device="cuda")
+    a2 = torch.zeros(4000, dtype=torch.uint8, device="cuda")
+    b2 = torch.zeros(4000, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        for _ in range(2):  # warm up: descriptors, word tables, attributes
+            comm.sendrecv(A, 1, t, 0, B, 1, t, 0, sbuf_offset=org, rbuf_offset=org, stream=s)
+            comm.sendrecv(a2, 1, v, 0, b2, 1, v, 0, stream=s)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        comm.sendrecv(A, 1, t, 0, B, 1, t, 0, sbuf_offset=org, rbuf_offset=org, stream=s)
+        comm.sendrecv(a2, 1, v, 0, b2, 1, v, 0, stream=s)
+    for r in range(4):
+        src_h = fill_bytes(parent, 100 + r)
+        A.copy_(torch.from_numpy(src_h))
+        a2.copy_(torch.from_numpy(fill_bytes(4000, 200 + r)))
+        g.replay()
+        torch.cuda.synchronize()
+        comm.check()
+        exp_b = B.cpu().numpy().copy()
+        oracle.sendrecv(ot, 1, src_h, ot, 1, exp_b, org, org)
+        assert np.array_equal(B.cpu().numpy(), exp_b), r
+        assert torch.equal(b2, a2), r
+    comm.free()

@@ -19,7 +19,8 @@ def main():
     units = os.environ.get("LAT_UNITS", "BYTE,V16").split(",")
     src = torch.empty(max(sizes), dtype=torch.uint8, device="cuda").random_(0, 255)
     dst = torch.zeros_like(src)
-    s = torch.cuda.current_stream()
+    s = torch.cuda.Stream()
+    torch.cuda.set_stream(s)
     N = 50
     for unit in units:
         b = dt.Type.basic("BYTE").commit() if unit == "BYTE" else dt.Type.basic("INT64").contiguous(2).commit()
@@ -43,8 +44,25 @@ def main():
                 torch.cuda.synchronize()
                 comm.check()
                 assert torch.equal(dst[:n], src[:n])
-                row[f"{n >> 10}K"] = (round(e0.elapsed_time(e1) / N * 1e3, 1), round(host_us, 1))
-            print(f"unit={unit} chunk={chunk >> 10}K depth={depth or 'auto'} (gpu us, host us)/msg:", row, flush=True)
+                # the same messages captured once in a CUDA graph and replayed (device-resident
+                # sequence numbers): no per-call host work, no per-launch CPU->GPU submission
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=s):
+                    for _ in range(N):
+                        one()
+                g.replay()
+                torch.cuda.synchronize()
+                g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                g0.record(s)
+                g.replay()
+                g1.record(s)
+                torch.cuda.synchronize()
+                comm.check()
+                row[f"{n >> 10}K"] = (round(e0.elapsed_time(e1) / N * 1e3, 1), round(host_us, 1),
+                                      round(g0.elapsed_time(g1) / N * 1e3, 1))
+                del g
+            print(f"unit={unit} chunk={chunk >> 10}K depth={depth or 'auto'} (gpu us, host us, graph-replay us)/msg:",
+                  row, flush=True)
             comm.free()
 
 
