@@ -42,8 +42,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     os.makedirs(LIBDIR, exist_ok=True)
     objs, cmds = [], []
+    headers = [p for p in _deps() if not p.endswith((".cu", ".cpp"))]
+    flags_file = os.path.join(LIBDIR, "flags.txt")
+    flags = os.environ.get("DT_NVCC_FLAGS", "") + "|" + os.environ.get("DT_PTXAS_V", "")
+    same_flags = os.path.exists(flags_file) and open(flags_file).read() == flags
     for src in _sources():
         obj = os.path.join(LIBDIR, os.path.basename(src) + ".o")
+        objs.append(obj)
+        # per-object rebuild: its source, any header or this script newer than the object
+        if (not force and same_flags and os.path.exists(obj)
+                and all(os.path.getmtime(p) <= os.path.getmtime(obj) for p in [src, *headers])):
+            continue
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
                "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
         if src.endswith(".cpp"):
@@ -55,11 +64,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
         cmds.append(cmd)
-        objs.append(obj)
     # translation units are independent: compile them concurrently
     from concurrent.futures import ThreadPoolExecutor
     with ThreadPoolExecutor(max_workers=len(cmds) or 1) as ex:
         list(ex.map(subprocess.check_call, cmds))
+    with open(flags_file, "w") as fh:
+        fh.write(flags)
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-ldl", "-lpthread", "-lrt"]
     if verbose:

@@ -43,6 +43,16 @@ struct Form {
   mutable int span_local_cache = -1;  // block-span kernel: are 32-block windows locally dense?
   mutable int sdesc_ok_cache = -1;    // do the blocks fit the compact span descriptors?
   mutable int64_t span_lo = 0, span_hi = -1;  // cached min bd / max bd+bl (span_hi < span_lo: not computed)
+  // f2 GPU-side flattening: the merged block list was built on the device and the host
+  // arrays bd/bl stay empty until a host consumer asks for them (materialize_host);
+  // nb_dev blocks, the first block (bd0_dev, bl0_dev), and whether the blocks are sorted
+  // and disjoint (mono_dev, the unpack legality fact) come from the device pass
+  int64_t nb_dev = -1, bd0_dev = 0, bl0_dev = 0;
+  int mono_dev = -1;
+  bool host_missing() const { return nb_dev >= 0; }  // (materialize_host resets nb_dev to -1)
+  int64_t nblocks() const { return host_missing() ? nb_dev : (int64_t)bl.size(); }
+  int64_t first_bd() const { return host_missing() ? bd0_dev : bd.empty() ? 0 : bd[0]; }
+  int64_t first_bl() const { return host_missing() ? bl0_dev : bl.empty() ? 0 : bl[0]; }
   void span(int64_t* lo, int64_t* hi) const {
     if (span_hi < span_lo) {
       int64_t a = INT64_MAX, b = INT64_MIN;
@@ -62,6 +72,7 @@ struct Form {
   }
   mutable std::vector<int64_t> hoff_cache;  // host exclusive prefix of bl (launch planning)
   void invalidate() const {
+    if (host_missing()) return;  // (device facts stay: the device form is never edited)
     gran_cache = tsize_cache = lvl_gran_cache = -1;
     fits32_cache = -1;
     span_local_cache = -1;
@@ -79,10 +90,14 @@ struct Form {
     return hoff_cache;
   }
   int64_t nelem() const { int64_t n = 1; for (auto& l : lv) n *= l.cnt; return n; }
-  bool empty() const { return bl.empty(); }
+  bool empty() const { return nblocks() == 0; }
 };
 
 void normalize(Form& f);
+struct DeviceDesc;
+// f2: download a device-flattened form's block list into its host arrays (no-op when
+// present); dd: a descriptor holding it
+dt_status materialize_host(const Form& f, const DeviceDesc& dd);
 // Expand into merged blocks (typemap order).  Returns false if > cap.
 bool expand(const Form& f, std::vector<int64_t>& d, std::vector<int64_t>& l, int64_t cap);
 int64_t form_granularity(const Form& f);

@@ -26,6 +26,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <climits>
 
 #include "dt_device.cuh"
 #include "dt_internal.h"
@@ -363,6 +364,10 @@ dt_status upload_desc(dt_type_s* t, const Form& f, DeviceDesc& dd) {
 static dt_status ensure_wtab(const Form& f, DeviceDesc& dd, int64_t g, const int32_t** out) {
   int li = log2_small(g);
   if (!dd.wtab[li]) {
+    if (f.host_missing()) {
+      dt_status ms = materialize_host(f, dd);
+      if (ms != DT_OK) return ms;
+    }
     const int64_t nw = f.tsize() / g;
     std::vector<int32_t> h((size_t)nw);
     int64_t k = 0;
@@ -393,7 +398,7 @@ dt_status ensure_sdesc(const Form& f, DeviceDesc& dd, const uint64_t** sdesc, co
     // representable? (host check once per descriptor, O(n))
     const char* no = getenv("DT_NO_SDESC");  // (A/B switch)
     bool ok = !(no && *no && *no != '0');
-    const size_t n = f.bd.size();
+    const size_t n = (size_t)f.nblocks();
     if (ok && f.sdesc_ok_cache >= 0) {
       ok = f.sdesc_ok_cache == 1;  // (known from the flattening pass)
     } else {
@@ -459,6 +464,7 @@ void build_levels(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t cou
 
 static bool template_fits_int32(const Form& f) {
   if (f.fits32_cache >= 0) return f.fits32_cache == 1;
+  if (f.host_missing()) return false;  // (device forms carry the fact)
   f.fits32_cache = 0;
   for (size_t b = 0; b < f.bd.size(); b++)
     if (f.bd[b] < INT32_MIN || f.bd[b] + f.bl[b] > INT32_MAX) return false;
@@ -473,9 +479,9 @@ Eff effective(const Form& f, const DeviceDesc* dd, dt_type_s* t, int64_t count) 
   Eff E;
   build_levels(f, dd, t, count, E.L);
   E.tsize = f.tsize();
-  E.nblocks = (int64_t)f.bl.size();
-  E.bd0 = f.bd.empty() ? 0 : f.bd[0];
-  E.bl0 = f.bl.empty() ? 0 : f.bl[0];
+  E.nblocks = f.nblocks();
+  E.bd0 = f.first_bd();
+  E.bl0 = f.first_bl();
   E.merged = false;
   KLevels& L = E.L;
   while (E.nblocks == 1 && L.n >= 1 && !L.table[L.n - 1] && L.stride[L.n - 1] == E.bl0 &&
@@ -538,6 +544,10 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
   sl.count = -1;
   CU(cudaMalloc(&sl.d, sizeof(PlanEnt) * (size_t)(nw + 1)));
   const int64_t ce = P.tsize + alpha * P.nblocks;
+  if (f.host_missing() && P.nblocks > 1 && (P.pos % P.tsize || (P.pos + P.len) % P.tsize)) {
+    dt_status ms = materialize_host(f, dd);  // (host_cost needs the block prefix)
+    if (ms != DT_OK) return ms;
+  }
   const int64_t C0 = host_cost(P, f, alpha, P.pos), C1 = host_cost(P, f, alpha, P.pos + P.len);
   k_plan<<<(unsigned)((nw + 1 + 255) / 256), 256, 0, s>>>(P, alpha, make_fd((uint64_t)ce), ce, C0, C1, nw,
                                                           gran, (PlanEnt*)sl.d);
@@ -561,13 +571,13 @@ static dt_status get_plan(dt_type_s* t, const KP& P, const Form& f, DeviceDesc& 
 // 16-byte-aligned span of <= 128 B that is at least half payload.
 bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
                   int64_t g, RecGeo* R) {
-  if (g < 4 || f.bl.empty() || len <= 0) return false;
+  if (g < 4 || f.empty() || len <= 0) return false;
   if ((nc_addr & 15) || ((c_addr - (uint64_t)pos) & 15)) return false;
   int64_t lg = level_granularity(f);
   for (int i = 0; i < L.n; i++)
     if (!L.table[i]) lg = std::min(lg, lowp2((uint64_t)L.stride[i]));
   if (lg < 16) return false;
-  if (f.bl.size() > 64) return false;  // (a <= 128-byte span holds few blocks; keeps planning O(1))
+  if (f.nblocks() > 64) return false;  // (a <= 128-byte span holds few blocks; keeps planning O(1))
   int64_t lo, hi;
   f.span(&lo, &hi);
   const int64_t a0 = lo >= 0 ? lo & ~int64_t(15) : -((-lo + 15) & ~int64_t(15));
@@ -603,6 +613,7 @@ bool rec_geometry(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_
 // of the innermost level (its stride, or consecutive entries of its table).
 static bool span_local(const Form& f) {
   if (f.span_local_cache >= 0) return f.span_local_cache != 0;
+  if (f.host_missing()) return false;  // (device forms carry the fact)
   const int64_t nb = (int64_t)f.bl.size();
   constexpr int64_t kBuf = 4 * 4096;
   int good = 0, tot = 0;
@@ -648,8 +659,8 @@ static bool span_local(const Form& f) {
 
 int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_addr, int64_t pos, int64_t len,
                 int64_t* gran) {
-  if (len <= 0 || f.bl.empty()) return 0;
-  const int64_t nb = (int64_t)f.bl.size();
+  if (len <= 0 || f.empty()) return 0;
+  const int64_t nb = f.nblocks();
   const int64_t ts = f.tsize();
   int64_t g = form_granularity(f);
   for (int i = 0; i < L.n; i++)
@@ -918,6 +929,10 @@ dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out) {
   std::lock_guard<std::mutex> g(t->mu);
   for (auto& dd : t->devs)
     if (dd.device == dev) { *out = &dd; return DT_OK; }
+  if (f.host_missing()) {  // device-flattened on another device: its host arrays first
+    dt_status ms = t->devs.empty() ? DT_ERR_ARG : materialize_host(f, t->devs[0]);
+    if (ms != DT_OK) return ms;
+  }
   t->devs.emplace_back();
   DeviceDesc& dd = t->devs.back();
   dd.device = dev;
@@ -931,19 +946,27 @@ dt_status ensure_committed_on_device(dt_type_s* t, DeviceDesc** out) {
   return DT_OK;
 }
 
+static dt_status materialize_t(dt_type_s* t, const Form& f);
+
 // Unpack legality (reading A9): the typemap of `count` instances must not
 // overlap.  Cheap structural proof first, exact sorted-interval check if needed.
 static int check_nonoverlap(dt_type_s* t, const Form& f, int64_t count) {
-  if (f.bl.empty() || count == 0) return 1;
-  // template: sorted intervals
+  if (f.empty() || count == 0) return 1;
   std::vector<std::pair<int64_t, int64_t>> iv;
-  iv.reserve(f.bl.size());
-  for (size_t i = 0; i < f.bl.size(); i++) iv.push_back({f.bd[i], f.bd[i] + f.bl[i]});
-  std::sort(iv.begin(), iv.end());
-  for (size_t i = 1; i < iv.size(); i++)
-    if (iv[i].first < iv[i - 1].second) return 0;
-  int64_t lo = iv.front().first, hi = 0;
-  for (auto& x : iv) hi = std::max(hi, x.second);
+  int64_t lo = 0, hi = 0;
+  if (f.host_missing() && f.mono_dev == 1) {
+    f.span(&lo, &hi);  // device form: the flattening pass proved the blocks sorted and disjoint
+  } else {
+    if (materialize_t(t, f) != DT_OK) return -1;
+    // template: sorted intervals
+    iv.reserve(f.bl.size());
+    for (size_t i = 0; i < f.bl.size(); i++) iv.push_back({f.bd[i], f.bd[i] + f.bl[i]});
+    std::sort(iv.begin(), iv.end());
+    for (size_t i = 1; i < iv.size(); i++)
+      if (iv[i].first < iv[i - 1].second) return 0;
+    lo = iv.front().first;
+    for (auto& x : iv) hi = std::max(hi, x.second);
+  }
   bool proven = true;
   auto level = [&](int64_t cnt, int64_t stride, const std::vector<int64_t>* tab) {
     if (!proven || cnt <= 1) return;
@@ -972,6 +995,7 @@ static int check_nonoverlap(dt_type_s* t, const Form& f, int64_t count) {
   for (int i = (int)f.lv.size() - 1; i >= 0; i--) level(f.lv[i].cnt, f.lv[i].stride, f.lv[i].table.get());
   level(count, t->extent(), nullptr);
   if (proven) return 1;
+  if (materialize_t(t, f) != DT_OK) return -1;
   // exact check on the expanded list
   Form g = f;
   if (count > 1) {
@@ -1017,6 +1041,317 @@ static bool host_mapped(const void* p, void** dptr) {
   if (a.type != cudaMemoryTypeHost || !a.devicePointer) return false;
   *dptr = a.devicePointer;
   return true;
+}
+
+// ------------------------------------------------------- f2: GPU-side flattening
+// A huge block list -- an hindexed list of a contiguous element (d0, l0) with per-entry
+// counts, the C5b shape -- is flattened ON THE DEVICE at commit (the
+// paper prepares its DEV lists on the CPU and pipelines that with the kernels,
+// [L18:c1121]-[L18:c1649 §3.2]; here the preparation itself moves to the GPU).  Only the
+// raw entry arrays cross the host link; four passes build what the host flattening
+// builds -- entry i opens a new block unless it starts where entry i-1 ends (adjacent
+// blocks merged, the DEV list of [L16:c5201 §3.2] in typemap order) -- plus the stream
+// prefix boff, the compact span descriptors and every fact launch planning asks of the
+// form (granularity, span, 32-bit fit, sorted-disjoint, window locality).
+//   k_flat_tiles  per 1024-entry tile: sum of lengths, number of block heads, zero count
+//   k_scan_sums   exclusive scans of the tile sums (lengths; heads) -> tile offsets
+//   k_flat_emit   re-derives each entry's (length, head) and its in-tile prefix; a head
+//                 writes bd[o] = disp, boff[o] = stream offset, o = heads before it
+//   k_flat_fin    bl[o] = boff[o+1] - boff[o]; descriptors and facts (atomics)
+//   k_flat_win    the 64 sampled 32-block windows of span_local()
+// Entries of count 0 would make "the previous entry" ambiguous: the pass reports them
+// and the commit takes the host flattening instead.  The host arrays of the form are
+// downloaded only if a host consumer needs them (materialize_host).
+struct FlatFacts {
+  unsigned long long orr;  // OR of every merged disp and length
+  long long lo, hi;        // min disp, max disp + len
+  int not_sdesc, not_mono, zeros, span_good;
+  long long bl0;
+};
+
+__device__ __forceinline__ void flat_entry(const int64_t* __restrict__ D, const int64_t* __restrict__ B, int64_t i,
+                                           int64_t l0, int64_t* l, int64_t* h, int* z) {
+  const int64_t b = B[i];
+  *l = b * l0;
+  *z += b <= 0;
+  *h = i == 0 || D[i - 1] + B[i - 1] * l0 != D[i];  // (d0 cancels)
+}
+
+__global__ void __launch_bounds__(kScanNT) k_flat_tiles(const int64_t* __restrict__ D, const int64_t* __restrict__ B,
+                                                        int64_t n, int64_t l0, int64_t* __restrict__ sl,
+                                                        int64_t* __restrict__ sh, FlatFacts* F) {
+  const int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanItems;
+  int64_t a = 0, c = 0;
+  int z = 0;
+#pragma unroll
+  for (int k = 0; k < kScanItems; k++) {
+    if (base + k >= n) break;
+    int64_t l, h;
+    flat_entry(D, B, base + k, l0, &l, &h, &z);
+    a += l;
+    c += h;
+  }
+  int64_t ta, tc;
+  block_exclusive_scan<kScanNT>(a, &ta);
+  block_exclusive_scan<kScanNT>(c, &tc);
+  if (threadIdx.x == 0) {
+    sl[blockIdx.x] = ta;
+    sh[blockIdx.x] = tc;
+  }
+  if (z) atomicAdd(&F->zeros, z);
+}
+
+__global__ void __launch_bounds__(kScanNT) k_flat_emit(const int64_t* __restrict__ D, const int64_t* __restrict__ B,
+                                                       int64_t n, int64_t d0, int64_t l0,
+                                                       const int64_t* __restrict__ sl, const int64_t* __restrict__ sh,
+                                                       int64_t* __restrict__ bd, int64_t* __restrict__ boff) {
+  const int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanItems;
+  int64_t l[kScanItems], h[kScanItems], a = 0, c = 0;
+  int z = 0;
+#pragma unroll
+  for (int k = 0; k < kScanItems; k++) {
+    l[k] = h[k] = 0;
+    if (base + k < n) flat_entry(D, B, base + k, l0, &l[k], &h[k], &z);
+    a += l[k];
+    c += h[k];
+  }
+  int64_t ta, tc;
+  int64_t L = sl[blockIdx.x] + block_exclusive_scan<kScanNT>(a, &ta);
+  int64_t H = sh[blockIdx.x] + block_exclusive_scan<kScanNT>(c, &tc);
+#pragma unroll
+  for (int k = 0; k < kScanItems; k++) {
+    if (h[k]) {
+      bd[H] = D[base + k] + d0;
+      boff[H] = L;
+    }
+    H += h[k];
+    L += l[k];
+  }
+}
+
+__global__ void __launch_bounds__(256) k_flat_fin(const int64_t* __restrict__ bd, const int64_t* __restrict__ boff,
+                                                  int64_t nb, int64_t total, int64_t* __restrict__ bl,
+                                                  uint64_t* __restrict__ sdesc, int64_t* __restrict__ wbase,
+                                                  FlatFacts* F) {
+  unsigned long long orr = 0;
+  long long lo = LLONG_MAX, hi = LLONG_MIN;
+  int bad_s = 0, bad_m = 0;
+  for (int64_t o = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; o < nb; o += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t d = bd[o];
+    const int64_t l = (o + 1 < nb ? boff[o + 1] : total) - boff[o];
+    bl[o] = l;
+    if (o == 0) F->bl0 = l;
+    orr |= (unsigned long long)d | (unsigned long long)l;
+    lo = min(lo, (long long)d);
+    hi = max(hi, (long long)(d + l));
+    if (o + 1 < nb && d + l > bd[o + 1]) bad_m = 1;
+    const int64_t gb = bd[o & ~int64_t(31)];
+    if ((o & 31) == 0) wbase[o >> 5] = gb;
+    const int64_t r = d - gb;
+    bad_s |= r < INT32_MIN || r > INT32_MAX || l >= (int64_t(1) << 32);
+    sdesc[o] = ((uint64_t)l << 32) | (uint32_t)(int32_t)r;
+  }
+  // warp reduce, then one atomic per warp
+  for (int x = 16; x; x >>= 1) {
+    orr |= __shfl_xor_sync(0xffffffffu, orr, x);
+    lo = min(lo, (long long)__shfl_xor_sync(0xffffffffu, lo, x));
+    hi = max(hi, (long long)__shfl_xor_sync(0xffffffffu, hi, x));
+    bad_s |= __shfl_xor_sync(0xffffffffu, bad_s, x);
+    bad_m |= __shfl_xor_sync(0xffffffffu, bad_m, x);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (orr) atomicOr(&F->orr, orr);
+    if (lo != LLONG_MAX) atomicMin(&F->lo, lo);
+    if (hi != LLONG_MIN) atomicMax(&F->hi, hi);
+    if (bad_s) atomicOr(&F->not_sdesc, 1);
+    if (bad_m) atomicOr(&F->not_mono, 1);
+  }
+}
+
+// span_local()'s sample: window s = blocks [(nb-32)*s/63, +32) within 16 KiB
+__global__ void k_flat_win(const int64_t* __restrict__ bd, const int64_t* __restrict__ bl, int64_t nb, FlatFacts* F) {
+  const int s = blockIdx.x * 32 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  const int64_t i = (nb - 32) * s / 63 + lane;
+  long long lo = bd[i], hi = bd[i] + bl[i];
+  for (int x = 16; x; x >>= 1) {
+    lo = min(lo, (long long)__shfl_xor_sync(0xffffffffu, lo, x));
+    hi = max(hi, (long long)__shfl_xor_sync(0xffffffffu, hi, x));
+  }
+  if (lane == 0 && hi - lo <= 4 * 4096) atomicAdd(&F->span_good, 1);
+}
+
+// DT_OK: flattened and installed; DT_ERR_ARG with *fallback: an entry of count 0 (the
+// host flattening handles it); other errors are errors
+static dt_status gpu_flatten(dt_type_s* t, int64_t d0, int64_t l0, bool* fallback) {
+  *fallback = false;
+  const std::vector<int64_t>& B = t->bls;
+  const std::vector<int64_t>& Dv = *t->hdps;
+  const int64_t n = (int64_t)B.size();
+  int dev = 0;
+  CU(cudaGetDevice(&dev));
+  const int64_t nt = (n + kScanTile - 1) / kScanTile;
+  DeviceDesc dd;
+  dd.device = dev;
+  int64_t *D = nullptr, *Bd = nullptr, *sl = nullptr, *sh = nullptr;
+  FlatFacts* F = nullptr;
+  FlatFacts h;
+  cudaStream_t s = nullptr;
+  dt_status st = DT_OK;
+  int64_t nb = 0, tot[2] = {0, 0};
+  auto fail = [&](cudaError_t e, const char* what) {
+    set_error("GPU flattening: %s: %s", what, cudaGetErrorString(e));
+    return DT_ERR_CUDA;
+  };
+#define FU(call)                                                  \
+  do {                                                            \
+    cudaError_t _e = (call);                                      \
+    if (_e != cudaSuccess) { st = fail(_e, #call); goto out; }    \
+  } while (0)
+  FU(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  FU(cudaMallocAsync(&D, sizeof(int64_t) * n, s));
+  FU(cudaMallocAsync(&Bd, sizeof(int64_t) * n, s));
+  FU(cudaMallocAsync(&sl, sizeof(int64_t) * (nt + 1), s));
+  FU(cudaMallocAsync(&sh, sizeof(int64_t) * (nt + 1), s));
+  FU(cudaMallocAsync(&F, sizeof(FlatFacts), s));
+  std::memset(&h, 0, sizeof(h));
+  h.lo = LLONG_MAX;
+  h.hi = LLONG_MIN;
+  FU(cudaMemcpyAsync(F, &h, sizeof(h), cudaMemcpyHostToDevice, s));
+  {
+    // the raw entry arrays, in chunks so the tile pass of a chunk... (pageable sources:
+    // the driver stages them; the tile pass needs the whole array only for the scan)
+    const int64_t ch = int64_t(1) << 22;
+    for (int64_t i0 = 0; i0 < n; i0 += ch) {
+      const int64_t m = std::min(ch, n - i0);
+      FU(cudaMemcpyAsync(D + i0, Dv.data() + i0, sizeof(int64_t) * m, cudaMemcpyHostToDevice, s));
+      FU(cudaMemcpyAsync(Bd + i0, B.data() + i0, sizeof(int64_t) * m, cudaMemcpyHostToDevice, s));
+    }
+  }
+  k_flat_tiles<<<(unsigned)nt, kScanNT, 0, s>>>(D, Bd, n, l0, sl, sh, F);
+  FU(cudaMemsetAsync(sl + nt, 0, sizeof(int64_t), s));
+  FU(cudaMemsetAsync(sh + nt, 0, sizeof(int64_t), s));
+  k_scan_sums<<<1, kScanNT, 0, s>>>(sl, nt + 1);
+  k_scan_sums<<<1, kScanNT, 0, s>>>(sh, nt + 1);
+  FU(cudaGetLastError());
+  FU(cudaMemcpyAsync(&tot[0], sl + nt, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  FU(cudaMemcpyAsync(&tot[1], sh + nt, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  FU(cudaMemcpyAsync(&h, F, sizeof(h), cudaMemcpyDeviceToHost, s));
+  FU(cudaStreamSynchronize(s));
+  if (h.zeros) {
+    *fallback = true;
+    st = DT_ERR_ARG;
+    goto out;
+  }
+  nb = tot[1];
+  if (tot[0] != t->size || nb < 1 || nb > n) {
+    set_error("GPU flattening: %lld bytes in %lld blocks (type size %lld)", (long long)tot[0], (long long)nb,
+              (long long)t->size);
+    st = DT_ERR_CUDA;
+    goto out;
+  }
+  FU(cudaMalloc(&dd.bd, sizeof(int64_t) * nb));
+  FU(cudaMalloc(&dd.bl, sizeof(int64_t) * nb));
+  FU(cudaMalloc(&dd.boff, sizeof(int64_t) * nb));
+  FU(cudaMalloc(&dd.sdesc, sizeof(uint64_t) * nb));
+  FU(cudaMalloc(&dd.wbase, sizeof(int64_t) * ((nb + 31) / 32)));
+  k_flat_emit<<<(unsigned)nt, kScanNT, 0, s>>>(D, Bd, n, d0, l0, sl, sh, dd.bd, dd.boff);
+  k_flat_fin<<<(unsigned)std::min<int64_t>((nb + 255) / 256, (int64_t)num_sms() * 8), 256, 0, s>>>(
+      dd.bd, dd.boff, nb, tot[0], dd.bl, dd.sdesc, dd.wbase, F);
+  if (nb >= 32) k_flat_win<<<2, 32 * 32, 0, s>>>(dd.bd, dd.bl, nb, F);
+  FU(cudaGetLastError());
+  FU(cudaMemcpyAsync(&h, F, sizeof(h), cudaMemcpyDeviceToHost, s));
+  FU(cudaStreamSynchronize(s));
+out:
+#undef FU
+  if (s) {
+    for (void* p : {(void*)D, (void*)Bd, (void*)sl, (void*)sh, (void*)F})
+      if (p) cudaFreeAsync(p, s);
+    cudaStreamSynchronize(s);
+    cudaStreamDestroy(s);
+  }
+  if (st != DT_OK) {
+    free_desc(dd);
+    return st;
+  }
+  Form f;
+  f.nb_dev = nb;
+  f.bd0_dev = Dv[0] + d0;
+  f.bl0_dev = h.bl0;
+  f.mono_dev = h.not_mono ? 0 : 1;
+  f.tsize_cache = tot[0];
+  f.gran_cache = std::min<int64_t>(16, lowp2(h.orr));
+  f.lvl_gran_cache = 16;
+  f.fits32_cache = (h.lo >= INT32_MIN && h.hi <= INT32_MAX) ? 1 : 0;
+  f.sdesc_ok_cache = h.not_sdesc ? 0 : 1;
+  f.span_lo = h.lo;
+  f.span_hi = h.hi;
+  f.span_local_cache = nb < 32 ? 1 : (h.span_good * 2 >= 64 ? 1 : 0);
+  if (nb <= 4096) {  // a short merged list: keep the host arrays (the ordinary form)
+    f.bd.resize((size_t)nb);
+    f.bl.resize((size_t)nb);
+    if (cudaMemcpy(f.bd.data(), dd.bd, sizeof(int64_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess ||
+        cudaMemcpy(f.bl.data(), dd.bl, sizeof(int64_t) * nb, cudaMemcpyDeviceToHost) != cudaSuccess) {
+      free_desc(dd);
+      set_error("GPU flattening: download of a short list failed");
+      return DT_ERR_CUDA;
+    }
+    f.nb_dev = -1;
+  }
+  const char* no = getenv("DT_NO_SDESC");
+  if (h.not_sdesc || nb < 2 || (no && *no && *no != '0')) {
+    cudaFree(dd.sdesc);
+    cudaFree(dd.wbase);
+    dd.sdesc = nullptr;
+    dd.wbase = nullptr;
+    dd.sdesc_state = 0;
+  } else {
+    dd.sdesc_state = 1;
+  }
+  {
+    std::lock_guard<std::mutex> g(t->mu);
+    t->devs.push_back(dd);
+  }
+  install_form(t, std::move(f));
+  if (getenv("DT_PIPE_DEBUG")) fprintf(stderr, "[dt] GPU flattening: %lld entries -> %lld blocks\n", (long long)n, (long long)nb);
+  return DT_OK;
+}
+
+// f2: the host arrays of a device-flattened form, downloaded once on demand (host
+// consumers: overlap proofs that the device facts do not settle, partial-range launch
+// plans, dt_flatten, serialization, another device's upload)
+dt_status materialize_host(const Form& f, const DeviceDesc& dd) {
+  static std::mutex mm;
+  std::lock_guard<std::mutex> g(mm);
+  if (!f.host_missing()) return DT_OK;
+  Form& F = const_cast<Form&>(f);  // (the form object is owned non-const by its type)
+  int cur = -1;
+  CU(cudaGetDevice(&cur));
+  if (dd.device != cur) CU(cudaSetDevice(dd.device));
+  std::vector<int64_t> bd, bl;
+  huge_reserve(bd, (size_t)f.nb_dev);
+  huge_reserve(bl, (size_t)f.nb_dev);
+  bd.resize((size_t)f.nb_dev);
+  bl.resize((size_t)f.nb_dev);
+  cudaError_t e1 = cudaMemcpy(bd.data(), dd.bd, sizeof(int64_t) * f.nb_dev, cudaMemcpyDeviceToHost);
+  cudaError_t e2 = cudaMemcpy(bl.data(), dd.bl, sizeof(int64_t) * f.nb_dev, cudaMemcpyDeviceToHost);
+  if (dd.device != cur) cudaSetDevice(cur);
+  if (e1 != cudaSuccess || e2 != cudaSuccess) {
+    set_error("materialize_host: %s", cudaGetErrorString(e1 != cudaSuccess ? e1 : e2));
+    return DT_ERR_CUDA;
+  }
+  F.bd.swap(bd);
+  F.bl.swap(bl);
+  F.nb_dev = -1;
+  return DT_OK;
+}
+
+static dt_status materialize_t(dt_type_s* t, const Form& f) {
+  if (!f.host_missing()) return DT_OK;
+  if (t->devs.empty()) {
+    set_error("device-flattened form without a device descriptor");
+    return DT_ERR_ARG;
+  }
+  return materialize_host(f, t->devs[0]);
 }
 
 // f2: the first whole-stream pack of a huge block list (an hindexed list of a
@@ -1277,14 +1612,28 @@ dt_status dt_commit(dt_t t) {
     return DT_ERR_ARG;
   }
   {
-    // f2: a huge block list is flattened by its first whole-stream pack, pipelined with it
+    // f2: a huge block list is flattened on the GPU (default, DT_FLATTEN=gpu), or by its
+    // first whole-stream pack pipelined with it (DT_FLATTEN=pipe: the paper's overlap of
+    // host preparation with the kernels), or on the host (DT_FLATTEN=host / DT_NO_PIPE)
     int64_t d0, l0;
-    if (!t->committed && !t->form && t->kind == K_HINDEXED && t->count >= pipe_min() && !getenv("DT_NO_PIPE") &&
+    const char* fm = getenv("DT_FLATTEN");
+    const std::string mode = getenv("DT_NO_PIPE") ? "host" : fm ? fm : "gpu";
+    if (!t->committed && !t->form && t->kind == K_HINDEXED && t->count >= pipe_min() && mode != "host" &&
         pipe_list(t, &d0, &l0)) {
-      t->lazy_pipe = true;
-      t->committed = true;
-      if (const char* e = getenv("DT_NOCHECK")) g_check_ptrs = (e[0] == '0');
-      return DT_OK;
+      if (mode == "pipe") {
+        t->lazy_pipe = true;
+        t->committed = true;
+        if (const char* e = getenv("DT_NOCHECK")) g_check_ptrs = (e[0] == '0');
+        return DT_OK;
+      }
+      bool fallback = false;
+      dt_status gs = gpu_flatten(t, d0, l0, &fallback);
+      if (gs == DT_OK) {
+        t->committed = true;
+        if (const char* e = getenv("DT_NOCHECK")) g_check_ptrs = (e[0] == '0');
+        return DT_OK;
+      }
+      if (!fallback) return gs;  // (entries of count 0: the host flattening below)
     }
   }
   try {
@@ -1324,12 +1673,12 @@ static dt_status make_kp(dt_type_s* t, int64_t count, const void* nc, int64_t n,
   P.pos = 0;
   P.len = n;
   P.tsize = f.tsize();
-  P.nblocks = (int64_t)f.bl.size();
+  P.nblocks = f.nblocks();
   P.bd = dd->bd;
   P.bl = dd->bl;
   P.boff = dd->boff;
-  P.bd0 = f.bd[0];
-  P.bl0 = f.bl[0];
+  P.bd0 = f.first_bd();
+  P.bl0 = f.first_bl();
   P.nlev = L.n;
   for (int i = 0; i < L.n; i++) {
     P.cnt[i] = L.cnt[i];

@@ -759,7 +759,7 @@ dt_status dt_get_form(dt_t t, dt_form_info* o) {
   o->extent = t->extent();
   o->true_lb = t->true_lb;
   o->true_extent = t->true_ub - t->true_lb;
-  o->nblocks = (int64_t)f->bl.size();
+  o->nblocks = f->nblocks();
   o->tsize = f->tsize();
   o->nlevels = (int32_t)f->lv.size();
   for (int i = 0; i < o->nlevels && i < 8; i++) {
@@ -777,6 +777,7 @@ dt_status dt_flatten(dt_t t, int64_t count, int64_t* disps, int64_t* lens, int64
   const Form* f;
   dt_status s = safe_form(t, &f);
   if (s != DT_OK) return s;
+  if (f->host_missing() && (s = materialize_host(*f, t->devs[0])) != DT_OK) return s;
   Form g = *f;
   if (count != 1) prepend_regular(g, count, t->extent());
   normalize(g);
@@ -807,6 +808,7 @@ dt_status dt_type_serialize(dt_t t, void* out, size_t* nbytes) {
   const Form* f;
   dt_status s = safe_form(t, &f);
   if (s != DT_OK) return s;
+  if (f->host_missing() && (s = materialize_host(*f, t->devs[0])) != DT_OK) return s;
   std::vector<int64_t> w = {kSerMagic, 1, t->size, t->lb, t->ub, t->true_lb, t->true_ub, t->align,
                             t->has_lb ? 1 : 0, t->has_ub ? 1 : 0, (int64_t)f->lv.size(), (int64_t)f->bd.size()};
   for (auto& l : f->lv) {

@@ -584,6 +584,7 @@ def test_pipelined_first_pack(torch_cuda, first, seed, monkeypatch):
     from paper_conf_hpdc_wubvjd16_b200 import dt
     monkeypatch.setenv("DT_PIPE_MIN", "1000")
     monkeypatch.setenv("DT_PIPE_CHUNK", "7001")
+    monkeypatch.setenv("DT_FLATTEN", "pipe")
     rng = np.random.default_rng(40 + seed)
     n = 120_000
     lens = rng.integers(1, 17, size=n) * (4 if seed == 0 else 1)
@@ -614,3 +615,82 @@ def test_pipelined_first_pack(torch_cuda, first, seed, monkeypatch):
     # the installed form is the ordinary one
     bd, bl = t.flatten(1)
     assert int(bl.sum()) == len(exp)
+
+
+# ------------------------------------------------------------------ f2: GPU-side flattening
+def _oracle_blocks(ot):
+    """Merged block list of a BYTE-element typemap: runs of consecutive byte addresses, in
+    typemap order (the flattening's definition, computed from the oracle's typemap)."""
+    _, d = ot.typemap()
+    if len(d) == 0:
+        return d, d
+    starts = np.concatenate([[0], np.flatnonzero(np.diff(d) != 1) + 1])
+    lens = np.diff(np.concatenate([starts, [len(d)]]))
+    return d[starts], lens
+
+
+@pytest.mark.parametrize("case", ["sorted", "shuffled", "negative", "zeros", "all_adjacent"])
+def test_gpu_flatten(torch_cuda, case, monkeypatch):
+    """f2: dt_commit of a huge block list (an hindexed list of BYTE with per-entry
+    counts) flattens it ON THE DEVICE (tile sums, scans, head emission, facts); the
+    merged list (downloaded by dt_flatten), pack, unpack, the launch plan and the form
+    facts must equal the oracle's / the host flattening's.  Cases: sorted with zero gaps
+    (merges, also across 1024-entry tiles), shuffled entries (not sorted: unpack legality
+    needs the host proof), negative displacements with a misaligned origin, entries of
+    count 0 (the host flattening takes over), every entry adjacent (one block)."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    monkeypatch.setenv("DT_PIPE_MIN", "1000")
+    rng = np.random.default_rng({"sorted": 1, "shuffled": 2, "negative": 3, "zeros": 4, "all_adjacent": 5}[case])
+    n = 50_000
+    lens = rng.integers(1, 17, size=n) * 4
+    gaps = rng.integers(0, 4, size=n) * 4
+    if case == "all_adjacent":
+        gaps[:] = 0
+    if case == "zeros":
+        lens[rng.integers(0, n, size=50)] = 0
+    d = np.concatenate([[0], np.cumsum(lens + gaps)[:-1]]).astype(np.int64)
+    if case == "shuffled":
+        perm = rng.permutation(n)
+        lens, d = lens[perm], d[perm]
+    org = 0
+    if case == "negative":
+        d = d - int(d[-1]) // 2
+        org = int(-d.min()) + 3
+    rec = ("hindexed", lens, d, ("basic", "BYTE"))
+    parent = int((d + lens).max()) + org + 64
+    ot = oracle.from_recipe(rec)
+    ob, ol = _oracle_blocks(ot)
+    t = dt.from_recipe(rec).commit()
+    monkeypatch.setenv("DT_FLATTEN", "host")
+    th = dt.from_recipe(rec).commit()
+    monkeypatch.delenv("DT_FLATTEN")
+    # launch plans and form facts equal the host flattening's (before any download)
+    fi, fh = t.form(), th.form()
+    assert (fi.nblocks, fi.tsize, fi.granularity) == (fh.nblocks, fh.tsize, fh.granularity) == (len(ob), ot.size,
+                                                                                                fh.granularity)
+    for addr, pk in ((0x10000, 0x20000), (0x10003, 0x20000), (0x10000, 0x20008)):
+        assert t.plan(1, addr, pk, 0, ot.size) == th.plan(1, addr, pk, 0, ot.size)
+    src_h = fill_bytes(parent, 91)
+    exp = oracle.pack(ot, 1, src_h, org)
+    src = _dev(torch, src_h)
+    out = _poisoned(torch, len(exp))
+    dt.pack(t, 1, src, out.data_ptr() + GUARD, origin_offset=org)
+    torch.cuda.synchronize()
+    o = out.cpu().numpy()
+    assert np.all(o[:GUARD] == 0xA5) and np.all(o[GUARD + len(exp):] == 0xA5)
+    assert np.array_equal(o[GUARD:GUARD + len(exp)], exp)
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8, device="cuda")
+    dt.unpack(t, 1, _dev(torch, exp), dst, origin_offset=org)
+    ref = np.full(parent, 0xA5, dtype=np.uint8)
+    oracle.unpack(ot, 1, exp, ref, org)
+    torch.cuda.synchronize()
+    assert np.array_equal(dst.cpu().numpy(), ref)
+    # a fragment (partial range: the launch plan needs the block prefix on the host)
+    p0, p1 = len(exp) // 3 + 5, 2 * len(exp) // 3 + 1
+    out.fill_(0xA5)
+    dt.pack(t, 1, src, out.data_ptr() + GUARD, pos=p0, nbytes=p1 - p0, origin_offset=org)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy()[GUARD:GUARD + p1 - p0], exp[p0:p1])
+    bd, bl = t.flatten(1)
+    assert np.array_equal(bd, ob) and np.array_equal(bl, ol)

@@ -8,9 +8,13 @@ device prefix scan); the first pack also builds its launch plan.  For each
 workload this prints, in ms: type construction, host flattening, device upload,
 the first pack (upload pipelined with it when the list is large), a cached pack,
 and first-use total (flatten + upload + first pack + the second pack's one-time
-extra) vs cached.  FU_PIPELINED=1: no separate host flattening, so a huge
-block list (C5b) is flattened by its first pack, pipelined with the upload and the pack
-kernels (dt_commit defers it); otherwise the flattening is forced before the commit.
+extra) vs cached.  FU_MODE selects how a huge block list (C5b) is prepared:
+  host  the host flattening is forced before the commit (t.form()), then uploaded;
+  pipe  flattened by its first pack, pipelined with the upload and the pack kernels
+        (DT_FLATTEN=pipe: dt_commit defers it -- the paper's overlap);
+  gpu   flattened on the GPU by dt_commit (the default): only the raw entry arrays
+        cross the host link.
+(FU_PIPELINED=1 is FU_MODE=pipe.)
 """
 import json
 import os
@@ -32,7 +36,10 @@ def main():
     dev = torch.device("cuda")
     torch.zeros(1, device=dev)
     s = torch.cuda.current_stream()
-    pipelined = os.environ.get("FU_PIPELINED") == "1"
+    mode = os.environ.get("FU_MODE", "pipe" if os.environ.get("FU_PIPELINED") == "1" else "host")
+    if mode == "pipe":
+        os.environ["DT_FLATTEN"] = "pipe"
+    pipelined = mode != "host"
     for name in names:
         rec, org, parent = mk[name]()
         src = torch.empty(parent, dtype=torch.uint8, device=dev).random_(0, 255)
@@ -67,7 +74,7 @@ def main():
             cached = min(cached, time.perf_counter() - c0)
         same = bool(torch.equal(first, pk))
         ms = lambda x: round(x * 1e3, 3)  # noqa: E731
-        print(json.dumps({"config": name, "pipelined_first_pack": pipelined, "bytes": t.size, "create_ms": ms(t1 - t0), "host_flatten_ms": ms(t2 - t1),
+        print(json.dumps({"config": name, "mode": mode, "bytes": t.size, "create_ms": ms(t1 - t0), "host_flatten_ms": ms(t2 - t1),
                           "commit_upload_ms": ms(t3 - t2), "first_pack_ms": ms(t5 - t4),
                           "second_pack_ms": ms(second), "cached_pack_ms": ms(cached),
                           "first_use_ms": ms((t2 - t1) + (t3 - t2) + (t5 - t4) + second - cached),
