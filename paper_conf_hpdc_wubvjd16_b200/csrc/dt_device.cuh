@@ -599,7 +599,10 @@ __device__ __forceinline__ void group_sync(int bar, int nthr) {
 // words into the tile buffer; the finished tile leaves with one bulk store.
 // NB tile buffers: NB-1 tiles of gathers in flight while the oldest finished tile
 // is stored, so a CTA keeps (NB-1)*16 KiB of loads outstanding.
-template <int G, int NB>
+// PLAIN: the finished tile leaves with coalesced 16-byte stores of the group's threads
+// instead of a TMA bulk store (a ring slot in another GPU's memory: generic-proxy
+// stores over NVLink, ordered by the control warp's system-scope release)
+template <int G, int NB, bool PLAIN = false>
 __device__ __forceinline__ void stage_pack(const KP& P, uint8_t* cb, const int32_t* wt, int64_t lo, int64_t hi,
                                            uint8_t* sbuf, const int tid, const int nthr, const int bar = 0) {
   constexpr int T = kStageTile, L = NB - 1;
@@ -623,7 +626,7 @@ __device__ __forceinline__ void stage_pack(const KP& P, uint8_t* cb, const int32
   for (int64_t t = 0; t < ntiles + L - 1; t++) {
     if (t < ntiles) {
       uint8_t* buf = sbuf + (t % NB) * T - (t * T);  // word iw lands at buf + iw*G
-      if (tid == 0) bulk_wait_read<1>();  // the store that last read this buffer (tile t-NB) is done reading
+      if (!PLAIN && tid == 0) bulk_wait_read<1>();  // the store that last read this buffer (tile t-NB) is done reading
       group_sync(bar, nthr);
       const int64_t wend = (t + 1) * (T / G) < nwords ? (t + 1) * (T / G) : nwords;
       while (iw < wend) {
@@ -641,7 +644,16 @@ __device__ __forceinline__ void stage_pack(const KP& P, uint8_t* cb, const int32
     if (u >= 0) {
       cp_async_wait<L - 1>();
       group_sync(bar, nthr);
-      if (tid == 0) {
+      if (PLAIN) {
+        const int64_t s1 = lo + u * T;
+        const int64_t tl = hi - s1 < T ? hi - s1 : (int64_t)T;
+        const uint8_t* buf = sbuf + (u % NB) * T;
+        const int nv = (int)(tl >> 4);
+        for (int i = tid; i < nv; i += nthr)
+          stv(reinterpret_cast<uint4*>(cb + s1) + i, reinterpret_cast<const uint4*>(buf)[i]);
+        if (tid == 0)
+          for (int64_t k = tl & ~int64_t(15); k < tl; k++) cb[s1 + k] = buf[k];  // ragged tail
+      } else if (tid == 0) {
         const int64_t s1 = lo + u * T;
         const int64_t tl = hi - s1 < T ? hi - s1 : (int64_t)T;
         const uint8_t* buf = sbuf + (u % NB) * T;
@@ -654,7 +666,7 @@ __device__ __forceinline__ void stage_pack(const KP& P, uint8_t* cb, const int32
       }
     }
   }
-  if (tid == 0) bulk_wait_all();
+  if (!PLAIN && tid == 0) bulk_wait_all();
 }
 
 // Unpack: tiles of the contiguous stream arrive by TMA bulk loads (NB in flight,
@@ -948,7 +960,16 @@ __device__ __forceinline__ void blk_range(const KP& P, uint8_t* cbase, int64_t p
 //     copy work, not a DRAM round trip.
 // Every DRAM sector of the layout is requested once by a 16-byte access instead
 // of once per G-byte word (the per-word gathers of blk_range).
-constexpr int kSpanBuf = 4096;  // layout span bytes per window (multiple of 16)
+#ifndef DT_SPAN_BUF
+#define DT_SPAN_BUF 4096
+#endif
+#ifndef DT_SPAN_MINB
+#define DT_SPAN_MINB 2
+#endif
+// layout span bytes per window (multiple of 16).  (Measured: 3 KiB spans with three
+// 256-thread CTAs per SM -- 80 registers, 128-184 bytes of spills -- made C5b 64 MiB
+// pack / unpack 70.6 / 94.2 us vs 53-56 / 78 us with 4 KiB and two CTAs.)
+constexpr int kSpanBuf = DT_SPAN_BUF;
 constexpr int kSpanOut = 2048;  // packed bytes per window (multiple of 16)
 constexpr int kSpanOutB = kSpanOut + 32;
 constexpr int kSpanDesc = 32 * 16;  // one window's (len, disp) pairs

@@ -112,7 +112,8 @@ __global__ void __launch_bounds__(kDirThreads) k_direct(const __grid_constant__ 
     const int64_t t0 = X.ntiles * j / X.ncta, t1 = X.ntiles * (j + 1) / X.ncta;
     const int64_t lo = t0 * kStageTile, hi = min(t1 * (int64_t)kStageTile, X.n);
     if (lo < hi) {
-      if (X.g == 8) stage_copy<8, kStageBufs>(X.S, wts, X.R, wtr, lo, hi, dsm);
+      if (X.g == 4) stage_copy<4, kStageBufs>(X.S, wts, X.R, wtr, lo, hi, dsm);
+      else if (X.g == 8) stage_copy<8, kStageBufs>(X.S, wts, X.R, wtr, lo, hi, dsm);
       else stage_copy<16, kStageBufs>(X.S, wts, X.R, wtr, lo, hi, dsm);
     }
   }

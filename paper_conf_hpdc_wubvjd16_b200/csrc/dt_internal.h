@@ -2,6 +2,7 @@
 // kernel parameters).  Not part of the C-ABI (include/dt.h is).
 #pragma once
 #include <cstdint>
+#include <cstdlib>
 #include <memory>
 #include <mutex>
 #include <string>
@@ -16,6 +17,18 @@ constexpr int64_t kMaxFlatBlocks = int64_t(1) << 28;  // cap on an expanded bloc
 constexpr int64_t kMaxWordTable = 12288;              // word-table kernel: entries in smem
 
 void set_error(const char* fmt, ...);
+
+// Smallest word size G the smem/TMA staged family takes (cp.async gathers, persistent
+// element iterators); below it the register word-table family.  4 since round 2 (C4
+// x-face 1 MiB: staged pack/unpack 15.4 / 13.3 us vs 17.4 / 20.5 on 148 SMs, 21.5 vs
+// 44 us on 16 SMs); DT_STAGE_G=8 restores the round-1 rule.
+inline int64_t stage_min_g() {
+  static const int64_t g = [] {
+    const char* e = std::getenv("DT_STAGE_G");
+    return e && std::atoll(e) > 0 ? (int64_t)std::atoll(e) : (int64_t)4;
+  }();
+  return g;
+}
 
 // One level of the element iteration space above the block template.
 // Element index decomposes mixed-radix over the levels, the LAST level fastest

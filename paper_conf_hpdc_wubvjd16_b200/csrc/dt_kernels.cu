@@ -162,7 +162,7 @@ __global__ void __launch_bounds__(256) k_blk(const KP P) {
 // block-span pack/unpack (short blocks of a large irregular list): warp w owns
 // stream bytes [pos + w*per_warp, ...) and walks them 32 blocks at a time
 template <bool UNPACK, int G>
-__global__ void __launch_bounds__(256, 2) k_span(const KP P, const PlanEnt* __restrict__ plan, int64_t nw) {
+__global__ void __launch_bounds__(256, DT_SPAN_MINB) k_span(const KP P, const PlanEnt* __restrict__ plan, int64_t nw) {
   extern __shared__ __align__(16) uint8_t smem_span[];
   const int lane = threadIdx.x & 31;
   uint8_t* sm = smem_span + (threadIdx.x >> 5) * kSpanWarpSmem;
@@ -689,7 +689,7 @@ int plan_kernel(const Form& f, const KLevels& L, uint64_t nc_addr, uint64_t c_ad
   // segments; measured), with 4-byte words the register word kernel does
   // short blocks in small dense records (C5 particles): whole-record 16-byte loads
   if (mean < 256.0 && rec_ok && !force) return 6;
-  if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return stage_ok && g >= 8 ? 4 : 2;
+  if ((mean < 256.0 || (g == 16 && mean < 1024.0)) && word_ok) return stage_ok && g >= stage_min_g() ? 4 : 2;
   // many short blocks (no word table): block spans with >= 4-byte words, else block windows
   if (mean < 128.0 && g >= 4 && !force && span_local(f)) return 7;
   if (mean < 128.0 && blk_ok) return 3;
@@ -1746,7 +1746,7 @@ dt_status dt::dual_params(dt_type_s* st, int64_t scount, const void* src, dt_typ
   R.wtab = wb;
   R.nwords = (int32_t)(R.tsize / g);
   // staged for >= 8-byte words (DT_FORCE_KERNEL=2 keeps the register word kernel)
-  *kind = (g >= 8 && force != 2) ? 4 : 2;
+  *kind = (g >= stage_min_g() && g >= 4 && force != 2) ? 4 : 2;
   return DT_OK;
 }
 
@@ -1794,6 +1794,7 @@ static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, i
     const size_t smem2 = (size_t)kStageBufs * kStageTile + sizeof(int32_t) * (size_t)(S.nwords + R.nwords);
     bool& attr = devl().dual_attr;
     if (!attr) {
+      cudaFuncSetAttribute(k_dual_stage<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
       cudaFuncSetAttribute(k_dual_stage<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
       cudaFuncSetAttribute(k_dual_stage<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 120 * 1024);
       attr = true;
@@ -1803,7 +1804,8 @@ static dt_status copy_typed(dt_t st, int64_t scount, const void* src, dt_t rt, i
       occ = 1;
     const int64_t ntiles = (n + kStageTile - 1) / kStageTile;
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, ntiles));
-    if (g == 8) k_dual_stage<8><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
+    if (g == 4) k_dual_stage<4><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
+    else if (g == 8) k_dual_stage<8><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
     else k_dual_stage<16><<<grid, 256, smem2, s>>>(S, R, n, ntiles);
   } else if (kind == 2) {
     const size_t smem = sizeof(int32_t) * (size_t)(S.nwords + R.nwords);

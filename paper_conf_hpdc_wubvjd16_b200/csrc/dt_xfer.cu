@@ -145,6 +145,7 @@ template <bool UNPACK, int G>
 __device__ __noinline__ void xc_stage(const XOp& X, uint8_t* cb, const int32_t* wt, int64_t lo, int64_t bh,
                                       uint8_t* sbuf, uint64_t* mbar, int ctid, int cnthr, int bar, int64_t tb) {
   if (UNPACK) stage_unpack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf, mbar, ctid, cnthr, bar, tb);
+  else if (X.sys) stage_pack<G, kXferStageBufs, true>(X.P, cb, wt, lo, bh, sbuf, ctid, cnthr, bar);  // peer GPU
   else stage_pack<G, kXferStageBufs>(X.P, cb, wt, lo, bh, sbuf, ctid, cnthr, bar);
 }
 
@@ -199,7 +200,8 @@ __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo,
   if (X.kind == 4) {  // smem/TMA staging: bulk store into the (peer) ring slot / bulk load from it
     const int64_t bh = hi - len % X.g;
     uint8_t* gbuf = sbuf + (size_t)g * kXferStageBufs * kStageTile;
-    if (X.g == 8) xc_stage<UNPACK, 8>(X, cb, wt, lo, bh, gbuf, mbar, ctid, cnthr, bar, tb);
+    if (X.g == 4) xc_stage<UNPACK, 4>(X, cb, wt, lo, bh, gbuf, mbar, ctid, cnthr, bar, tb);
+    else if (X.g == 8) xc_stage<UNPACK, 8>(X, cb, wt, lo, bh, gbuf, mbar, ctid, cnthr, bar, tb);
     else xc_stage<UNPACK, 16>(X, cb, wt, lo, bh, gbuf, mbar, ctid, cnthr, bar, tb);
     tb += (bh - lo + kStageTile - 1) / kStageTile;  // tiles through this group's mbarriers
     if (bh < hi) {
@@ -207,7 +209,7 @@ __device__ __forceinline__ void cta_piece(const XOp& X, uint8_t* cb, int64_t lo,
       if (w == 0) xc_seg<UNPACK, false>(X, cb, bh, hi, lane);
     }
     // the TMA bulk stores (async proxy) of the piece precede the control warp's release
-    if (!UNPACK && ctid == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
+    if (!UNPACK && !X.sys && ctid == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
     return;
   }
   if (X.kind == 2) {
@@ -248,7 +250,7 @@ struct PieceIt {
     gu = (int)min((int64_t)gs, ((n < C ? n : C) + Cs - 1) / Cs);
     if (gu < 1) gu = 1;
     const int npairs = gu * rep;
-    one = role == 0 || ncta >= npairs;
+    one = ncta >= npairs;  // (either role: fewer CTAs than pairs take pairs j, j + ncta, ...)
     if (one && j >= npairs) return false;
     kstep = one ? rep : 1;
     jstep = one ? gu : ncta;
@@ -929,17 +931,18 @@ static dt_status side_params(dt_t t, int64_t count, const void* nc, int64_t nbyt
   int kind = E.merged ? 1 : plan_kernel(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, &g);
   if (kind == 6) {  // record spans: pieces start on 512-byte stream boundaries (16-byte aligned)
     if (!rec_geometry(f, L, (uint64_t)(uintptr_t)nc, 0, 0, nbytes, g, &X.rg) || getenv("DT_XFER_NOREC"))
-      kind = g >= 8 ? 4 : 2;
+      kind = g >= stage_min_g() ? 4 : 2;
   }
   if ((kind == 2 || kind == 4 || kind == 6 || kind == 7) && lowp2u((uint64_t)chunk) < g) kind = 1;
-  if (kind == 4 && g < 8) kind = 2;
+  if (kind == 4 && g < std::max<int64_t>(4, stage_min_g())) kind = 2;
+  if (kind == 2 && g >= std::max<int64_t>(4, stage_min_g()) && !getenv("DT_XFER_NOSTAGE")) kind = 4;
   if (kind == 7 && getenv("DT_XFER_NOSPAN")) kind = 1;
   // the block-window kernel (3) is not used inside the pipeline
   X.kind = (kind == 2 || kind == 4 || kind == 6 || kind == 7) ? kind : 1;
   if (const char* fk = getenv("DT_XFER_KIND")) {  // tuning: force a family where it applies
     const int k = atoi(fk);
     const bool wt_ok = f.tsize() / g <= kMaxWordTable && f.tsize() % g == 0 && !E.merged;
-    if ((k == 2 && wt_ok) || (k == 4 && wt_ok && g >= 8) || k == 1) X.kind = k;
+    if ((k == 2 && wt_ok) || (k == 4 && wt_ok && g >= 4) || k == 1) X.kind = k;
   }
   if (X.kind == 7) {
     P.fnb = make_fd((uint64_t)P.nblocks);
@@ -981,12 +984,24 @@ static int default_ctas(const dt_comm_s* c) {
 struct Geo {
   int gs, gu, rep;
 };
-static Geo geometry(int64_t n, int64_t C, int D, int budget) {
-  static const int64_t kPiece = getenv("DT_XFER_PIECE") ? atoll(getenv("DT_XFER_PIECE")) : (32 << 10);
+static Geo geometry(int64_t n, int64_t C, int D, int budget, double w = 1.0) {
+  static const int64_t kPiece0 = getenv("DT_XFER_PIECE") ? atoll(getenv("DT_XFER_PIECE")) : (32 << 10);
+  // a family that moves bytes w times slower per CTA amortises the per-piece fixed cost
+  // (flag release, barriers) over w times fewer bytes
+  int64_t kPiece = std::max<int64_t>(4096, (int64_t)(kPiece0 / std::max(1.0, w)));
+  // a message of one fragment is latency-bound: spread it over up to the budget's CTAs in
+  // pieces of >= 4 KiB (a piece's fixed costs overlap across CTAs instead of adding up)
+  if (n > C) kPiece = kPiece0;  // (several fragments: teams on alternate fragments matter more)
+  else if (!getenv("DT_XFER_PIECE")) kPiece = std::min(kPiece, std::max<int64_t>(4096, n / std::max(1, budget)));
   const int64_t eff = std::min<int64_t>(C, std::max<int64_t>(512, (n + 511) & ~int64_t(511)));
-  // p: CTAs per fragment, pieces of >= kPiece bytes
+  // p: pieces per fragment, >= kPiece bytes each, up to two per CTA of the budget (a
+  // CTA's two copy groups take alternate pieces: with one piece per CTA -- a message of
+  // one fragment -- the second group would idle)
   int p = 1;
-  while (p * 2 <= kMaxSub && p * 2 <= budget && eff / (p * 2) >= kPiece) p *= 2;
+  // (one fragment: as many pieces as the slot layout allows, several per CTA, so the
+  // receiver starts on the first pieces while the sender packs the later ones -- the
+  // paper's pipeline inside one fragment)
+  while (p * 2 <= kMaxSub && (n <= C || p * 2 <= 2 * budget) && eff / (p * 2) >= kPiece) p *= 2;
   // gs: the slot layout, pieces of C/gs >= eff/p bytes (a message shorter than C uses
   // gu < gs of them)
   const int64_t want = (((eff + p - 1) / p) + 511) & ~int64_t(511);
@@ -1036,10 +1051,9 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
       X.seqp = c->dseq + ((size_t)0 * c->nranks + p.dest) * c->nch + ch;
       X.done = c->ddone + ((size_t)0 * c->nranks + p.dest) * c->nch + ch;
       X.sys = !c->same_dev[p.dest];
-      // a peer on another GPU: the staged family's TMA bulk stores would target peer
-      // memory, never exercised on a one-GPU lease -- use the word-table family's
-      // plain 16-byte stores there (DT_XFER_PEER_TMA=1 keeps TMA)
-      if (X.sys && X.kind == 4 && !getenv("DT_XFER_PEER_TMA")) X.kind = 2;
+      // a peer on another GPU: the staged family's tiles leave with plain coalesced
+      // 16-byte stores (no TMA bulk stores into peer memory, never exercised on a
+      // one-GPU lease; X.sys selects them in xc_stage)
     }
     if (p.source >= 0) {
       if (nops >= kMaxOps) { set_error("dt_sendrecv: too many ops in one group"); return DT_ERR_UNSUPPORTED; }
@@ -1092,7 +1106,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   // Unpacking G-byte words scatters partial-sector writes (each a DRAM read-modify-write
   // when G < 32): measured ~2x the pack cost, so the factor doubles on the receive side.
   auto cost = [](const XOp& X) {
-    double w = X.kind == 2 ? 16.0 / X.g : (X.kind == 6 || X.kind == 7) ? 2.0 : 1.0;
+    double w = (X.kind == 2 || X.kind == 4) ? 16.0 / X.g : (X.kind == 6 || X.kind == 7) ? 2.0 : 1.0;
     if (X.role == 1 && X.g < 16 && X.kind != 1) w *= 2;
     return (double)std::max<int64_t>(X.n, 4096) * w;
   };
@@ -1108,11 +1122,13 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
                             : std::max(1, std::min(default_ctas(c), (int)(total * cost(X) / csum)));
     // send role: one CTA per (team, piece); receive role: as many as the capacity
     // would need (the actual geometry arrives in the header; CTAs map onto it)
-    const Geo G = geometry(X.n, X.chunk, X.depth, budget);
+    const Geo G = geometry(X.n, X.chunk, X.depth, budget, cost(X) / (double)std::max<int64_t>(X.n, 4096));
     X.gs = G.gs;
     X.rep = G.rep;
     X.cta0 = cta;
-    X.ncta = G.gu * G.rep;
+    // pairs (team, piece) beyond the budget: CTAs take several (pairs j, j + ncta, ...)
+    const int npairs = G.gu * G.rep, ppc = (npairs + budget - 1) / budget;
+    X.ncta = (npairs + ppc - 1) / ppc;
     cta += X.ncta;
   }
   if (getenv("DT_XFER_DEBUG"))

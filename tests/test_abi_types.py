@@ -100,18 +100,19 @@ def test_plan_selects_kernels():
     t = dt.from_recipe(c2_lower_triangle()[0])
     assert t.plan(1, 0x10000, 0x20000, 0, 1 << 30) == (1, 8)     # long runs: warp segments
     t = dt.from_recipe(c4_face("x-")[0])
-    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 30)[0] == 2       # 4-byte elements: word kernel
+    assert t.plan(1, 0x10000, 0x20000, 0, 1 << 30)[0] == 4       # 4-byte elements: smem-staged gathers
+    assert t.plan(1, 0x10000, 0x20004, 0, 1 << 30)[0] == 2       # packed side not 16-B aligned: word kernel
     k, g = t.plan(1, 0x10000, 0x20000, 0, 1 << 30)
     assert g == 4
     t = dt.from_recipe(c5_particles(56 * 100)[0])
     assert t.plan(1, 0x10000, 0x20000, 0, 1 << 30) == (6, 4)     # dense records: record spans
     assert t.plan(1, 0x10000, 0x20004, 0, 1 << 30) == (2, 4)     # packed side not 16-B aligned: words
-    assert t.plan(1, 0x10008, 0x20000, 0, 1 << 30) == (2, 4)     # record bases not 16-B aligned: words
+    assert t.plan(1, 0x10008, 0x20000, 0, 1 << 30) == (4, 4)     # record bases not 16-B aligned: staged words
     assert t.plan(1, 0x10000, 0x20000, 32, 4000) == (6, 4)       # 16-B-congruent fragment
-    # sparse records (8 of 32 span bytes) stay on word gathers
+    # sparse records (8 of 32 span bytes) stay on word gathers (smem-staged)
     t = dt.from_recipe(("hvector", 100, 1, 64, ("resized", ("struct", [1, 1], [0, 28], [("basic", "INT32")] * 2),
                                                 0, 64)))
-    assert t.plan(1, 0x10000, 0x20000, 0, 800)[0] == 2
+    assert t.plan(1, 0x10000, 0x20000, 0, 800)[0] == 4
     # byte-granular start position lowers the word size
     assert t.plan(1, 0x10000, 0x20000, 3, 100) == (2, 1)
     # irregular short blocks under a template too large for a word table: block spans
@@ -128,7 +129,7 @@ def test_plan_selects_kernels():
     slots = np.random.default_rng(5).permutation(1 << 16)[: 1 << 15].astype(np.int64)
     t = dt.from_recipe(("hindexed", np.ones(1 << 15, dtype=np.int64), slots * 16, rs))
     assert t.plan(1, 0x10000, 0x20000, 0, 1 << 16)[0] == 6    # whole-record loads, any order
-    assert t.plan(1, 0x10008, 0x20000, 0, 1 << 16)[0] == 2    # records not 16-B aligned: word table
+    assert t.plan(1, 0x10008, 0x20000, 0, 1 << 16)[0] == 4    # records not 16-B aligned: staged word table
     # contiguous type, many instances: one long run
     t = dt.Type.basic("DOUBLE").contiguous(10)
     assert t.plan(1000, 0x10000, 0x20000, 0, 80000)[0] == 1

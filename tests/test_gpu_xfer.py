@@ -56,6 +56,27 @@ def test_loopback_block_cyclic(torch_cuda, chunk, depth, ring):
     comm.free()
 
 
+@pytest.mark.parametrize("wl", ["c3", "c4x"])
+def test_loopback_system_scope(torch_cuda, wl, monkeypatch):
+    """The peer-on-another-GPU configuration on one GPU (DT_XFER_SYS: system-scope flags,
+    as across NVLink): the staged family's tiles leave with plain coalesced stores
+    instead of TMA bulk stores into the peer's ring slot.  C3 (16-byte words) and the
+    C4 x-face (4-byte words at a 2056-byte pitch), several fragments and one."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    from workloads import c4_face
+    monkeypatch.setenv("DT_XFER_SYS", "1")
+    for chunk in (256 << 10, 1 << 20):
+        comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=0, ring_loopback=True)
+        if wl == "c3":
+            rec, org, parent = c3_block_cyclic(2048, 64)
+            _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent)
+        else:
+            s, so, sp = c4_face("x-", 128)
+            r, ro, rp = c4_face("x+", 128, ghost=True)
+            _loop_check(torch_cuda, comm, s, so, sp, r, ro, rp)
+        comm.free()
+
+
 @pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
 def test_loopback_different_types(torch_cuda, ring):
     """Same signature, different layouts (vector <-> contiguous, triangle -> packed;
