@@ -1116,6 +1116,7 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
   // every op gets the default budget when all of them fit; otherwise shares by cost
   const bool fits = (int64_t)nops * default_ctas(c) <= total;
   int cta = 0;
+  int np[kMaxOps], ppc[kMaxOps];
   for (int i = 0; i < nops; i++) {
     XOp& X = A.ops[i];
     const int budget = fits ? default_ctas(c)
@@ -1125,11 +1126,33 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
     const Geo G = geometry(X.n, X.chunk, X.depth, budget, cost(X) / (double)std::max<int64_t>(X.n, 4096));
     X.gs = G.gs;
     X.rep = G.rep;
-    X.cta0 = cta;
     // pairs (team, piece) beyond the budget: CTAs take several (pairs j, j + ncta, ...)
-    const int npairs = G.gu * G.rep, ppc = (npairs + budget - 1) / budget;
-    X.ncta = (npairs + ppc - 1) / ppc;
+    np[i] = G.gu * G.rep;
+    ppc[i] = (np[i] + budget - 1) / budget;
+    X.ncta = (np[i] + ppc[i] - 1) / ppc[i];
     cta += X.ncta;
+  }
+  // Co-resident CTAs the shares left unused (budgets round down to whole pieces per CTA):
+  // give them to the op whose CTAs carry the most work (cost per piece x pieces per CTA)
+  // while the next step fits -- the group's makespan is its slowest op's.
+  while (!fits) {
+    int best = -1;
+    double bt = -1;
+    for (int i = 0; i < nops; i++) {
+      const double t = cost(A.ops[i]) / np[i] * ppc[i];
+      if (t > bt) { bt = t; best = i; }
+    }
+    if (best < 0 || ppc[best] <= 1) break;
+    const int nn = (np[best] + ppc[best] - 2) / (ppc[best] - 1);
+    if (cta - A.ops[best].ncta + nn > total) break;
+    cta += nn - A.ops[best].ncta;
+    A.ops[best].ncta = nn;
+    ppc[best]--;
+  }
+  cta = 0;
+  for (int i = 0; i < nops; i++) {
+    A.ops[i].cta0 = cta;
+    cta += A.ops[i].ncta;
   }
   if (getenv("DT_XFER_DEBUG"))
     for (int i = 0; i < nops; i++)
