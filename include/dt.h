@@ -172,7 +172,7 @@ dt_status dt_type_deserialize(const void* in, size_t nbytes, dt_t* out);
 /* ------------------------------------------------------------------ GPU <-> GPU transfer */
 enum { DT_XFER_P2P = 0, DT_XFER_NCCL = 1 };
 typedef struct {
-  int64_t chunk_bytes; /* pipeline fragment size C (reading A15); 0 = default 1 MiB        */
+  int64_t chunk_bytes; /* pipeline fragment size C (reading A15); 0 = default 1 MiB; <= 1 GiB */
   int32_t depth;       /* ring slots D (fragments in flight) per (peer, channel), <= 256;
                           0 = auto: D*C >= 8 MiB, at least 4 slots (NCCL mode: 4)      */
   int32_t mode;        /* DT_XFER_P2P (pack straight into the peer's ring over NVLink) or

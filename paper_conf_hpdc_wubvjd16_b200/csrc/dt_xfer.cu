@@ -245,9 +245,11 @@ struct PieceIt {
   // (fewer than gs when the whole message is shorter than one slot)
   __device__ __forceinline__ bool init(int role, int64_t n_, int64_t C_, int D_, int gs_, int rep_, int ncta_, int j_) {
     n = n_; C = C_; D = D_; gs = gs_; rep = rep_; ncta = ncta_; j = j_;
-    Cs = C / gs;
+    // (one thread runs this on the critical path of a short message: 32-bit arithmetic
+    // where the values allow -- gs is a power of two, min(n, C) <= C < 2^31)
+    Cs = C >> (__ffs(gs) - 1);
     K = (int)((n + C - 1) / C);
-    gu = (int)min((int64_t)gs, ((n < C ? n : C) + Cs - 1) / Cs);
+    gu = (int)min((uint32_t)gs, ((uint32_t)(n < C ? n : C) + (uint32_t)Cs - 1u) / (uint32_t)Cs);
     if (gu < 1) gu = 1;
     const int npairs = gu * rep;
     one = ncta >= npairs;  // (either role: fewer CTAs than pairs take pairs j, j + ncta, ...)
@@ -357,6 +359,8 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   // have counted themselves done (op_done)
   const uint64_t seq = *(volatile const uint64_t*)X.seqp + 1;
   const bool sys = X.sys != 0;
+  PieceIt it;
+  bool more = X.role == 0 && it.init(0, X.n, X.chunk, X.depth, X.gs, X.rep, X.ncta, j);
   if (threadIdx.x == 0) {
     xtrace(A, op, j, kTracePieces - 1, 1);  // setup done
     uint64_t v = 0;
@@ -415,8 +419,8 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   }
   __syncthreads();
   if (threadIdx.x == 0) xtrace(A, op, j, kTracePieces - 1, 2);  // handshake done
-  PieceIt it;
-  bool more = it.init(X.role, n, X.chunk, X.depth, s_gs, s_rep, X.ncta, j);
+  // (a sender's geometry is its own: its piece sequence was set up before the handshake)
+  if (X.role == 1) more = it.init(X.role, n, X.chunk, X.depth, s_gs, s_rep, X.ncta, j);
   if (threadIdx.x < 32) {  // ---- control warp
     if (threadIdx.x != 0) return;
     // Event loop over two conditions, never blocking on one while the other could
@@ -669,6 +673,9 @@ static void fill_opts(dt_xfer_opts& o, const dt_xfer_opts* in) {
     o.ctas = in->ctas;
   }
   o.chunk_bytes = (o.chunk_bytes + 511) & ~int64_t(511);
+  // a fragment is a ring slot: <= 1 GiB (the transfer kernel's piece arithmetic is 32-bit
+  // within a fragment)
+  o.chunk_bytes = std::min<int64_t>(o.chunk_bytes, int64_t(1) << 30);
   if ((!in || in->depth <= 0) && o.mode == DT_XFER_NCCL) {
     o.depth = 4;  // NCCL mode: depth = staging buffers of the pack/net/unpack overlap
   } else if (!in || in->depth <= 0) {

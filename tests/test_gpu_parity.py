@@ -356,6 +356,43 @@ def test_full_size_sampled_c5_large(torch_cuda):
     del gaps
 
 
+def test_full_size_sampled_c5b_1g_gpu_flatten(torch_cuda):
+    """C5b at 1 GiB (3.0e7 irregular 4..64-byte blocks) committed through the GPU-side
+    flattening (f2, the default for lists this long) and packed / unpacked by the
+    block-span kernel: 200k sampled stream bytes against the oracle's per-position
+    addresses, the unpack -> pack round trip, and sampled gap bytes left untouched."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c5b_irregular(1 << 30)
+    ot = oracle.from_recipe(rec)
+    t = dt.from_recipe(rec).commit()
+    fi = t.form()
+    assert fi.tsize == ot.size == 1 << 30
+    src_h = fill_bytes(parent, 0x5EED0015)
+    src = _dev(torch, src_h)
+    n = t.size
+    out = torch.empty(n, dtype=torch.uint8, device="cuda")
+    dt.pack(t, 1, src, out)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(15)
+    ps = np.unique(np.concatenate([rng.integers(0, n, size=200000), [0, n - 1]]))
+    addr = oracle.addr_of(ot, 1, ps)
+    got = out[torch.from_numpy(ps).cuda()].cpu().numpy()
+    assert np.array_equal(got, src_h[org + addr])
+    del src
+    dst = torch.full((parent,), 0xA5, dtype=torch.uint8, device="cuda")
+    dt.unpack(t, 1, out, dst)
+    back = torch.empty_like(out)
+    dt.pack(t, 1, dst, back)
+    torch.cuda.synchronize()
+    assert torch.equal(back, out)
+    lens, disp = rec[1], rec[2]
+    gap_at = disp[:-1] + lens[:-1]
+    has_gap = np.flatnonzero(disp[1:] > gap_at)[:: 101][:20000]
+    assert len(has_gap) > 1000
+    assert np.all(dst[torch.from_numpy(gap_at[has_gap]).cuda()].cpu().numpy() == 0xA5)
+
+
 # ------------------------------------------------------------------ record-span kernel (k_rec)
 REC_TYPES = {
     # C5 particle records (G = 4): blocks (0,4),(8,52) of a 64-byte span
