@@ -220,6 +220,17 @@ def test_every_kernel_family(torch_cuda, kind, name, monkeypatch):
     check_pack_unpack(torch_cuda, rec, org, parent, pos=20, nbytes=size - 37)
 
 
+@pytest.mark.parametrize("extent", [8, 2, 40])
+def test_resume_overlapping_instances(torch_cuda, extent):
+    """count > 1 instances whose extent is smaller than their size (overlapping, pack-only)
+    or larger: every kernel resumes at stream position p in instance p // size
+    (the oracle pin test_pos_resume_overlapping_instances fixes the closed form)."""
+    rec = ("resized", ("contiguous", 4, ("basic", "INT32")), 0, extent)
+    for count in (3, 7):
+        for pos, nbytes in ((0, None), (1, 30), (16, 16), (20, 100), (47, 5)):
+            check_or_overlap(torch_cuda, rec, 16, 16 + count * 64 + 64, count, pos=pos, nbytes=nbytes)
+
+
 def test_unpack_rejects_overlap(torch_cuda):
     import torch
     from paper_conf_hpdc_wubvjd16_b200 import dt

@@ -319,6 +319,27 @@ def test_pos_len_concatenation():
     assert len(oracle.pack(t, 2, buf, org, len(whole) + 5, 10)) == 0
 
 
+@pytest.mark.parametrize("extent", [8, 16, 40, 2])
+def test_pos_resume_overlapping_instances(extent):
+    """Resuming at a stream position with count > 1 must seek instances by SIZE: instance
+    k covers stream bytes [k*size, (k+1)*size) and sits at k*extent in memory (MPI-3.1
+    §4.1.6; the fragment restart of [L18:c1430 §3.2]).  Closed form for a contiguous
+    element resized to extent e (e < size: overlapping instances, legal to pack):
+    stream byte p comes from address (p // size)*e + p % size."""
+    size = 16
+    rec = ("resized", ("contiguous", 4, ("basic", "INT32")), 0, extent)
+    t = oracle.from_recipe(rec)
+    count = 5
+    n = count * size
+    buf = fill_bytes(n * 4, 21)
+    p = np.arange(n)
+    whole = buf[(p // size) * extent + p % size]
+    assert np.array_equal(oracle.pack(t, count, buf), whole)
+    for pos in (1, 15, 16, 20, 33, 47, 64, 79):
+        for ln in (1, 7, 16, 30, n):
+            assert np.array_equal(oracle.pack(t, count, buf, 0, pos, ln), whole[pos:pos + ln]), (pos, ln)
+
+
 def test_multithreaded_equals_single():
     rec, _, nbytes = c2_lower_triangle(300)
     t = oracle.from_recipe(rec)
@@ -346,9 +367,11 @@ def test_addr_of_matches_typemap():
 
 
 def test_oracle_mutants_killed():
-    """Each deliberate bug in oracle.c (tools/oracle_mutants.py: extent-vs-size
-    scaling in vector/indexed/hindexed/contiguous, a dropped j*extent term, the struct
-    ε rule) makes at least one pin above fail."""
+    """Each deliberate bug in oracle.c (tools/oracle_mutants.py: extent-vs-size scaling
+    in the constructors' bounds and in the typemap walk, a dropped j*extent term, the
+    struct ε rule, subarray order and starts, instance placement, fragment resume,
+    pos handling of pack/unpack, resized/marker/true bounds) makes at least one pin above
+    fail, and the unmutated oracle passes them in the tool's scratch copy."""
     import subprocess
     import sys
     tool = os.path.join(os.path.dirname(HERE), "tools", "oracle_mutants.py")
