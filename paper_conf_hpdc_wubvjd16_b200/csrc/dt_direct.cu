@@ -498,7 +498,9 @@ dt_status dt_xplan_connect(dt_xplan_t p, const void* blobs, const size_t* sizes)
     }
     total += n;
   }
-  // launch shape: CTA 0 controls, the sends share the co-resident rest by bytes
+  // launch shape: CTA 0 controls, the sends share the co-resident rest by bytes x a
+  // per-family cost (G-byte word gathers/scatters move bytes ~16/G times slower per CTA
+  // than long runs: the C4 x faces next to the y/z faces)
   A.wt_off = any_stage ? kStageBufs * kStageTile : 0;
   p->smem = (size_t)A.wt_off + wt_bytes;
   CUD(cudaFuncSetAttribute(k_direct, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)std::max<size_t>(p->smem, 1)));
@@ -512,12 +514,15 @@ dt_status dt_xplan_connect(dt_xplan_t p, const void* blobs, const size_t* sizes)
     set_error("dt_xplan_connect: %d sends need more co-resident CTAs than the device offers", A.nops);
     return DT_ERR_UNSUPPORTED;
   }
+  auto cost = [](const DOp& X) { return (double)X.n * ((X.kind == 2 || X.kind == 4) ? 16.0 / X.g : 1.0); };
+  double ctot = 0;
+  for (int i = 0; i < A.nops; i++) ctot += cost(A.ops[i]);
   int next = 1;
   int left = budget;
   for (int i = 0; i < A.nops; i++) {
     DOp& X = A.ops[i];
     const int rest = A.nops - i - 1;  // keep one CTA for every later send
-    int want = total > 0 ? (int)((double)budget * (double)X.n / (double)total) : 1;
+    int want = ctot > 0 ? (int)((double)budget * cost(X) / ctot) : 1;
     want = std::max(1, std::min(want, (int)std::max<int64_t>(1, X.n / 16384)));
     want = std::min(want, left - rest);
     X.cta0 = next;
