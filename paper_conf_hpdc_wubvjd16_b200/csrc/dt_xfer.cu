@@ -340,6 +340,10 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   const XOp& X = A.ops[op];
   const int j = (int)blockIdx.x - X.cta0;
   const bool sleep_ok = !(A.flags & 2);
+  // programmatic dependent launch (DT_XFER_PDL): the next transfer on the stream may start
+  // its launch and setup now; it waits (griddepcontrol.wait below) before touching memory
+  // this kernel or any earlier one writes.  (No-ops without PDL.)
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   if (threadIdx.x == 0) xtrace(A, op, j, kTracePieces - 1, 0);  // (diagnostics: kernel entry)
 
   if (X.kind == 2 || X.kind == 4)
@@ -355,12 +359,13 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
                      default: rec_maps<false, 16>(R, omap); break; }
     }
   }
+  // prerequisite grids (the previous message's kernel, whatever produced the send buffer)
+  // have completed and their memory is visible from here on
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   // every CTA of the op reads the same number: it is advanced only after all of them
   // have counted themselves done (op_done)
   const uint64_t seq = *(volatile const uint64_t*)X.seqp + 1;
   const bool sys = X.sys != 0;
-  PieceIt it;
-  bool more = X.role == 0 && it.init(0, X.n, X.chunk, X.depth, X.gs, X.rep, X.ncta, j);
   if (threadIdx.x == 0) {
     xtrace(A, op, j, kTracePieces - 1, 1);  // setup done
     uint64_t v = 0;
@@ -419,8 +424,8 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   }
   __syncthreads();
   if (threadIdx.x == 0) xtrace(A, op, j, kTracePieces - 1, 2);  // handshake done
-  // (a sender's geometry is its own: its piece sequence was set up before the handshake)
-  if (X.role == 1) more = it.init(X.role, n, X.chunk, X.depth, s_gs, s_rep, X.ncta, j);
+  PieceIt it;
+  bool more = it.init(X.role, n, X.chunk, X.depth, s_gs, s_rep, X.ncta, j);
   if (threadIdx.x < 32) {  // ---- control warp
     if (threadIdx.x != 0) return;
     // Event loop over two conditions, never blocking on one while the other could
@@ -1184,8 +1189,30 @@ static dt_status issue_p2p(dt_comm_s* c, const std::vector<PendingOp>& ops, cuda
     std::memcpy(A2.ops, A.ops, sizeof(XOp) * 2);
     args[0] = &A2;
   }
-  if (coop) CU(cudaLaunchCooperativeKernel(kfn, dim3(cta), dim3(kXferThreads), args, smem, s));
-  else CU(cudaLaunchKernel(kfn, dim3(cta), dim3(kXferThreads), args, smem, s));
+  // DT_XFER_PDL=1: a plain launch with programmatic stream serialisation, so back-to-back
+  // transfers overlap the next kernel's launch and setup with the current one (the grid is
+  // sized to fit co-resident, as for DT_XFER_NOCOOP; no cooperative guarantee);
+  // DT_XFER_PDL=2: cooperative as well
+  static const bool pdl = getenv("DT_XFER_PDL") && atoi(getenv("DT_XFER_PDL")) > 0;
+  if (pdl) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(cta);
+    cfg.blockDim = dim3(kXferThreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[2];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    at[1].id = cudaLaunchAttributeCooperative;  // DT_XFER_PDL=2: keep the co-residency guarantee too
+    at[1].val.cooperative = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = atoi(getenv("DT_XFER_PDL")) >= 2 && coop ? 2 : 1;
+    CU(cudaLaunchKernelExC(&cfg, kfn, args));
+  } else if (coop) {
+    CU(cudaLaunchCooperativeKernel(kfn, dim3(cta), dim3(kXferThreads), args, smem, s));
+  } else {
+    CU(cudaLaunchKernel(kfn, dim3(cta), dim3(kXferThreads), args, smem, s));
+  }
   if (tr) {
     bool hung = false;
     for (int w = 0; cudaStreamQuery(s) == cudaErrorNotReady; w++) {
