@@ -665,7 +665,7 @@ def xfer_sweep(ws, rank, local, chunks, depths, mode_name, ctas, steps, warmup, 
     A = torch.from_numpy(fill_bytes(parent, seed_for(3) + rank)).to(dev)
     B = torch.full((parent,), 0xA5, dtype=torch.uint8, device=dev)
     s = torch.cuda.current_stream()
-    mode = dt.XFER_NCCL if mode_name == "nccl" else dt.XFER_P2P
+    mode = {"nccl": dt.XFER_NCCL, "ce": dt.XFER_CE}.get(mode_name, dt.XFER_P2P)
     results = []
     if mode_name == "direct":  # persistent direct plan: chunk and depth do not apply
         chunks, depths = [0], [0]
@@ -991,7 +991,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--workload", default="c2", choices=["c2", "xfer", "halo", "sweep"])
     ap.add_argument("--sweep", default="all", help="--workload sweep: comma-separated config names or 'all'")
-    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "direct", "hybrid"],
+    ap.add_argument("--xfer-mode", default="p2p", choices=["p2p", "nccl", "ce", "direct", "hybrid"],
                     help="p2p ring pipeline, NCCL double buffering, a persistent direct plan (dt_xplan), "
                          "or (halo only) hybrid: y/z faces direct, x faces through the ring")
     ap.add_argument("--xfer-workload", default="c3", choices=["c3", "c5", "c5b"])

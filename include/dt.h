@@ -170,13 +170,15 @@ dt_status dt_type_serialize(dt_t t, void* out, size_t* nbytes);
 dt_status dt_type_deserialize(const void* in, size_t nbytes, dt_t* out);
 
 /* ------------------------------------------------------------------ GPU <-> GPU transfer */
-enum { DT_XFER_P2P = 0, DT_XFER_NCCL = 1 };
+enum { DT_XFER_P2P = 0, DT_XFER_NCCL = 1, DT_XFER_CE = 2 };
 typedef struct {
   int64_t chunk_bytes; /* pipeline fragment size C (reading A15); 0 = default 1 MiB; <= 1 GiB */
   int32_t depth;       /* ring slots D (fragments in flight) per (peer, channel), <= 256;
                           0 = auto: D*C >= 8 MiB, at least 4 slots (NCCL mode: 4)      */
-  int32_t mode;        /* DT_XFER_P2P (pack straight into the peer's ring over NVLink) or
-                          DT_XFER_NCCL (double-buffered ncclSend/ncclRecv of packed chunks) */
+  int32_t mode;        /* DT_XFER_P2P (pack straight into the peer's ring over NVLink),
+                          DT_XFER_NCCL (double-buffered ncclSend/ncclRecv of packed chunks) or
+                          DT_XFER_CE (pack into local staging, copy-engine copy into the peer's
+                          ring, stream-ordered flag kernels; host-driven, a comparator) */
   int32_t ctas;        /* CTAs per direction for the P2P pipeline kernel; 0 = default      */
   int32_t flags;       /* bit 0: loopback (dest = source = self) through the ring pipeline
                           instead of the fused datatype -> datatype copy (dt_copy)        */

@@ -524,6 +524,31 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
   }
 }
 
+// ------------------------------------------------------------------ copy-engine mode
+// DT_XFER_CE: the paper's receiver staging with the copy engine as the wire
+// ([L20:c4255 §4.1]): the sender packs each fragment into a local staging
+// slot (a pack kernel), the copy engine moves it into the receiver's ring slot
+// (cudaMemcpyAsync to the IPC-mapped peer address), and stream-ordered one-thread
+// kernels publish / await the same tag flags the P2P kernel uses.  Host-driven: every
+// fragment is a few stream operations on three internal streams.
+__global__ void k_ce_wait(const uint64_t* __restrict__ p, uint64_t v, int sys, int64_t timeout_ns, int32_t* err) {
+  if (threadIdx.x != 0) return;
+  const uint64_t t0 = gtimer();
+  while (ld_acquire(p, sys != 0) < v) {
+    __nanosleep(64);
+    if ((int64_t)(gtimer() - t0) > timeout_ns) {
+      atomicCAS(err, 0, XERR_TIMEOUT);
+      return;
+    }
+  }
+}
+// p[1..nx] = x[0..nx) (relaxed), then p[0] = v (release)
+__global__ void k_ce_signal(uint64_t* p, uint64_t v, int sys, uint64_t x0, int nx) {
+  if (threadIdx.x != 0) return;
+  if (nx > 0) p[1] = x0;
+  st_release(p, v, sys != 0);
+}
+
 // ------------------------------------------------------------------ NCCL (dlopen)
 typedef struct { char internal[128]; } ncclUniqueId_t;
 typedef void* ncclComm_t;
@@ -616,6 +641,10 @@ struct dt_comm_s {
   // group
   bool in_group = false;
   std::vector<PendingOp> pending;
+  // CE mode: host sequence numbers per (role, peer, channel) and the last tag published
+  // into each of a peer's ring slots (a slot is reused once its ack has reached that tag)
+  std::vector<uint64_t> hseq;
+  std::vector<uint64_t> slot_tag;  // [nranks][nch][depth]
   // NCCL mode
   ncclComm_t nccl = nullptr;
   cudaStream_t s_pack = nullptr, s_net = nullptr, s_unpack = nullptr;
@@ -720,7 +749,7 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
   c->nranks = nranks;
   c->device = device;
   fill_opts(c->o, o);
-  if (c->o.mode != DT_XFER_P2P && c->o.mode != DT_XFER_NCCL) {
+  if (c->o.mode != DT_XFER_P2P && c->o.mode != DT_XFER_NCCL && c->o.mode != DT_XFER_CE) {
     delete c;
     set_error("dt_comm_init: unknown mode");
     return DT_ERR_ARG;
@@ -737,7 +766,7 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
   }
   c->ring_bytes = (size_t)nranks * c->nch * c->o.depth * (size_t)c->o.chunk_bytes;
   c->flag_words = c->err_idx() + 1;
-  if (c->o.mode == DT_XFER_P2P) {
+  if (c->o.mode == DT_XFER_P2P || c->o.mode == DT_XFER_CE) {
     e = cudaMalloc(&c->ring, c->ring_bytes);
     if (e == cudaSuccess) e = cudaMalloc(&c->flags, c->flag_words * 8);
     if (e == cudaSuccess) e = cudaMemset(c->flags, 0, c->flag_words * 8);
@@ -753,6 +782,20 @@ dt_status dt_comm_init(int rank, int nranks, const void* nccl_unique_id, int dev
       cudaFree(c->ddone);
       delete c;
       return cufail(e, "dt_comm_init alloc");
+    }
+    if (c->o.mode == DT_XFER_CE) {
+      const size_t st = (size_t)kMaxOps * c->o.depth * (size_t)c->o.chunk_bytes;
+      e = cudaMalloc(&c->stage, st);
+      if (e == cudaSuccess) e = cudaMalloc(&c->szbuf, sizeof(int64_t) * 2 * kMaxOps);
+      if (e == cudaSuccess) e = cudaMallocHost(&c->szhost, sizeof(int64_t) * 2 * kMaxOps);
+      if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s_pack, cudaStreamNonBlocking);
+      if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s_net, cudaStreamNonBlocking);
+      if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->s_unpack, cudaStreamNonBlocking);
+      if (e != cudaSuccess) return cufail(e, "dt_comm_init ce alloc");
+      c->ev.resize((size_t)kMaxOps * c->o.depth * 3 + 2);
+      for (auto& x : c->ev) cudaEventCreateWithFlags(&x, cudaEventDisableTiming);
+      c->hseq.assign((size_t)2 * nranks * c->nch, 0);
+      c->slot_tag.assign((size_t)nranks * c->nch * c->o.depth, 0);
     }
   } else {
     if (!load_nccl()) {
@@ -829,7 +872,7 @@ dt_status dt_comm_local_handle(dt_comm_t c, void* out, size_t* nbytes) {
   }
   b.ring_ptr = (uint64_t)(uintptr_t)c->ring;
   b.flags_ptr = (uint64_t)(uintptr_t)c->flags;
-  if (c->o.mode == DT_XFER_P2P) {
+  if (c->o.mode == DT_XFER_P2P || c->o.mode == DT_XFER_CE) {
     CU(cudaIpcGetMemHandle(&b.ring_h, c->ring));
     CU(cudaIpcGetMemHandle(&b.flags_h, c->flags));
   }
@@ -843,7 +886,7 @@ dt_status dt_comm_connect(dt_comm_t c, const void* all, size_t per) {
     set_error("dt_comm_connect: bad argument");
     return DT_ERR_ARG;
   }
-  if (c->o.mode != DT_XFER_P2P) {
+  if (c->o.mode == DT_XFER_NCCL) {
     c->connected = true;
     return DT_OK;
   }
@@ -1334,6 +1377,134 @@ static dt_status issue_nccl(dt_comm_s* c, const std::vector<PendingOp>& ops, cud
   return DT_OK;
 }
 
+// Copy-engine mode (DT_XFER_CE, see k_ce_wait): per message a header {seq, n} in the
+// receiver's flags (the receiver's host reads n: its unpack launches need the fragment
+// lengths), then per fragment k (slot k % D): sender -- pack into its staging slot
+// (s_pack), wait until the receiver acked the slot's previous tag, copy-engine copy into
+// the receiver's ring slot and publish the ready tag (s_net); receiver -- wait for the
+// ready tag, unpack from its ring slot, publish the ack tag into the sender's flags
+// (s_unpack).  Tags are the P2P kernel's (seq, round) tags; a slot's first piece word
+// carries them.
+static dt_status issue_ce(dt_comm_s* c, const std::vector<PendingOp>& ops, cudaStream_t s) {
+  const int64_t C = c->o.chunk_bytes;
+  const int D = c->o.depth;
+  struct Side { const PendingOp* p; int peer, ch; uint64_t seq; int64_t n; };
+  std::vector<Side> sends, recvs;
+  std::vector<int> sch(c->nranks, 0), rch(c->nranks, 0);
+  for (const auto& p : ops) {
+    if (p.dest >= 0) {
+      const int ch = sch[p.dest]++;
+      if (ch >= c->nch) { set_error("dt_sendrecv: more than %d messages to one peer in a group", c->nch); return DT_ERR_UNSUPPORTED; }
+      uint64_t& q = c->hseq[((size_t)0 * c->nranks + p.dest) * c->nch + ch];
+      sends.push_back({&p, p.dest, ch, ++q, p.scount * p.stype->size});
+    }
+    if (p.source >= 0) {
+      const int ch = rch[p.source]++;
+      if (ch >= c->nch) { set_error("dt_sendrecv: more than %d messages from one peer in a group", c->nch); return DT_ERR_UNSUPPORTED; }
+      uint64_t& q = c->hseq[((size_t)1 * c->nranks + p.source) * c->nch + ch];
+      recvs.push_back({&p, p.source, ch, ++q, 0});
+    }
+  }
+  if ((int)sends.size() > kMaxOps || (int)recvs.size() > kMaxOps) {
+    set_error("dt_sendrecv: too many ops in one group");
+    return DT_ERR_UNSUPPORTED;
+  }
+  const char* to = getenv("DT_TIMEOUT_MS");
+  const int64_t tmo = (int64_t)(to ? atoll(to) : 30000) * 1000000ll;
+  int32_t* err = reinterpret_cast<int32_t*>(c->flags + c->err_idx());
+  cudaEvent_t* ev = c->ev.data();
+  cudaEvent_t ev_start = ev[(size_t)kMaxOps * D * 3], ev_end = ev[(size_t)kMaxOps * D * 3 + 1];
+  CU(cudaEventRecord(ev_start, s));
+  CU(cudaStreamWaitEvent(c->s_pack, ev_start, 0));
+  CU(cudaStreamWaitEvent(c->s_net, ev_start, 0));
+  CU(cudaStreamWaitEvent(c->s_unpack, ev_start, 0));
+  // headers first (a loopback receiver below waits for them on the host)
+  for (const Side& x : sends) {
+    uint64_t* hdr = c->peer_flags[x.peer] + c->hdr_idx(c->rank, x.ch);
+    k_ce_signal<<<1, 32, 0, c->s_net>>>(hdr, x.seq, !c->same_dev[x.peer], (uint64_t)x.n, 1);
+  }
+  CU(cudaGetLastError());
+  for (size_t i = 0; i < recvs.size(); i++) {
+    const Side& x = recvs[i];
+    const uint64_t* hdr = c->flags + c->hdr_idx(x.peer, x.ch);
+    k_ce_wait<<<1, 32, 0, c->s_unpack>>>(hdr, x.seq, !c->same_dev[x.peer], tmo, err);
+    CU(cudaMemcpyAsync(c->szhost + kMaxOps + i, hdr + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, c->s_unpack));
+  }
+  CU(cudaGetLastError());
+  if (!recvs.empty()) CU(cudaStreamSynchronize(c->s_unpack));
+  for (size_t i = 0; i < recvs.size(); i++) {
+    recvs[i].n = c->szhost[kMaxOps + i];
+    const int64_t cap = recvs[i].p->rcount * recvs[i].p->rtype->size;
+    if (recvs[i].n > cap) {
+      // consume the message without unpacking it: ack every fragment with its final tag
+      const int64_t K = (recvs[i].n + C - 1) / C;
+      for (int64_t k = std::max<int64_t>(0, K - D); k < K; k++)
+        k_ce_signal<<<1, 32, 0, c->s_unpack>>>(c->peer_flags[recvs[i].peer] + c->ack_idx(c->rank, recvs[i].ch) +
+                                                   (size_t)(k % D) * kMaxSub,
+                                               xtag(recvs[i].seq, k / D), !c->same_dev[recvs[i].peer], 0, 0);
+      set_error("dt_sendrecv: message of %lld bytes truncated by a %lld-byte receive", (long long)recvs[i].n,
+                (long long)cap);
+      recvs[i].n = -1;
+    }
+  }
+  bool trunc = false;
+  for (const Side& x : recvs) trunc = trunc || x.n < 0;
+  int64_t K = 0;
+  for (const Side& x : sends) K = std::max(K, (x.n + C - 1) / C);
+  for (const Side& x : recvs) K = std::max(K, (x.n + C - 1) / C);
+  const size_t slot_span = (size_t)kMaxOps * C;
+  auto ev_packed = [&](size_t i, int slot) { return ev[(i * D + slot) * 3]; };
+  auto ev_sent = [&](size_t i, int slot) { return ev[(i * D + slot) * 3 + 1]; };
+  for (int64_t k = 0; k < K; k++) {
+    const int slot = (int)(k % D);
+    const int64_t round = k / D;
+    for (size_t i = 0; i < sends.size(); i++) {
+      const Side& x = sends[i];
+      int64_t pos = k * C, len = std::min<int64_t>(C, x.n - pos);
+      if (len <= 0) continue;
+      uint8_t* st_slot = c->stage + slot * slot_span + i * C;
+      if (k >= D) CU(cudaStreamWaitEvent(c->s_pack, ev_sent(i, slot), 0));  // staging slot copied out
+      dt_status st = dt_pack(x.p->stype, x.p->scount, x.p->sbuf, st_slot, pos, &len, c->s_pack);
+      if (st != DT_OK) return st;
+      CU(cudaEventRecord(ev_packed(i, slot), c->s_pack));
+      CU(cudaStreamWaitEvent(c->s_net, ev_packed(i, slot), 0));
+      // the receiver's ring slot is free once it acked the last tag published into it
+      uint64_t& last = c->slot_tag[((size_t)x.peer * c->nch + x.ch) * D + slot];
+      const bool sys = !c->same_dev[x.peer];
+      if (last) k_ce_wait<<<1, 32, 0, c->s_net>>>(c->flags + c->ack_idx(x.peer, x.ch) + (size_t)slot * kMaxSub, last,
+                                                   sys, tmo, err);
+      uint8_t* dst = c->peer_ring[x.peer] + c->ring_off(c->rank, x.ch) + (size_t)slot * C;
+      CU(cudaMemcpyAsync(dst, st_slot, (size_t)len, cudaMemcpyDeviceToDevice, c->s_net));
+      last = xtag(x.seq, round);
+      k_ce_signal<<<1, 32, 0, c->s_net>>>(c->peer_flags[x.peer] + c->ready_idx(c->rank, x.ch) + (size_t)slot * kMaxSub,
+                                          last, sys, 0, 0);
+      CU(cudaGetLastError());
+      CU(cudaEventRecord(ev_sent(i, slot), c->s_net));
+    }
+    for (size_t i = 0; i < recvs.size(); i++) {
+      const Side& x = recvs[i];
+      int64_t pos = k * C, len = std::min<int64_t>(C, x.n - pos);
+      if (x.n < 0 || len <= 0) continue;
+      const bool sys = !c->same_dev[x.peer];
+      k_ce_wait<<<1, 32, 0, c->s_unpack>>>(c->flags + c->ready_idx(x.peer, x.ch) + (size_t)slot * kMaxSub,
+                                           xtag(x.seq, round), sys, tmo, err);
+      dt_status st = dt_unpack(x.p->rtype, x.p->rcount, c->ring + c->ring_off(x.peer, x.ch) + (size_t)slot * C,
+                               x.p->rbuf, pos, &len, c->s_unpack);
+      if (st != DT_OK) return st;
+      k_ce_signal<<<1, 32, 0, c->s_unpack>>>(c->peer_flags[x.peer] + c->ack_idx(c->rank, x.ch) + (size_t)slot * kMaxSub,
+                                             xtag(x.seq, round), sys, 0, 0);
+      CU(cudaGetLastError());
+    }
+  }
+  CU(cudaEventRecord(ev_end, c->s_pack));
+  CU(cudaStreamWaitEvent(s, ev_end, 0));
+  CU(cudaEventRecord(ev_end, c->s_net));
+  CU(cudaStreamWaitEvent(s, ev_end, 0));
+  CU(cudaEventRecord(ev_end, c->s_unpack));
+  CU(cudaStreamWaitEvent(s, ev_end, 0));
+  return trunc ? DT_ERR_TRUNCATE : DT_OK;
+}
+
 static dt_status validate(dt_comm_s* c, const PendingOp& p) {
   if (p.dest >= c->nranks || p.source >= c->nranks || p.dest < -1 || p.source < -1) {
     set_error("dt_sendrecv: rank out of range");
@@ -1373,6 +1544,7 @@ static dt_status validate(dt_comm_s* c, const PendingOp& p) {
 static dt_status issue(dt_comm_s* c, const std::vector<PendingOp>& ops_in, void* stream) {
   cudaStream_t s = (cudaStream_t)stream;
   if (c->o.mode == DT_XFER_NCCL) return issue_nccl(c, ops_in, s);
+  if (c->o.mode == DT_XFER_CE) return issue_ce(c, ops_in, s);
   if (c->o.flags & 1) return issue_p2p(c, ops_in, s);
   std::vector<PendingOp> ops = ops_in;
   std::vector<size_t> sends, recvs;

@@ -19,7 +19,7 @@ _lib = None
 STATUS = {0: "DT_OK", 1: "DT_ERR_ARG", 2: "DT_ERR_NOT_COMMITTED", 3: "DT_ERR_OVERLAP", 4: "DT_ERR_TRUNCATE",
           5: "DT_ERR_CUDA", 6: "DT_ERR_NCCL", 7: "DT_ERR_NOMEM", 8: "DT_ERR_TIMEOUT", 9: "DT_ERR_UNSUPPORTED"}
 BASIC = {"BYTE": 0, "CHAR": 1, "INT8": 2, "INT16": 3, "INT32": 4, "INT64": 5, "FLOAT": 6, "DOUBLE": 7}
-XFER_P2P, XFER_NCCL = 0, 1
+XFER_P2P, XFER_NCCL, XFER_CE = 0, 1, 2
 
 
 class DTError(RuntimeError):

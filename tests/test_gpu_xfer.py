@@ -198,7 +198,7 @@ def _free_port():
     return p
 
 
-def _ipc_worker(rank, port, q):
+def _ipc_worker(rank, port, q, mode=0):
     try:
         import torch
         import torch.distributed as tdist
@@ -208,7 +208,7 @@ def _ipc_worker(rank, port, q):
         tdist.init_process_group("gloo", rank=rank, world_size=2)
         torch.cuda.set_device(0)
         from paper_conf_hpdc_wubvjd16_b200 import dt
-        comm = dt.Comm.from_process_group(device=0, chunk_bytes=256 << 10, depth=2, ctas=4)
+        comm = dt.Comm.from_process_group(device=0, chunk_bytes=256 << 10, depth=2, ctas=4, mode=mode)
         rec, org, parent = c2_lower_triangle(1024)
         t = dt.from_recipe(rec).commit()
         mine = fill_bytes(parent, 100 + rank)
@@ -231,13 +231,16 @@ def _ipc_worker(rank, port, q):
         q.put((rank, traceback.format_exc() + repr(e)))
 
 
-def test_two_processes_one_gpu_ipc(torch_cuda):
-    """Two ranks (processes) exchange triangles through IPC-mapped rings on one GPU."""
+@pytest.mark.parametrize("mode", [0, 2], ids=["p2p", "ce"])
+def test_two_processes_one_gpu_ipc(torch_cuda, mode):
+    """Two ranks (processes) exchange triangles through IPC-mapped rings on one GPU (the
+    P2P kernel, or the copy-engine mode: staging, cudaMemcpyAsync into the peer ring,
+    stream-ordered flag kernels)."""
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_ipc_worker, args=(r, port, q)) for r in range(2)]
+    ps = [ctx.Process(target=_ipc_worker, args=(r, port, q, mode)) for r in range(2)]
     for p in ps:
         p.start()
     res = [q.get(timeout=300) for _ in ps]
@@ -675,4 +678,37 @@ def test_ring_exchange_graph_replay(torch_cuda):
         oracle.sendrecv(ot, 1, src_h, ot, 1, exp_b, org, org)
         assert np.array_equal(B.cpu().numpy(), exp_b), r
         assert torch.equal(b2, a2), r
+    comm.free()
+
+
+@pytest.mark.parametrize("chunk,depth", [(64 << 10, 2), (256 << 10, 4), (1 << 20, 0)])
+def test_copy_engine_mode_loopback(torch_cuda, chunk, depth):
+    """DT_XFER_CE ([L20:c4255 §4.1] receiver staging with the copy engine as the wire):
+    block-cyclic exchanges repeated on one channel (ring slots reused across rounds and
+    messages), different send/receive layouts, short-block particles, and truncation
+    (reported by dt_sendrecv; the channel stays usable)."""
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    comm = dt.Comm(0, 1, 0, chunk_bytes=chunk, depth=depth, mode=dt.XFER_CE)
+    rec, org, parent = c3_block_cyclic(2048, 64)
+    for s_ in range(3):
+        _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent, seed=20 + s_)
+    v, vorg, vpar = c1_submatrix(256, 1024, 1, 1)
+    contig = ("contiguous", 256 * 256, ("basic", "DOUBLE"))
+    _loop_check(torch_cuda, comm, v, vorg, vpar, contig, 0, 256 * 256 * 8)
+    tri, _, tpar = c2_lower_triangle(600)
+    n = 600 * 601 // 2
+    _loop_check(torch_cuda, comm, tri, 0, tpar, ("contiguous", n + 100, ("basic", "DOUBLE")), 0, (n + 100) * 8)
+    prec, porg, ppar = c5_particles(1 << 20)
+    _loop_check(torch_cuda, comm, prec, porg, ppar, prec, porg, ppar)
+    import torch
+    big = dt.Type.basic("BYTE").contiguous(3 * chunk + 5).commit()
+    small = dt.Type.basic("BYTE").contiguous(3 * chunk).commit()
+    sb = torch.randint(0, 255, (3 * chunk + 5,), dtype=torch.uint8, device="cuda")
+    rb = torch.full((3 * chunk + 5,), 0xA5, dtype=torch.uint8, device="cuda")
+    with pytest.raises(dt.DTError) as e:
+        comm.sendrecv(sb, 1, big, 0, rb, 1, small, 0)
+    assert e.value.name == "DT_ERR_TRUNCATE"
+    torch.cuda.synchronize()
+    assert torch.all(rb == 0xA5)
+    _loop_check(torch_cuda, comm, rec, org, parent, rec, org, parent, seed=30)
     comm.free()
