@@ -503,7 +503,7 @@ def run_multi(args):
     exchange between pairs (r, r^1) through dt_sendrecv's P2P ring (best of 1 and 4
     MiB fragments, auto depth); beside it, in the same run, the same bytes contiguous
     through the same path (the paper's "C" comparator, [L26:c977 §5.2]) and through
-    torch/NCCL, the NCCL mode and the direct plan on C3, the C4 halo (ring and direct)
+    torch/NCCL, the NCCL mode, the copy-engine mode and the direct plan on C3, the C4 halo (ring and direct)
     and C5 pairs.  Replica C2 pack/unpack moves to a side field."""
     import torch
     os.environ.setdefault("DT_TIMEOUT_MS", "15000")
@@ -534,6 +534,7 @@ def run_multi(args):
     sub["contiguous_same_bytes"]["how"] = "dt_sendrecv of 128 MiB contiguous bytes, same ring (paper's C)"
     sub["nccl_contiguous"] = _guard(_torch_nccl_contig, ws, rank, local, payload, steps, w)
     sub["nccl_mode_c3"] = _guard(sweep1, "nccl", "c3", (4 << 20,), (4,))
+    sub["copy_engine_c3"] = _guard(sweep1, "ce", "c3", (4 << 20,))
     sub["direct_plan_c3"] = _guard(sweep1, "direct", "c3")
     sub["c4_halo_ring"] = _guard(_halo, ws, rank, local, "p2p", steps, w)
     sub["c4_halo_direct"] = _guard(_halo, ws, rank, local, "direct", steps, w)
