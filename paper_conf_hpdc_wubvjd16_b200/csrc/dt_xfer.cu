@@ -90,7 +90,8 @@ template <int NOPS>
 struct XArgsT {
   int32_t nops;
   int32_t wt_off;  // byte offset of the word table in dynamic smem (after the staging buffers)
-  int32_t flags;   // DT_XFER_FLAGS: bit1 = no sleep in polls, bit2 = SC system fence before each flag
+  int32_t flags;   // DT_XFER_FLAGS: 2 = no sleep in polls, 4 = SC system fence before each flag, 8 = no proxy
+                   // fence before TMA reads of a slot, 16 = one piece outstanding, 64 = publish every ack
   int32_t pad2;
   int64_t timeout_ns;
   uint64_t* trace;  // diagnostics (DT_XFER_TRACE): per-piece globaltimer stamps of the first CTAs
@@ -435,6 +436,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
     int i_acq = 0, i_rel = 0;
     int q_fi[2] = {0, 0};
     uint64_t q_tag[2] = {0, 0};
+    bool q_pub[2] = {true, true};
     uint64_t t_idle = 0;
     int ns = 0;
     while (more || i_rel < i_acq) {
@@ -443,7 +445,7 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
         xtrace(A, op, j, i_rel, 2);
         if (A.flags & 4) __threadfence_system();
         const int b = i_rel & 1;
-        st_release(X.role == 0 ? X.ready + q_fi[b] : X.ack + q_fi[b], q_tag[b], sys);
+        if (q_pub[b]) st_release(X.role == 0 ? X.ready + q_fi[b] : X.ack + q_fi[b], q_tag[b], sys);
         xtrace(A, op, j, i_rel, 3);
         i_rel++;
         progress = true;
@@ -460,6 +462,10 @@ __global__ void __launch_bounds__(kXferThreads, 1) k_xfer(const __grid_constant_
           const int b = i_acq & 1;
           q_fi[b] = fi;
           q_tag[b] = tag;
+          // an ack is read only by the same message's sender before it reuses the slot
+          // (fragment k + D); the last D fragments' acks are dead (the next message
+          // starts after "consumed", op_done) -- skipping them shortens a short message
+          q_pub[b] = X.role == 0 || (A.flags & 64) || (int64_t)it.k + it.D < it.K;
           mbar_arrive(full + b);  // piece i_acq may be copied (the arrive releases the acquire)
           i_acq++;
           more = it.next();
