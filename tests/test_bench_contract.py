@@ -23,6 +23,7 @@ def test_reference_arm_json_line():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
     assert "workload" in d["config"]
+    assert (d["steps"], d["warmup"]) == (1, 3)  # exactly the requested K timed / W warm-up steps
 
 
 def test_reference_arm_nonzero_rank_is_silent():
