@@ -151,16 +151,20 @@ def test_truncation_detected(torch_cuda):
     comm.free()
 
 
-@pytest.mark.parametrize("ring", [True, False], ids=["ring", "fused"])
+@pytest.mark.parametrize("ring", [True, False, "ce"], ids=["ring", "fused", "ce"])
 def test_loopback_halo_all_faces(torch_cuda, ring):
-    """1-rank periodic halo: the 12 transfers of one exchange in one group."""
+    """1-rank periodic halo: the 12 transfers of one exchange in one group (through the
+    ring kernel, the fused copy, or the copy-engine mode)."""
     import torch
 
     from paper_conf_hpdc_wubvjd16_b200 import dt
     from paper_conf_hpdc_wubvjd16_b200.halo import FACES, face_box, make_plan
     n, h = 64, 1
     L = n + 2 * h
-    comm = dt.Comm(0, 1, 0, chunk_bytes=16 << 10, depth=2, ring_loopback=ring)
+    if ring == "ce":
+        comm = dt.Comm(0, 1, 0, chunk_bytes=16 << 10, depth=2, mode=dt.XFER_CE)
+    else:
+        comm = dt.Comm(0, 1, 0, chunk_bytes=16 << 10, depth=2, ring_loopback=ring)
     plan = make_plan(0, n, h, dims=(1, 1, 1))
     A = np.full((L, L, L), 0xA5A5A5A5, dtype=np.uint32)
     z, y, x = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
