@@ -231,6 +231,20 @@ def test_resume_overlapping_instances(torch_cuda, extent):
             check_or_overlap(torch_cuda, rec, 16, 16 + count * 64 + 64, count, pos=pos, nbytes=nbytes)
 
 
+@pytest.mark.parametrize("nbytes", [16, 4096, (1 << 20) + 16, 64 << 20])
+def test_contiguous_run_copy(torch_cuda, nbytes):
+    """A contiguous layout (one run after normalisation) moves with the grid-stride run
+    copy when the run, the packed side and the length are 16-byte aligned, else with the
+    warp-slice kernel: whole streams, 16-aligned and misaligned fragments, count > 1."""
+    rec = ("contiguous", nbytes // 8, ("basic", "DOUBLE"))
+    check_pack_unpack(torch_cuda, rec, 0, nbytes)
+    check_pack_unpack(torch_cuda, rec, 16, nbytes, origin_pad=16)
+    if nbytes >= 4096:
+        check_pack_unpack(torch_cuda, rec, 0, nbytes, pos=32, nbytes=nbytes // 2)
+        check_pack_unpack(torch_cuda, rec, 0, nbytes, pos=8, nbytes=nbytes // 2 + 8)
+    check_pack_unpack(torch_cuda, rec, 0, nbytes, count=3)
+
+
 def test_unpack_rejects_overlap(torch_cuda):
     import torch
     from paper_conf_hpdc_wubvjd16_b200 import dt
