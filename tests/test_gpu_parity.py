@@ -231,6 +231,19 @@ def test_resume_overlapping_instances(torch_cuda, extent):
             check_or_overlap(torch_cuda, rec, 16, 16 + count * 64 + 64, count, pos=pos, nbytes=nbytes)
 
 
+@pytest.mark.parametrize("slice_", ["2048", "16384"])
+def test_warp_segments_multi_wave(torch_cuda, slice_, monkeypatch):
+    """The long-run kernel with fixed slices (several waves of short CTAs, as for streams of
+    more than 128 KiB per warp of one wave): triangles, a block-cyclic vector and a skewed
+    indexed list, whole streams, counts 2 and ragged fragments."""
+    monkeypatch.setenv("DT_SEG_SLICE", slice_)
+    for rec, org, parent in (c2_lower_triangle(700), stair_triangle(640, 64), c1_submatrix(300, 700, 3, 5)):
+        size = oracle.from_recipe(rec).size
+        check_pack_unpack(torch_cuda, rec, org, parent)
+        check_pack_unpack(torch_cuda, rec, org, parent, count=2, pos=8, nbytes=2 * size - 24)
+        check_pack_unpack(torch_cuda, rec, org, parent, pos=4096 + 8, nbytes=size // 3)
+
+
 @pytest.mark.parametrize("nbytes", [16, 4096, (1 << 20) + 16, 64 << 20])
 def test_contiguous_run_copy(torch_cuda, nbytes):
     """A contiguous layout (one run after normalisation) moves with the grid-stride run
