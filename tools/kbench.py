@@ -33,7 +33,7 @@ def main():
         "C2": lambda: W.c2_lower_triangle(), "C3": lambda: W.c3_block_cyclic(),
         "C4x": lambda: W.c4_face("x-"), "C4y": lambda: W.c4_face("y-"), "C4z": lambda: W.c4_face("z-"),
         "C5_64M": lambda: W.c5_particles(64 << 20), "C5_1G": lambda: W.c5_particles(1 << 30),
-        "C5b_64M": lambda: W.c5b_irregular(64 << 20),
+        "C5b_64M": lambda: W.c5b_irregular(64 << 20), "C5b_1G": lambda: W.c5b_irregular(1 << 30),
         "V4K": lambda: W.c1_submatrix(4096, 8192), "V8K": lambda: W.c1_submatrix(8192, 16384),
         "V16K": lambda: W.c1_submatrix(16384, 16384),
         "T16K": lambda: W.c2_lower_triangle(16384), "Tstair8K": lambda: W.stair_triangle(8192, 256),
