@@ -822,6 +822,7 @@ dt_status launch_pack_unpack(bool unpack, dt_type_s* t, const Form& f, DeviceDes
     const int occ = seg_occupancy(unpack, true);
     const int64_t max_warps = (int64_t)sms * occ * 8;
     int64_t per = std::max<int64_t>(1024, (len + max_warps - 1) / max_warps);
+    if (per > (int64_t(128) << 10)) per = 16384;  // long streams: several waves of 16 KiB slices (as k_seg)
     per = (per + 15) & ~int64_t(15);
     const int64_t nw = (len + per - 1) / per;
     const unsigned grid = (unsigned)((nw + 7) / 8);

@@ -244,6 +244,34 @@ def test_warp_segments_multi_wave(torch_cuda, slice_, monkeypatch):
         check_pack_unpack(torch_cuda, rec, org, parent, pos=4096 + 8, nbytes=size // 3)
 
 
+def test_full_size_sampled_long_vector(torch_cuda):
+    """A 512 MiB column sub-matrix (V8K: 8192 columns of 64 KiB at a 128 KiB pitch) -- long
+    enough for the multi-wave 16 KiB slices of the single-block kernel: 200k sampled stream
+    bytes against the vector's closed form (stream byte p = column p // 64 KiB, byte
+    p % 64 KiB), then unpack -> pack round trip."""
+    import torch
+    from paper_conf_hpdc_wubvjd16_b200 import dt
+    rec, org, parent = c1_submatrix(8192, 16384)
+    t = dt.from_recipe(rec).commit()
+    n = t.size
+    assert n == 8192 * 8192 * 8
+    src = torch.empty(parent, dtype=torch.uint8, device="cuda").random_(0, 256)
+    out = torch.empty(n, dtype=torch.uint8, device="cuda")
+    dt.pack(t, 1, src, out, origin_offset=org)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(8)
+    ps = np.unique(np.concatenate([rng.integers(0, n, size=200000), [0, n - 1]]))
+    addr = (ps // 65536) * (16384 * 8) + ps % 65536 + org
+    pt = torch.from_numpy(ps).cuda()
+    assert torch.equal(out[pt], src[torch.from_numpy(addr).cuda()])
+    dst = torch.zeros_like(src)
+    dt.unpack(t, 1, out, dst, origin_offset=org)
+    back = torch.empty_like(out)
+    dt.pack(t, 1, dst, back, origin_offset=org)
+    torch.cuda.synchronize()
+    assert torch.equal(back, out)
+
+
 @pytest.mark.parametrize("nbytes", [16, 4096, (1 << 20) + 16, 64 << 20])
 def test_contiguous_run_copy(torch_cuda, nbytes):
     """A contiguous layout (one run after normalisation) moves with the grid-stride run
